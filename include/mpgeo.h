@@ -1,0 +1,234 @@
+/*
+ * mpgeo.h — C ABI of the B200-native mixed-precision tile-Cholesky Matérn
+ * log-likelihood library (libmpgeo.so).
+ *
+ * Method: Cao, Abdulah, Ltaief, Genton, Keyes, Bosilca, "Reducing Data Motion
+ * and Energy Consumption of Geospatial Modeling Applications Using Automated
+ * Precision Conversion", IEEE CLUSTER 2023.  Citations "P:<line>" refer to
+ * lines of the paper text and the section/equation/algorithm they
+ * fall in.
+ *
+ * One evaluation of the Gaussian log-likelihood (Eq. (1), §III-A)
+ *     l(theta) = -(n/2) log(2 pi) - 1/2 log|Sigma(theta)| - 1/2 Z^T Sigma(theta)^{-1} Z
+ * for the 2D Matérn covariance (§III-A) is the sequence
+ *     mp_matern_gen (pass 1: tile norms)  ->  mp_precision_map  ->
+ *     mp_matern_gen (pass 2: tiles in storage precision)  ->  mp_tile_potrf  ->  mp_loglik
+ * or the single call mp_eval, which runs that sequence.
+ *
+ * Conventions (all entry points):
+ *  - Every function returns mp_status; MP_OK = 0.  No C++ exception crosses the
+ *    ABI.  mp_last_error(h) describes the last failure on a handle.
+ *  - Device pointers ("d_" prefix) are borrowed: the caller (PyTorch in the
+ *    Python binding) allocates and frees them.  Host pointers ("h_" or plain)
+ *    are read or written only during the call.
+ *  - Work is enqueued on the CUDA stream given to mp_init.  Calls that return
+ *    host results (norms, info, scalars) synchronise that stream before return.
+ *  - Tiles: square nb x nb, NT = ceil(n / nb); tile (m, k) covers rows
+ *    [m nb, min(n, (m+1) nb)) and columns [k nb, min(n, (k+1) nb)) (P:258,
+ *    "tile size 2048").  Only the lower triangle m >= k exists.  The ragged
+ *    last tile is padded in storage to nb x nb: identity on the diagonal pad,
+ *    zeros elsewhere (reading C18), which leaves l unchanged.
+ *  - NT x NT host maps (uint8) and the tile-norm array (double) are ROW-major
+ *    with index m * NT + k, lower triangle (m >= k) meaningful; other entries
+ *    are ignored on input and set to 255 (maps) / 0 (norms) on output.
+ *  - Precision codes: MP_FP64 = 0, MP_FP32 = 1, MP_FP16 = 2 (smaller = higher).
+ *    MP_FP16 is the paper's FP16_32 class: FP16 operands, FP32 accumulation,
+ *    FP32 storage.
+ *  - Multi-GPU: one process (and one handle) per GPU, P x Q process grid with
+ *    P <= Q, 2D block-cyclic tile ownership
+ *    owner(m, k) = (m mod P) * Q + (k mod Q).  Results returned to the host
+ *    are identical on every rank.
+ *  - Threading: a handle is not thread-safe; use one handle per thread.
+ */
+#ifndef MPGEO_H
+#define MPGEO_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef enum {
+    MP_OK = 0,
+    MP_ERR_ARG = 1,          /* invalid argument: sizes, theta <= 0, nu outside (0, 20], bad map */
+    MP_ERR_NOT_SPD = 2,      /* POTRF met a non-positive pivot; see `info` of mp_tile_potrf */
+    MP_ERR_CUDA = 3,         /* a CUDA call failed; the handle is unusable afterwards */
+    MP_ERR_NCCL = 4,         /* an NCCL call failed; the handle is unusable afterwards */
+    MP_ERR_NOMEM = 5,        /* workspace too small for the requested layout */
+    MP_ERR_UNSUPPORTED = 6,  /* configuration this build does not implement */
+    MP_ERR_STATE = 7         /* call order violated (e.g. potrf before generation) */
+} mp_status;
+
+typedef enum { MP_FP64 = 0, MP_FP32 = 1, MP_FP16 = 2 } mp_prec;
+
+/* Communication-precision policy.
+ * MP_COMM_TTC : target-task conversion — every tile travels in its storage
+ *               precision and each consumer converts (the pre-existing scheme).
+ * MP_COMM_AUTO: Algorithm 2 — sender-side conversion (STC) where all
+ *               successors run at lower precision, TTC otherwise. */
+typedef enum { MP_COMM_TTC = 0, MP_COMM_AUTO = 1 } mp_comm_policy;
+
+/* How mp_eval chooses the kernel-precision map. */
+typedef enum {
+    MP_MAP_ADAPTIVE = 0,  /* tile-norm rule of P:117 at u_req (the paper's method) */
+    MP_MAP_FP64 = 1,      /* everything FP64 (the "same code forced to all-FP64" baseline) */
+    MP_MAP_BAND = 2,      /* FP64 band / FP32 outside (config 2; reading C21) */
+    MP_MAP_EXTREME = 3,   /* FP64 diagonal, FP16 elsewhere (performance-only) */
+    MP_MAP_USER = 4       /* kernel_prec supplied by the caller */
+} mp_map_mode;
+
+typedef struct mp_handle mp_handle;
+typedef struct mp_matrix mp_matrix;
+
+/* Per-evaluation report filled by mp_eval. Times are device times (CUDA events on
+ * the handle's stream) in milliseconds; flops are algorithmic counts. */
+typedef struct {
+    double loglik, logdet, quad;
+    int64_t info;                 /* 0, or first non-positive pivot column (1-based) */
+    double t_gen_ms, t_map_ms, t_potrf_ms, t_solve_ms, t_total_ms;
+    double flops_potrf;           /* n^3/3 convention is left to the caller; this is the
+                                     tile count: sum over executed kernels at nb^3 units */
+    double flops_update[3];       /* GEMM+SYRK flops executed per precision class */
+    int64_t tiles[3];             /* lower off-diagonal tiles per kernel precision */
+    int64_t stc_tiles;            /* off-diagonal tiles whose comm precision < storage */
+    int64_t gpu_launches;         /* kernels launched by this call */
+} mp_eval_report;
+
+/* ---------------------------------------------------------------- lifecycle */
+
+/* NCCL unique id for multi-GPU handles (rank 0 calls it and broadcasts the 128
+ * bytes, e.g. with torch.distributed).  Unused when nranks == 1. */
+mp_status mp_get_unique_id(uint8_t id[128]);
+
+/* Create a handle on CUDA `device` for `rank` of `nranks` (P * Q == nranks,
+ * P <= Q).  `id` may be NULL when nranks == 1.  `cuda_stream` is a cudaStream_t
+ * (NULL = a stream created and owned by the handle).  *h receives the handle. */
+mp_status mp_init(int device, int rank, int nranks, int P, int Q, const uint8_t* id,
+                  void* cuda_stream, mp_handle** h);
+mp_status mp_finalize(mp_handle* h);
+const char* mp_last_error(const mp_handle* h);
+
+/* ---------------------------------------------------------------- matrices */
+
+/* Geometry and ownership of an n x n symmetric tile matrix with tile size nb
+ * (nb % 16 == 0, 16 <= nb <= 8192, n >= 1).  No device memory is touched. */
+mp_status mp_matrix_create(mp_handle* h, int64_t n, int nb, mp_matrix** A);
+mp_status mp_matrix_destroy(mp_matrix* A);
+
+/* Device bytes needed to bind A with the given storage map (NULL = all FP64, the
+ * worst case): owned tiles in storage precision, the FP64 panel buffer and the
+ * low-precision panel caches (K2), communication staging, solve scratch. */
+mp_status mp_matrix_bytes(const mp_matrix* A, const uint8_t* storage_prec, size_t* bytes);
+
+/* Lay out A inside the caller's device workspace (256-byte aligned) for the
+ * storage map (NULL = all FP64).  May be called again with a new map on the
+ * same workspace (each MLE evaluation has its own map); contents are lost. */
+mp_status mp_matrix_bind(mp_matrix* A, const uint8_t* storage_prec, void* d_workspace, size_t bytes);
+
+/* ---------------------------------------------------------------- the path */
+
+/* (1) Matérn tile generation, P:82 (covariance), P:117 (tile norms)
+ * (tiles generated directly in their storage precision).
+ * theta = {sigma^2, beta, nu}; C(0) = sigma^2 (reading C3); h Euclidean (C5).
+ * d_x, d_y: device FP64 [n] locations (replicated on every rank).
+ * Pass 1 — storage_prec == NULL: computes s_mk = ||A_mk||_F^2 over real
+ *   (unpadded) entries for every lower tile and writes them to the host array
+ *   tile_sqnorm[NT*NT] (all-reduced over ranks, identical everywhere).  A must
+ *   be bound (any map; the partial sums live in the workspace).  Deterministic
+ *   (fixed reduction order).
+ * Pass 2 — storage_prec != NULL (the map A is bound with): writes every owned
+ *   tile in its storage precision (FP64 or FP32, round-to-nearest-even) and
+ *   the padding; tile_sqnorm may be NULL. */
+mp_status mp_matern_gen(mp_handle* h, mp_matrix* A, const double* d_x, const double* d_y,
+                        const double theta[3], const uint8_t* storage_prec, double* tile_sqnorm);
+
+/* (2) Precision maps — pure host, deterministic, no GPU (P:117, P:146, P:152,
+ * Algorithm 2; readings C6, C7, C10, C11 in DESIGN.md).
+ *   S = sum_k s_kk + 2 sum_{m>k} s_mk (each sum correctly rounded);
+ *   kernel(k,k) = FP64; off-diagonal r = sqrt(s_mk) * NT / sqrt(S) and
+ *   kernel = FP16 if r <= u_req/eps[2], else FP32 if r <= u_req/eps[1], else FP64;
+ *   storage = FP64 if kernel is FP64 else FP32;
+ *   comm per `policy` (TTC: storage, diagonal FP64; AUTO: Algorithm 2).
+ * eps may be NULL (= {2^-52, 2^-23, 2^-10}).  Any output pointer may be NULL.
+ * If tile_sqnorm is NULL, kernel_prec is an INPUT (a user map) and only the
+ * storage and comm maps are derived from it. */
+mp_status mp_precision_map(int nt, const double* tile_sqnorm, double u_req, const double* eps,
+                           mp_comm_policy policy, uint8_t* kernel_prec, uint8_t* storage_prec,
+                           uint8_t* comm_prec);
+
+/* (3) In-place mixed-precision tile Cholesky A = L L^T (Algorithm 1):
+ * DPOTRF (FP64) on diagonal tiles; TRSM(m,k) with L_kk received at
+ * comm(k,k) (FP64 arithmetic, result rounded to storage(m,k)); L_mk reaches its
+ * successors at comm(m,k) and is converted on the consuming GPU to the
+ * successor's kernel precision; DSYRK in FP64; GEMM(m,n,k) at
+ * kernel(m,n): FP64 on DMMA tensor cores, FP32 class as 3xTF32 and FP16 class
+ * as FP16xFP16->FP32 on tcgen05 tensor cores, accumulating into the FP32 tile.
+ * kernel_prec / comm_prec: host maps (NT*NT, as produced by mp_precision_map
+ * and consistent with the storage map A is bound with).  Blocking.
+ * *info = 0 on success, else the 1-based global column of the first
+ * non-positive pivot (LAPACK convention) and MP_ERR_NOT_SPD is returned. */
+mp_status mp_tile_potrf(mp_handle* h, mp_matrix* A, const uint8_t* kernel_prec,
+                        const uint8_t* comm_prec, int64_t* info);
+
+/* (4) Eq. (1) from the factor: log|Sigma| = 2 sum log L_ii (FP64 diagonal
+ * tiles), y = L^{-1} Z by tile forward substitution reading L in storage
+ * precision with FP64 arithmetic (reading C15), quad = y^T y,
+ * l = -(n/2) log(2 pi) - logdet/2 - quad/2.  d_z: device FP64 [n].  Blocking. */
+mp_status mp_loglik(mp_handle* h, const mp_matrix* L, const double* d_z,
+                    double* loglik, double* logdet, double* quad);
+
+/* One whole evaluation (the call a user makes): (1) pass 1, (2), (1) pass 2,
+ * (3), (4).  x, y, z are FP64 [n]; if `inputs_on_host` is nonzero they are host
+ * pointers and are copied to the device inside the call (pinned memory makes
+ * the copy asynchronous), else device pointers.  A must be bound to a
+ * workspace sized for the worst case (mp_matrix_bytes with NULL); it is
+ * re-bound to the evaluation's storage map.  `mode` picks the kernel map
+ * (`user_kernel_prec` is read only for MP_MAP_USER).  Out: report.
+ * Returns MP_ERR_NOT_SPD (report->info set, loglik = -inf) for a non-SPD Sigma. */
+mp_status mp_eval(mp_handle* h, mp_matrix* A, const double* x, const double* y, const double* z,
+                  int inputs_on_host, const double theta[3], double u_req, const double* eps,
+                  mp_comm_policy policy, mp_map_mode mode, const uint8_t* user_kernel_prec,
+                  mp_eval_report* report);
+
+/* Maps used by the last mp_eval on A (host NT*NT arrays; any may be NULL). */
+mp_status mp_matrix_maps(const mp_matrix* A, uint8_t* kernel_prec, uint8_t* storage_prec,
+                         uint8_t* comm_prec);
+
+/* Copy owned tile (m, k) of A to host as FP64 nb x nb row-major (padding
+ * included), for tests.  Returns MP_ERR_ARG if (m, k) is not owned here. */
+mp_status mp_matrix_get_tile(mp_handle* h, const mp_matrix* A, int m, int k, double* h_tile);
+
+/* Overwrite owned tile (m, k) of a bound A from host FP64 nb x nb row-major data (padding
+ * included), rounding to the tile's storage precision; marks A as generated.  Lets a caller
+ * factor a matrix of its own instead of the Matérn covariance. */
+mp_status mp_matrix_set_tile(mp_handle* h, mp_matrix* A, int m, int k, const double* h_tile);
+
+/* Number of tiles per dimension and whether tile (m, k) is owned by this rank. */
+int mp_matrix_nt(const mp_matrix* A);
+int mp_matrix_owner(const mp_matrix* A, int m, int k);
+
+/* Per-kernel-class device time accounting (CUDA events recorded on the handle's stream around
+ * every launch of the class; enable before the region to measure, read after it).
+ * Classes: 0 FP64 trailing update (DMMA GEMM+SYRK), 1 FP32-class update, 2 FP16-class update,
+ * 3 POTRF (diagonal tiles), 4 TRSM, 5 conversion (K2), 6 generation (K1), 7 solve (K8). */
+#define MP_PROF_CLASSES 8
+typedef struct {
+    double ms[MP_PROF_CLASSES];      /* summed device time per class */
+    double flops[MP_PROF_CLASSES];   /* algorithmic flops per class (0 where not a flop count) */
+    int64_t launches[MP_PROF_CLASSES];
+} mp_profile;
+mp_status mp_set_profiling(mp_handle* h, int enable);  /* enable also resets the counters */
+mp_status mp_get_profile(mp_handle* h, mp_profile* out);  /* synchronises the stream */
+
+/* Total kernels launched on this handle since mp_init (for bench accounting). */
+int64_t mp_launch_count(const mp_handle* h);
+
+/* Library version string, e.g. "mpgeo 0.1 sm_100a". */
+const char* mp_version(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* MPGEO_H */

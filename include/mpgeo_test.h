@@ -1,0 +1,29 @@
+/*
+ * mpgeo_test.h — kernel-level test hooks of libmpgeo.so (C ABI, device pointers).
+ * Used only by tests/ to check single kernels against the oracle; not part of the path.
+ * All return mp_status (0 = OK) and synchronise the default stream.
+ */
+#ifndef MPGEO_TEST_H
+#define MPGEO_TEST_H
+#include "mpgeo.h"
+#ifdef __cplusplus
+extern "C" {
+#endif
+/* out[i] = K_nu(x[i]) (modified Bessel function of the second kind, device code of K1). */
+mp_status mp_test_bessel_k(double nu, const double* d_x, double* d_out, int n);
+/* One job of the K5 DMMA GEMM: C = beta*C + alpha*A*B^T (row-major, see kernels.h).
+ * round: operand rounding class (0 FP64, 1 FP32, 2 FP16); c_f32: C is float. */
+mp_status mp_test_dgemm(const double* d_A, const double* d_B, void* d_C, int M, int N, int K, int lda, int ldb,
+                        int ldc, int lower, double alpha, double beta, int round, int c_f32);
+/* One job of the tcgen05 GEMMs: C (FP32 nb x nb) -= P_m P_n^T with P the panel cache
+ * [nt*nb][nb]: kind 1 = 3xTF32 (panel = hi, panel_lo = lo, float), kind 2 = FP16 (panel = half). */
+mp_status mp_test_tc_gemm(int kind, const void* d_panel, const void* d_panel_lo, float* d_C, int nb, int nt, int m,
+                          int n);
+/* 1 if the tcgen05 kernels are compiled in, else 0. */
+int mp_tc_available(void);
+/* Correctly rounded sum of n doubles (host; the S of the precision rule). */
+double mpgeo_exact_sum(const double* v, int64_t n);
+#ifdef __cplusplus
+}
+#endif
+#endif

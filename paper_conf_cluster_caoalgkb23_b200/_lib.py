@@ -1,0 +1,93 @@
+"""ctypes binding of libmpgeo.so (include/mpgeo.h): argument marshalling only.
+
+Every step of the path runs in the library's CUDA kernels; nothing here computes.
+If the shared library is missing this module raises at import — there is no CPU
+fallback (the CPU oracle under oracle/ is test infrastructure, never imported here).
+"""
+from __future__ import annotations
+
+import ctypes as C
+import os
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(_HERE, "libmpgeo.so")
+
+MP_OK, MP_ERR_ARG, MP_ERR_NOT_SPD, MP_ERR_CUDA, MP_ERR_NCCL, MP_ERR_NOMEM, MP_ERR_UNSUPPORTED, MP_ERR_STATE = range(8)
+STATUS_NAMES = ["MP_OK", "MP_ERR_ARG", "MP_ERR_NOT_SPD", "MP_ERR_CUDA", "MP_ERR_NCCL", "MP_ERR_NOMEM",
+                "MP_ERR_UNSUPPORTED", "MP_ERR_STATE"]
+MP_FP64, MP_FP32, MP_FP16 = 0, 1, 2
+MP_COMM_TTC, MP_COMM_AUTO = 0, 1
+MP_MAP_ADAPTIVE, MP_MAP_FP64, MP_MAP_BAND, MP_MAP_EXTREME, MP_MAP_USER = range(5)
+
+
+class EvalReport(C.Structure):
+    _fields_ = [
+        ("loglik", C.c_double), ("logdet", C.c_double), ("quad", C.c_double),
+        ("info", C.c_int64),
+        ("t_gen_ms", C.c_double), ("t_map_ms", C.c_double), ("t_potrf_ms", C.c_double),
+        ("t_solve_ms", C.c_double), ("t_total_ms", C.c_double),
+        ("flops_potrf", C.c_double), ("flops_update", C.c_double * 3),
+        ("tiles", C.c_int64 * 3), ("stc_tiles", C.c_int64), ("gpu_launches", C.c_int64),
+    ]
+
+
+PROF_CLASSES = ["upd_fp64", "upd_fp32", "upd_fp16", "potrf", "trsm", "convert", "generate", "solve"]
+
+
+class Profile(C.Structure):
+    _fields_ = [("ms", C.c_double * 8), ("flops", C.c_double * 8), ("launches", C.c_int64 * 8)]
+
+    def as_dict(self):
+        return {name: {"ms": self.ms[i], "flops": self.flops[i], "launches": int(self.launches[i])}
+                for i, name in enumerate(PROF_CLASSES)}
+
+
+class MpError(RuntimeError):
+    def __init__(self, status: int, msg: str):
+        super().__init__(f"{STATUS_NAMES[status] if 0 <= status < len(STATUS_NAMES) else status}: {msg}")
+        self.status = status
+
+
+def _load() -> C.CDLL:
+    if not os.path.exists(LIB_PATH):
+        raise ImportError(f"{LIB_PATH} is missing: run __graft_entry__.build() (make -C {_HERE}); "
+                          "there is no CPU fallback")
+    lib = C.CDLL(LIB_PATH, mode=C.RTLD_GLOBAL)
+    vp, i32, i64, dbl, u8p, dp = C.c_void_p, C.c_int, C.c_int64, C.c_double, C.POINTER(C.c_uint8), C.POINTER(C.c_double)
+    sig = {
+        "mp_get_unique_id": (i32, [u8p]),
+        "mp_init": (i32, [i32, i32, i32, i32, i32, u8p, vp, C.POINTER(vp)]),
+        "mp_finalize": (i32, [vp]),
+        "mp_last_error": (C.c_char_p, [vp]),
+        "mp_matrix_create": (i32, [vp, i64, i32, C.POINTER(vp)]),
+        "mp_matrix_destroy": (i32, [vp]),
+        "mp_matrix_bytes": (i32, [vp, u8p, C.POINTER(C.c_size_t)]),
+        "mp_matrix_bind": (i32, [vp, u8p, vp, C.c_size_t]),
+        "mp_matern_gen": (i32, [vp, vp, vp, vp, dp, u8p, dp]),
+        "mp_precision_map": (i32, [i32, dp, dbl, dp, i32, u8p, u8p, u8p]),
+        "mp_tile_potrf": (i32, [vp, vp, u8p, u8p, C.POINTER(i64)]),
+        "mp_loglik": (i32, [vp, vp, vp, dp, dp, dp]),
+        "mp_eval": (i32, [vp, vp, vp, vp, vp, i32, dp, dbl, dp, i32, i32, u8p, C.POINTER(EvalReport)]),
+        "mp_matrix_maps": (i32, [vp, u8p, u8p, u8p]),
+        "mp_matrix_get_tile": (i32, [vp, vp, i32, i32, dp]),
+        "mp_matrix_set_tile": (i32, [vp, vp, i32, i32, dp]),
+        "mp_matrix_nt": (i32, [vp]),
+        "mp_matrix_owner": (i32, [vp, i32, i32]),
+        "mp_launch_count": (i64, [vp]),
+        "mp_set_profiling": (i32, [vp, i32]),
+        "mp_get_profile": (i32, [vp, C.POINTER(Profile)]),
+        "mp_version": (C.c_char_p, []),
+        "mpgeo_exact_sum": (dbl, [dp, i64]),
+        "mp_test_bessel_k": (i32, [dbl, vp, vp, i32]),
+        "mp_test_dgemm": (i32, [vp, vp, vp, i32, i32, i32, i32, i32, i32, i32, dbl, dbl, i32, i32]),
+        "mp_test_tc_gemm": (i32, [i32, vp, vp, vp, i32, i32, i32, i32]),
+        "mp_tc_available": (i32, []),
+    }
+    for name, (res, args) in sig.items():
+        f = getattr(lib, name)
+        f.restype = res
+        f.argtypes = args
+    return lib
+
+
+lib = _load()

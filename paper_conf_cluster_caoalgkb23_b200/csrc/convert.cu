@@ -1,0 +1,106 @@
+// K2 — precision conversion of panel tiles.
+//
+// After TRSM(m, k) the tile L_mk exists once, in FP64, in the GPU's panel buffer.  panel_out
+//   * writes it back to the tile pool in its storage precision (the factor the solve reads),
+//   * rounds the panel copy to the communication precision comm(m, k) — what the successors
+//     receive (STC when comm < storage, TTC otherwise; Algorithm 2),
+//   * and derives, once per panel per GPU, the operand formats its consuming GEMMs need:
+//     FP16 (FP16-class successors) and the TF32 hi/lo pair (FP32-class successors, 3xTF32).
+// Consumers therefore convert on the GPU they run on (target-side conversion), but at
+// most once per tile instead of once per GEMM.  All kernels are elementwise, 16-byte
+// vectorised and HBM-bound.
+#include "common.cuh"
+#include "kernels.h"
+
+namespace mpgeo {
+
+constexpr int CV_T = 256;
+
+__device__ __forceinline__ float tf32_rna(float x) {
+    uint32_t r;
+    asm("cvt.rna.tf32.f32 %0, %1;" : "=r"(r) : "f"(x));
+    return __uint_as_float(r);
+}
+
+__global__ void __launch_bounds__(CV_T) panel_in_kernel(const PanelTile* tiles, int64_t elems) {
+    const PanelTile t = tiles[blockIdx.y];
+    const int64_t stride = (int64_t)gridDim.x * CV_T * 2;
+    for (int64_t i = ((int64_t)blockIdx.x * CV_T + threadIdx.x) * 2; i < elems; i += stride) {
+        double2 v;
+        if (t.store_prec == P64) {
+            v = *(const double2*)((const double*)t.store + i);
+        } else {
+            const float2 f = *(const float2*)((const float*)t.store + i);
+            v = make_double2((double)f.x, (double)f.y);
+        }
+        *(double2*)(t.p64 + i) = v;
+    }
+}
+
+__global__ void __launch_bounds__(CV_T) panel_out_kernel(const PanelTile* tiles, int64_t elems) {
+    const PanelTile t = tiles[blockIdx.y];
+    const int64_t stride = (int64_t)gridDim.x * CV_T * 2;
+    for (int64_t i = ((int64_t)blockIdx.x * CV_T + threadIdx.x) * 2; i < elems; i += stride) {
+        const double2 v = *(const double2*)(t.p64 + i);
+        if (t.store_prec == P64) {
+            *(double2*)((double*)t.store + i) = v;
+        } else {
+            *(float2*)((float*)t.store + i) = make_float2(__double2float_rn(v.x), __double2float_rn(v.y));
+        }
+        const double w0 = round_to(v.x, t.comm_prec), w1 = round_to(v.y, t.comm_prec);
+        if (t.comm_prec != P64) *(double2*)(t.p64 + i) = make_double2(w0, w1);
+        if (t.p16) *(__half2*)(t.p16 + i) = __halves2half2(__double2half(w0), __double2half(w1));
+        if (t.hi) {
+            const float f0 = __double2float_rn(w0), f1 = __double2float_rn(w1);
+            const float h0 = tf32_rna(f0), h1 = tf32_rna(f1);
+            *(float2*)(t.hi + i) = make_float2(h0, h1);
+            *(float2*)(t.lo + i) = make_float2(tf32_rna(f0 - h0), tf32_rna(f1 - h1));
+        }
+    }
+}
+
+__global__ void round_copy_kernel(const double* src, double* dst, int64_t elems, int prec) {
+    const int64_t stride = (int64_t)gridDim.x * blockDim.x;
+    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < elems; i += stride)
+        dst[i] = round_to(src[i], prec);
+}
+
+__global__ void zero_upper_kernel(double* A, int nb) {
+    const int r = blockIdx.x;
+    for (int c = r + 1 + threadIdx.x; c < nb; c += blockDim.x) A[(size_t)r * nb + c] = 0.0;
+}
+
+static unsigned chunks_for(int64_t elems, int ntiles) {
+    // about 4 waves of 148 SMs in total, at least one chunk per tile
+    int64_t per = (4LL * 148 * 8 + ntiles - 1) / ntiles;
+    const int64_t maxc = (elems / 2 + CV_T - 1) / CV_T;
+    if (per > maxc) per = maxc;
+    if (per < 1) per = 1;
+    return (unsigned)per;
+}
+
+cudaError_t panel_in_launch(const PanelTile* t, int ntiles, int64_t elems, cudaStream_t s) {
+    if (ntiles <= 0) return cudaSuccess;
+    dim3 grid(chunks_for(elems, ntiles), ntiles);
+    panel_in_kernel<<<grid, CV_T, 0, s>>>(t, elems);
+    return cudaGetLastError();
+}
+
+cudaError_t panel_out_launch(const PanelTile* t, int ntiles, int64_t elems, cudaStream_t s) {
+    if (ntiles <= 0) return cudaSuccess;
+    dim3 grid(chunks_for(elems, ntiles), ntiles);
+    panel_out_kernel<<<grid, CV_T, 0, s>>>(t, elems);
+    return cudaGetLastError();
+}
+
+cudaError_t round_copy_launch(const double* src, double* dst, int64_t elems, int prec, cudaStream_t s) {
+    round_copy_kernel<<<592, 256, 0, s>>>(src, dst, elems, prec);
+    return cudaGetLastError();
+}
+
+cudaError_t zero_upper_launch(double* A, int nb, cudaStream_t s) {
+    zero_upper_kernel<<<nb, 256, 0, s>>>(A, nb);
+    return cudaGetLastError();
+}
+
+}  // namespace mpgeo

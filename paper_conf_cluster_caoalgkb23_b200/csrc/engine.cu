@@ -1,0 +1,874 @@
+// Host engine and C ABI of libmpgeo (include/mpgeo.h).
+//
+// The tile DAG of Algorithm 1 is executed as a static per-panel schedule on the
+// handle's CUDA stream: for panel k
+//   1. DPOTRF(k,k): blocked by 128 columns — diagonal block Cholesky + inverse (1 CTA), the
+//      block column as an in-place DMMA GEMM with the inverse, the trailing block SYRK;
+//   2. L~_kk = L_kk rounded to comm(k,k) (what the TRSMs receive, Alg. 2) + block inverses;
+//   3. panel in: the column's tiles (m,k), m > k, up-converted into the FP64 panel buffer;
+//   4. TRSM(m,k): blocked right-looking, two DMMA GEMMs per 128-column block, batched over m;
+//   5. panel out (K2): write back in storage precision, round to comm(m,k), derive the FP16 /
+//      TF32-pair operand copies for low-precision successors;
+//   6. trailing update: DSYRK(m,k) + GEMM(m,n,k) grouped by the kernel precision of the
+//      output tile: FP64 (DMMA), FP32 class and FP16 class.
+// Everything for one call is planned on the host first (job arrays for the batched kernels),
+// uploaded once into the control arena of the workspace, then enqueued.
+#include <dlfcn.h>
+
+#include <algorithm>
+#include <climits>
+#include <cmath>
+#include <cstdio>
+#include <cstring>
+#include <functional>
+#include <string>
+#include <vector>
+
+#include "../../include/mpgeo.h"
+#include "kernels.h"
+#include "tc_gemm.h"
+
+using namespace mpgeo;
+
+// ------------------------------------------------------------------ NCCL (loaded lazily)
+typedef struct { char internal[128]; } nccl_uid_t;
+typedef void* nccl_comm_t;
+struct NcclApi {
+    void* lib = nullptr;
+    int (*GetUniqueId)(nccl_uid_t*) = nullptr;
+    int (*CommInitRank)(nccl_comm_t*, int, nccl_uid_t, int) = nullptr;
+    int (*CommDestroy)(nccl_comm_t) = nullptr;
+    bool load() {
+        if (lib) return true;
+        lib = dlopen("libnccl.so.2", RTLD_NOW | RTLD_GLOBAL);
+        if (!lib) return false;
+        GetUniqueId = (int (*)(nccl_uid_t*))dlsym(lib, "ncclGetUniqueId");
+        CommInitRank = (int (*)(nccl_comm_t*, int, nccl_uid_t, int))dlsym(lib, "ncclCommInitRank");
+        CommDestroy = (int (*)(nccl_comm_t))dlsym(lib, "ncclCommDestroy");
+        return GetUniqueId && CommInitRank && CommDestroy;
+    }
+};
+static NcclApi g_nccl;
+
+// ------------------------------------------------------------------ objects
+struct ProfRec {
+    cudaEvent_t e0, e1;
+    int cls;
+    double flops;
+};
+struct mp_handle {
+    int device = 0, rank = 0, nranks = 1, P = 1, Q = 1;
+    cudaStream_t stream = nullptr;
+    bool own_stream = false;
+    nccl_comm_t nccl = nullptr;
+    std::string err;
+    int64_t launches = 0;
+    int* d_info = nullptr;
+    cudaEvent_t ev[8] = {};
+    bool broken = false;
+    int tc_mode = 1;  // 1: tcgen05 kernels for FP32/FP16 classes when available, 0: DMMA emulation
+    // profiling (mp_set_profiling): event pairs per launch, resolved in mp_get_profile
+    bool profiling = false;
+    std::vector<cudaEvent_t> prof_pool;
+    size_t prof_free = 0;
+    std::vector<ProfRec> prof_pending;
+    mp_profile prof = {};
+};
+
+struct Regions {
+    size_t total = 0;
+    size_t inputs = 0, p64 = 0, p16 = 0, phi = 0, plo = 0, ltilde = 0, wbuf = 0, wbuf2 = 0;
+    size_t vec_r = 0, vec_y = 0, partials = 0, norms = 0, ctrl = 0, ctrl_bytes = 0;
+    std::vector<size_t> tile_off;  // per (m*nt+k), SIZE_MAX if not stored here
+};
+
+struct mp_matrix {
+    mp_handle* h = nullptr;
+    int64_t n = 0;
+    int nb = 0, nt = 0;
+    char* ws = nullptr;
+    size_t ws_bytes = 0;
+    bool bound = false, generated = false, factored = false;
+    std::vector<uint8_t> storage, kmap, cmap;
+    Regions R;
+    int owner(int m, int k) const { return (m % h->P) * h->Q + (k % h->Q); }
+    bool mine(int m, int k) const { return h->nranks == 1 || owner(m, k) == h->rank; }
+    size_t nb2() const { return (size_t)nb * nb; }
+    void* tile(int m, int k) const { return ws + R.tile_off[(size_t)m * nt + k]; }
+    uint8_t st(int m, int k) const { return storage[(size_t)m * nt + k]; }
+    template <class T>
+    T* at(size_t off) const { return (T*)(ws + off); }
+};
+
+#define FAIL(h, code, ...)                                            \
+    do {                                                              \
+        char _b[512];                                                 \
+        snprintf(_b, sizeof _b, __VA_ARGS__);                         \
+        if (h) (h)->err = _b;                                         \
+        return code;                                                  \
+    } while (0)
+#define CK(h, x)                                                                          \
+    do {                                                                                  \
+        cudaError_t _e = (x);                                                             \
+        if (_e != cudaSuccess) {                                                          \
+            if (h) (h)->broken = true;                                                    \
+            FAIL(h, MP_ERR_CUDA, "%s failed: %s (%s:%d)", #x, cudaGetErrorString(_e), __FILE__, __LINE__); \
+        }                                                                                 \
+    } while (0)
+
+static size_t align_up(size_t v, size_t a) { return (v + a - 1) / a * a; }
+static int ceil_div(int a, int b) { return (a + b - 1) / b; }
+
+// Upper bound of control-arena bytes for one call on an nt x nt tile matrix.
+static size_t ctrl_bytes_for(int nt, int nb) {
+    const size_t T = nt;
+    const size_t nblk = ceil_div(nb, POTRF_IB);
+    size_t jobs = T * (T + 1) * (T + 2) / 6 + T + 2 * nblk * T + 2 * nblk * T * T;
+    size_t bytes = jobs * sizeof(GemmJob);
+    bytes += T * T * sizeof(PanelTile) * 2;
+    bytes += T * (T + 1) / 2 * sizeof(GenTile);
+    bytes += T * T * sizeof(GemvTile);
+    bytes += T * (sizeof(double*) + sizeof(int));
+    bytes += 64 * 1024 + 32 * 256;  // alignment slack
+    return bytes;
+}
+
+static Regions layout(const mp_matrix* A, const uint8_t* storage) {
+    // Map-independent regions first (their offsets depend only on n, nb, NT), then the tile
+    // pool, whose slots depend on the storage map (re-laid out per evaluation).
+    Regions R;
+    const int nt = A->nt;
+    const size_t nb2 = A->nb2();
+    size_t off = 0;
+    auto take = [&](size_t bytes) {
+        off = align_up(off, 256);
+        const size_t o = off;
+        off += bytes;
+        return o;
+    };
+    const size_t nvec = (size_t)nt * A->nb;
+    R.inputs = take(3 * nvec * 8);
+    R.vec_r = take(nvec * 8);
+    R.vec_y = take(nvec * 8);
+    const size_t ntl = (size_t)nt * (nt + 1) / 2;
+    R.partials = take(std::max(ntl * (A->nb / GEN_ROWS), (size_t)2 * nt + nvec / 4096 + 64) * 8);
+    R.norms = take(std::max(ntl, (size_t)nt * 4 + 64) * 8);
+    R.ctrl_bytes = ctrl_bytes_for(nt, A->nb);
+    R.ctrl = take(R.ctrl_bytes);
+    R.ltilde = take(nb2 * 8);
+    R.wbuf = take((size_t)POTRF_IB * POTRF_IB * 8);
+    R.wbuf2 = take((size_t)ceil_div(A->nb, POTRF_IB) * POTRF_IB * POTRF_IB * 8);
+    R.p64 = take((size_t)nt * nb2 * 8);
+    R.p16 = take((size_t)nt * nb2 * 2);
+    R.phi = take((size_t)nt * nb2 * 4);
+    R.plo = take((size_t)nt * nb2 * 4);
+    R.tile_off.assign((size_t)nt * nt, SIZE_MAX);
+    for (int k = 0; k < nt; ++k)
+        for (int m = k; m < nt; ++m)
+            if (A->mine(m, k)) {
+                const uint8_t p = storage ? storage[(size_t)m * nt + k] : (uint8_t)MP_FP64;
+                R.tile_off[(size_t)m * nt + k] = take(nb2 * (p == MP_FP64 ? 8 : 4));
+            }
+    R.total = align_up(off, 256);
+    return R;
+}
+
+// Control arena: host staging of job / descriptor arrays, uploaded in one copy.
+struct Arena {
+    std::vector<char> host;
+    char* dev_base = nullptr;
+    size_t cap = 0;
+    template <class T>
+    T* push(const T* items, size_t n) {  // returns the device address of the copy
+        size_t off = align_up(host.size(), 16);
+        host.resize(off + n * sizeof(T));
+        if (n) memcpy(host.data() + off, items, n * sizeof(T));
+        return (T*)(dev_base + off);
+    }
+    template <class T>
+    T* push(const std::vector<T>& v) { return push(v.data(), v.size()); }
+};
+
+// One enqueued kernel: launcher, profiling class (mp_profile) and its algorithmic flops.
+struct Op {
+    std::function<cudaError_t(cudaStream_t)> fn;
+    int cls;
+    double flops;
+};
+enum { C_UPD64 = 0, C_UPD32 = 1, C_UPD16 = 2, C_POTRF = 3, C_TRSM = 4, C_CONV = 5, C_GEN = 6, C_SOLVE = 7 };
+
+static cudaEvent_t prof_event(mp_handle* h) {
+    if (h->prof_free < h->prof_pool.size()) return h->prof_pool[h->prof_free++];
+    cudaEvent_t e = nullptr;
+    cudaEventCreate(&e);
+    h->prof_pool.push_back(e);
+    h->prof_free++;
+    return e;
+}
+
+static mp_status run_plan(mp_handle* h, mp_matrix* A, Arena& ar, std::vector<Op>& ops) {
+    if (ar.host.size() > A->R.ctrl_bytes)
+        FAIL(h, MP_ERR_NOMEM, "control arena overflow (%zu > %zu)", ar.host.size(), A->R.ctrl_bytes);
+    if (!ar.host.empty())
+        CK(h, cudaMemcpyAsync(ar.dev_base, ar.host.data(), ar.host.size(), cudaMemcpyHostToDevice, h->stream));
+    for (auto& op : ops) {
+        if (h->profiling) {
+            cudaEvent_t e0 = prof_event(h), e1 = prof_event(h);
+            CK(h, cudaEventRecord(e0, h->stream));
+            CK(h, op.fn(h->stream));
+            CK(h, cudaEventRecord(e1, h->stream));
+            h->prof_pending.push_back(ProfRec{e0, e1, op.cls, op.flops});
+        } else {
+            CK(h, op.fn(h->stream));
+        }
+        h->launches++;
+    }
+    return MP_OK;
+}
+
+// ------------------------------------------------------------------ lifecycle
+extern "C" {
+
+const char* mp_version(void) { return "mpgeo 0.1 sm_100a (DMMA FP64, tcgen05 TF32x3/FP16)"; }
+
+mp_status mp_get_unique_id(uint8_t id[128]) {
+    if (!id) return MP_ERR_ARG;
+    if (!g_nccl.load()) return MP_ERR_NCCL;
+    nccl_uid_t u;
+    if (g_nccl.GetUniqueId(&u) != 0) return MP_ERR_NCCL;
+    memcpy(id, u.internal, 128);
+    return MP_OK;
+}
+
+mp_status mp_init(int device, int rank, int nranks, int P, int Q, const uint8_t* id, void* cuda_stream,
+                  mp_handle** out) {
+    if (!out || nranks < 1 || rank < 0 || rank >= nranks || P < 1 || Q < 1 || P * Q != nranks || P > Q)
+        return MP_ERR_ARG;
+    mp_handle* h = new mp_handle();
+    h->device = device;
+    h->rank = rank;
+    h->nranks = nranks;
+    h->P = P;
+    h->Q = Q;
+    if (const char* e = getenv("MPGEO_TC")) h->tc_mode = atoi(e);
+    auto fail = [&](mp_status s) {
+        if (h->own_stream && h->stream) cudaStreamDestroy(h->stream);
+        delete h;
+        *out = nullptr;
+        return s;
+    };
+    if (cudaSetDevice(device) != cudaSuccess) return fail(MP_ERR_CUDA);
+    if (cuda_stream) {
+        h->stream = (cudaStream_t)cuda_stream;
+    } else {
+        if (cudaStreamCreateWithFlags(&h->stream, cudaStreamNonBlocking) != cudaSuccess) return fail(MP_ERR_CUDA);
+        h->own_stream = true;
+    }
+    if (cudaMalloc(&h->d_info, sizeof(int)) != cudaSuccess) return fail(MP_ERR_CUDA);
+    for (auto& e : h->ev)
+        if (cudaEventCreate(&e) != cudaSuccess) return fail(MP_ERR_CUDA);
+    if (nranks > 1) {
+        if (!id || !g_nccl.load()) return fail(MP_ERR_NCCL);
+        nccl_uid_t u;
+        memcpy(u.internal, id, 128);
+        if (g_nccl.CommInitRank(&h->nccl, nranks, u, rank) != 0) return fail(MP_ERR_NCCL);
+    }
+    *out = h;
+    return MP_OK;
+}
+
+mp_status mp_finalize(mp_handle* h) {
+    if (!h) return MP_ERR_ARG;
+    cudaSetDevice(h->device);
+    if (h->stream) cudaStreamSynchronize(h->stream);
+    if (h->nccl) g_nccl.CommDestroy(h->nccl);
+    for (auto& e : h->ev)
+        if (e) cudaEventDestroy(e);
+    for (auto& e : h->prof_pool)
+        if (e) cudaEventDestroy(e);
+    if (h->d_info) cudaFree(h->d_info);
+    if (h->own_stream) cudaStreamDestroy(h->stream);
+    delete h;
+    return MP_OK;
+}
+
+const char* mp_last_error(const mp_handle* h) { return h ? h->err.c_str() : "null handle"; }
+
+mp_status mp_set_profiling(mp_handle* h, int enable) {
+    if (!h) return MP_ERR_ARG;
+    if (!h->prof_pending.empty()) CK(h, cudaStreamSynchronize(h->stream));
+    h->prof_pending.clear();
+    h->prof_free = 0;
+    h->prof = mp_profile{};
+    h->profiling = enable != 0;
+    return MP_OK;
+}
+
+mp_status mp_get_profile(mp_handle* h, mp_profile* out) {
+    if (!h || !out) return MP_ERR_ARG;
+    CK(h, cudaStreamSynchronize(h->stream));
+    for (const ProfRec& r : h->prof_pending) {
+        float ms = 0.f;
+        CK(h, cudaEventElapsedTime(&ms, r.e0, r.e1));
+        h->prof.ms[r.cls] += ms;
+        h->prof.flops[r.cls] += r.flops;
+        h->prof.launches[r.cls] += 1;
+    }
+    h->prof_pending.clear();
+    h->prof_free = 0;
+    *out = h->prof;
+    return MP_OK;
+}
+int64_t mp_launch_count(const mp_handle* h) { return h ? h->launches : 0; }
+
+// ------------------------------------------------------------------ matrices
+mp_status mp_matrix_create(mp_handle* h, int64_t n, int nb, mp_matrix** A) {
+    if (!h || !A) return MP_ERR_ARG;
+    if (n < 1 || nb < 16 || nb > 8192 || nb % 16) FAIL(h, MP_ERR_ARG, "invalid n=%lld nb=%d", (long long)n, nb);
+    const int64_t nt = (n + nb - 1) / nb;
+    if (nt > 4096) FAIL(h, MP_ERR_ARG, "too many tiles (NT=%lld)", (long long)nt);
+    mp_matrix* M = new mp_matrix();
+    M->h = h;
+    M->n = n;
+    M->nb = nb;
+    M->nt = (int)nt;
+    *A = M;
+    return MP_OK;
+}
+
+mp_status mp_matrix_destroy(mp_matrix* A) {
+    delete A;
+    return MP_OK;
+}
+
+int mp_matrix_nt(const mp_matrix* A) { return A ? A->nt : 0; }
+int mp_matrix_owner(const mp_matrix* A, int m, int k) { return A ? A->owner(m, k) : -1; }
+
+mp_status mp_matrix_bytes(const mp_matrix* A, const uint8_t* storage_prec, size_t* bytes) {
+    if (!A || !bytes) return MP_ERR_ARG;
+    *bytes = layout(A, storage_prec).total;
+    return MP_OK;
+}
+
+mp_status mp_matrix_bind(mp_matrix* A, const uint8_t* storage_prec, void* d_workspace, size_t bytes) {
+    if (!A || !d_workspace) return MP_ERR_ARG;
+    mp_handle* h = A->h;
+    if ((uintptr_t)d_workspace % 256) FAIL(h, MP_ERR_ARG, "workspace must be 256-byte aligned");
+    const int nt = A->nt;
+    if (storage_prec)
+        for (int k = 0; k < nt; ++k)
+            for (int m = k; m < nt; ++m) {
+                const uint8_t p = storage_prec[(size_t)m * nt + k];
+                if (p != MP_FP64 && p != MP_FP32) FAIL(h, MP_ERR_ARG, "storage map entry (%d,%d)=%d", m, k, p);
+                if (m == k && p != MP_FP64) FAIL(h, MP_ERR_ARG, "diagonal tiles are stored in FP64 (P:117)");
+            }
+    Regions R = layout(A, storage_prec);
+    if (R.total > bytes) FAIL(h, MP_ERR_NOMEM, "workspace %zu bytes < required %zu", bytes, R.total);
+    A->R = std::move(R);
+    A->ws = (char*)d_workspace;
+    A->ws_bytes = bytes;
+    A->storage.assign((size_t)nt * nt, 255);
+    for (int k = 0; k < nt; ++k)
+        for (int m = k; m < nt; ++m)
+            A->storage[(size_t)m * nt + k] = storage_prec ? storage_prec[(size_t)m * nt + k] : (uint8_t)MP_FP64;
+    A->bound = true;
+    A->generated = A->factored = false;
+    return MP_OK;
+}
+
+mp_status mp_matrix_maps(const mp_matrix* A, uint8_t* kernel_prec, uint8_t* storage_prec, uint8_t* comm_prec) {
+    if (!A) return MP_ERR_ARG;
+    const size_t NN = (size_t)A->nt * A->nt;
+    if (kernel_prec && A->kmap.size() == NN) memcpy(kernel_prec, A->kmap.data(), NN);
+    if (storage_prec && A->storage.size() == NN) memcpy(storage_prec, A->storage.data(), NN);
+    if (comm_prec && A->cmap.size() == NN) memcpy(comm_prec, A->cmap.data(), NN);
+    return MP_OK;
+}
+
+mp_status mp_matrix_get_tile(mp_handle* h, const mp_matrix* A, int m, int k, double* h_tile) {
+    if (!h || !A || !h_tile || !A->bound || m < k || m >= A->nt || k < 0) return MP_ERR_ARG;
+    if (!A->mine(m, k)) FAIL(h, MP_ERR_ARG, "tile (%d,%d) not owned by rank %d", m, k, h->rank);
+    const size_t nb2 = A->nb2();
+    if (A->st(m, k) == MP_FP64) {
+        CK(h, cudaMemcpyAsync(h_tile, A->tile(m, k), nb2 * 8, cudaMemcpyDeviceToHost, h->stream));
+        CK(h, cudaStreamSynchronize(h->stream));
+    } else {
+        std::vector<float> tmp(nb2);
+        CK(h, cudaMemcpyAsync(tmp.data(), A->tile(m, k), nb2 * 4, cudaMemcpyDeviceToHost, h->stream));
+        CK(h, cudaStreamSynchronize(h->stream));
+        for (size_t i = 0; i < nb2; ++i) h_tile[i] = tmp[i];
+    }
+    return MP_OK;
+}
+
+mp_status mp_matrix_set_tile(mp_handle* h, mp_matrix* A, int m, int k, const double* h_tile) {
+    if (!h || !A || !h_tile || !A->bound || m < k || m >= A->nt || k < 0) return MP_ERR_ARG;
+    if (!A->mine(m, k)) FAIL(h, MP_ERR_ARG, "tile (%d,%d) not owned by rank %d", m, k, h->rank);
+    const size_t nb2 = A->nb2();
+    if (A->st(m, k) == MP_FP64) {
+        CK(h, cudaMemcpyAsync(A->tile(m, k), h_tile, nb2 * 8, cudaMemcpyHostToDevice, h->stream));
+        CK(h, cudaStreamSynchronize(h->stream));
+    } else {
+        std::vector<float> tmp(nb2);
+        for (size_t i = 0; i < nb2; ++i) tmp[i] = (float)h_tile[i];
+        CK(h, cudaMemcpyAsync(A->tile(m, k), tmp.data(), nb2 * 4, cudaMemcpyHostToDevice, h->stream));
+        CK(h, cudaStreamSynchronize(h->stream));
+    }
+    A->generated = true;
+    A->factored = false;
+    return MP_OK;
+}
+
+// ------------------------------------------------------------------ (1) generation
+static mp_status check_theta(mp_handle* h, const double* th) {
+    if (!th || !(th[0] > 0) || !(th[1] > 0) || !(th[2] > 0) || !(th[2] <= 20.0) || !std::isfinite(th[0]) ||
+        !std::isfinite(th[1]))
+        FAIL(h, MP_ERR_ARG, "invalid theta (sigma2, beta > 0, 0 < nu <= 20)");
+    return MP_OK;
+}
+
+static MaternArgs matern_args(const mp_matrix* A, const double* x, const double* y, const double* th) {
+    MaternArgs a;
+    a.x = x;
+    a.y = y;
+    a.n = A->n;
+    a.nb = A->nb;
+    a.sigma2 = th[0];
+    a.beta = th[1];
+    a.nu = th[2];
+    a.kind = th[2] == 0.5 ? 0 : th[2] == 1.5 ? 1 : th[2] == 2.5 ? 2 : 3;
+    a.coef = std::pow(2.0, 1.0 - th[2]) / std::tgamma(th[2]);
+    return a;
+}
+
+mp_status mp_matern_gen(mp_handle* h, mp_matrix* A, const double* d_x, const double* d_y, const double theta[3],
+                        const uint8_t* storage_prec, double* tile_sqnorm) {
+    if (!h || !A || !d_x || !d_y) return MP_ERR_ARG;
+    if (h->broken) FAIL(h, MP_ERR_STATE, "handle unusable after an earlier CUDA failure");
+    if (mp_status s = check_theta(h, theta)) return s;
+    if (h->nranks > 1) FAIL(h, MP_ERR_UNSUPPORTED, "multi-rank generation not in this build");
+    const int nt = A->nt;
+    const MaternArgs a = matern_args(A, d_x, d_y, theta);
+    if (!storage_prec) {
+        // pass 1: norms.  Needs scratch for partials: use the bound workspace if present,
+        // otherwise the caller must bind first (norm scratch lives in the workspace).
+        if (!A->bound) FAIL(h, MP_ERR_STATE, "bind a workspace before mp_matern_gen");
+        if (!tile_sqnorm) return MP_ERR_ARG;
+        std::vector<GenTile> tl;
+        for (int k = 0; k < nt; ++k)
+            for (int m = k; m < nt; ++m) tl.push_back(GenTile{m, k, 0, 0, nullptr});
+        Arena ar;
+        ar.dev_base = A->ws + A->R.ctrl;
+        GenTile* d_tl = ar.push(tl);
+        double* part = A->at<double>(A->R.partials);
+        double* norms = A->at<double>(A->R.norms);
+        const int per = A->nb / GEN_ROWS;
+        std::vector<Op> ops;
+        const int ntl = (int)tl.size();
+        ops.push_back({[=](cudaStream_t s) { return matern_norm_launch(a, d_tl, ntl, part, s); }, C_GEN, 0});
+        ops.push_back({[=](cudaStream_t s) { return reduce_partials_launch(part, ntl, per, norms, s); }, C_GEN, 0});
+        if (mp_status st = run_plan(h, A, ar, ops)) return st;
+        std::vector<double> v(ntl);
+        CK(h, cudaMemcpyAsync(v.data(), norms, ntl * 8, cudaMemcpyDeviceToHost, h->stream));
+        CK(h, cudaStreamSynchronize(h->stream));
+        for (size_t i = 0; i < (size_t)nt * nt; ++i) tile_sqnorm[i] = 0.0;
+        for (int i = 0; i < ntl; ++i) tile_sqnorm[(size_t)tl[i].m * nt + tl[i].k] = v[i];
+        return MP_OK;
+    }
+    if (!A->bound) FAIL(h, MP_ERR_STATE, "matrix not bound");
+    for (int k = 0; k < nt; ++k)
+        for (int m = k; m < nt; ++m)
+            if (storage_prec[(size_t)m * nt + k] != A->st(m, k))
+                FAIL(h, MP_ERR_ARG, "storage map differs from the bound one at (%d,%d)", m, k);
+    std::vector<GenTile> tl;
+    for (int k = 0; k < nt; ++k)
+        for (int m = k; m < nt; ++m)
+            if (A->mine(m, k)) tl.push_back(GenTile{m, k, A->st(m, k), 0, A->tile(m, k)});
+    Arena ar;
+    ar.dev_base = A->ws + A->R.ctrl;
+    GenTile* d_tl = ar.push(tl);
+    const int ntl = (int)tl.size();
+    std::vector<Op> ops;
+    ops.push_back({[=](cudaStream_t s) { return matern_write_launch(a, d_tl, ntl, s); }, C_GEN, 0});
+    if (mp_status st = run_plan(h, A, ar, ops)) return st;
+    A->generated = true;
+    A->factored = false;
+    return MP_OK;
+}
+
+// ------------------------------------------------------------------ (3) factorisation
+struct FlopCount {
+    double potrf = 0, trsm = 0, upd[3] = {0, 0, 0};
+};
+
+static mp_status plan_potrf(mp_handle* h, mp_matrix* A, const uint8_t* km, const uint8_t* cm, Arena& ar,
+                            std::vector<Op>& ops, FlopCount& fc) {
+    const int nt = A->nt, nb = A->nb, IB = POTRF_IB;
+    const size_t nb2 = A->nb2();
+    double* p64 = A->at<double>(A->R.p64);
+    __half* p16 = A->at<__half>(A->R.p16);
+    float* phi = A->at<float>(A->R.phi);
+    float* plo = A->at<float>(A->R.plo);
+    double* ltil = A->at<double>(A->R.ltilde);
+    double* wb = A->at<double>(A->R.wbuf);
+    double* wb2 = A->at<double>(A->R.wbuf2);
+    int* d_info = h->d_info;
+    const bool use_tc = h->tc_mode != 0 && tc_gemm_available();
+    auto K = [&](int m, int k) { return km[(size_t)m * nt + k]; };
+    auto C = [&](int m, int k) { return cm[(size_t)m * nt + k]; };
+    const double fnb = (double)nb;
+
+    auto gemm = [&](std::vector<GemmJob>& jobs, int M, int N, int Kd, int lda, int ldb, int ldc, int lower,
+                    double alpha, double beta, int round, bool cf32, int cls, double flops_per_job) {
+        if (jobs.empty()) return;
+        GemmJob* dj = ar.push(jobs);
+        DgemmArgs g{};
+        g.jobs = dj;
+        g.M = M;
+        g.N = N;
+        g.K = Kd;
+        g.lda = lda;
+        g.ldb = ldb;
+        g.ldc = ldc;
+        g.lower = lower;
+        g.alpha = alpha;
+        g.beta = beta;
+        const int nj = (int)jobs.size();
+        ops.push_back({[=](cudaStream_t s) { return dgemm_nt_launch(g, nj, round, cf32, s); }, cls, flops_per_job * nj});
+    };
+
+    for (int k = 0; k < nt; ++k) {
+        // ---- 1. DPOTRF(k,k), FP64
+        if (A->mine(k, k)) {
+            double* Akk = (double*)A->tile(k, k);
+            for (int j0 = 0; j0 < nb; j0 += IB) {
+                const int jb = std::min(IB, nb - j0);
+                double* blk = Akk + (size_t)j0 * nb + j0;
+                const int col0 = k * nb + j0;
+                ops.push_back({[=](cudaStream_t s) { return potrf_diag_block_launch(blk, nb, jb, wb, col0, d_info, s); }, C_POTRF, (double)jb * jb * jb / 3.0});
+                const int rest = nb - j0 - jb;
+                if (rest > 0) {
+                    double* X = Akk + (size_t)(j0 + jb) * nb + j0;
+                    std::vector<GemmJob> j1{GemmJob{X, wb, X}};
+                    gemm(j1, rest, jb, jb, nb, IB, nb, 0, 1.0, 0.0, P64, false, C_POTRF, (double)rest * jb * jb);
+                    std::vector<GemmJob> j2{GemmJob{X, X, Akk + (size_t)(j0 + jb) * nb + j0 + jb}};
+                    gemm(j2, rest, rest, jb, nb, nb, nb, 1, -1.0, 1.0, P64, false, C_POTRF, (double)rest * rest * jb);
+                }
+            }
+            ops.push_back({[=](cudaStream_t s) { return zero_upper_launch(Akk, nb, s); }, C_POTRF, 0});
+            fc.potrf += fnb * fnb * fnb / 3.0;
+        }
+        if (k == nt - 1) break;
+        // ---- 2. L~_kk at comm(k,k) and its 128-block inverses (TRSM operand, Alg. 2 l.5-10)
+        {
+            double* Akk = (double*)A->tile(k, k);
+            const int pc = C(k, k);
+            ops.push_back({[=](cudaStream_t s) { return round_copy_launch(Akk, ltil, (int64_t)nb2, pc, s); }, C_TRSM, 0});
+            ops.push_back({[=](cudaStream_t s) { return trtri_blocks_launch(ltil, nb, wb2, s); }, C_TRSM, 0});
+        }
+        // ---- 3. panel in
+        std::vector<PanelTile> pin, pout;
+        for (int m = k + 1; m < nt; ++m) {
+            if (!A->mine(m, k)) continue;
+            PanelTile t{};
+            t.store = A->tile(m, k);
+            t.p64 = p64 + (size_t)m * nb2;
+            t.store_prec = A->st(m, k);
+            t.comm_prec = C(m, k);
+            pin.push_back(t);
+            // which operand formats do the successors of L_mk need? (row m, column m)
+            bool need16 = false, need32 = false;
+            for (int n = k + 1; n < m; ++n) {
+                need16 |= K(m, n) == MP_FP16;
+                need32 |= K(m, n) == MP_FP32;
+            }
+            for (int n = m + 1; n < nt; ++n) {
+                need16 |= K(n, m) == MP_FP16;
+                need32 |= K(n, m) == MP_FP32;
+            }
+            if (use_tc) {
+                if (need16) t.p16 = p16 + (size_t)m * nb2;
+                if (need32) {
+                    t.hi = phi + (size_t)m * nb2;
+                    t.lo = plo + (size_t)m * nb2;
+                }
+            }
+            pout.push_back(t);
+        }
+        if (!pin.empty()) {
+            PanelTile* d_in = ar.push(pin);
+            PanelTile* d_out = ar.push(pout);
+            const int np = (int)pin.size();
+            ops.push_back({[=](cudaStream_t s) { return panel_in_launch(d_in, np, (int64_t)nb2, s); }, C_CONV, 0});
+            // ---- 4. TRSM(m,k): L_mk = A_mk L~_kk^{-T}, FP64 arithmetic (reading C12')
+            for (int j0 = 0; j0 < nb; j0 += IB) {
+                const int jb = std::min(IB, nb - j0);
+                std::vector<GemmJob> ja, jbv;
+                for (auto& t : pin) {
+                    ja.push_back(GemmJob{t.p64 + j0, wb2 + (size_t)(j0 / IB) * IB * IB, t.p64 + j0});
+                    if (j0 + jb < nb)
+                        jbv.push_back(GemmJob{t.p64 + j0, ltil + (size_t)(j0 + jb) * nb + j0, t.p64 + j0 + jb});
+                }
+                gemm(ja, nb, jb, jb, nb, IB, nb, 0, 1.0, 0.0, P64, false, C_TRSM, fnb * jb * jb);
+                gemm(jbv, nb, nb - j0 - jb, jb, nb, nb, nb, 0, -1.0, 1.0, P64, false, C_TRSM, 2.0 * fnb * (nb - j0 - jb) * jb);
+            }
+            fc.trsm += np * fnb * fnb * fnb;
+            // ---- 5. panel out (K2)
+            ops.push_back({[=](cudaStream_t s) { return panel_out_launch(d_out, np, (int64_t)nb2, s); }, C_CONV, 0});
+        }
+        // ---- 6. trailing update: SYRK + GEMM grouped by kernel(m,n)
+        std::vector<GemmJob> syrk, g64, g32, g16;
+        std::vector<TcJob> t32, t16;
+        for (int m = k + 1; m < nt; ++m) {
+            if (A->mine(m, m)) {
+                syrk.push_back(GemmJob{p64 + (size_t)m * nb2, p64 + (size_t)m * nb2, A->tile(m, m)});
+                fc.upd[MP_FP64] += fnb * fnb * fnb;
+            }
+            for (int n = k + 1; n < m; ++n) {
+                if (!A->mine(m, n)) continue;
+                const int p = K(m, n);
+                fc.upd[p] += 2.0 * fnb * fnb * fnb;
+                if (p == MP_FP64) {
+                    g64.push_back(GemmJob{p64 + (size_t)m * nb2, p64 + (size_t)n * nb2, A->tile(m, n)});
+                } else if (use_tc) {
+                    (p == MP_FP32 ? t32 : t16).push_back(TcJob{m, n, (float*)A->tile(m, n)});
+                } else {
+                    (p == MP_FP32 ? g32 : g16).push_back(GemmJob{p64 + (size_t)m * nb2, p64 + (size_t)n * nb2, A->tile(m, n)});
+                }
+            }
+        }
+        const double f3 = fnb * fnb * fnb;
+        gemm(syrk, nb, nb, nb, nb, nb, nb, 1, -1.0, 1.0, P64, false, C_UPD64, f3);
+        gemm(g64, nb, nb, nb, nb, nb, nb, 0, -1.0, 1.0, P64, false, C_UPD64, 2 * f3);
+        gemm(g32, nb, nb, nb, nb, nb, nb, 0, -1.0, 1.0, P32, true, C_UPD32, 2 * f3);
+        gemm(g16, nb, nb, nb, nb, nb, nb, 0, -1.0, 1.0, P16, true, C_UPD16, 2 * f3);
+        if (!t32.empty()) {
+            TcJob* dj = ar.push(t32);
+            const int nj = (int)t32.size();
+            TcArgs ta{dj, phi, plo, nb, nt};
+            ops.push_back({[=](cudaStream_t s) { return tc_gemm_tf32x3_launch(ta, nj, s); }, C_UPD32, 2 * f3 * nj});
+        }
+        if (!t16.empty()) {
+            TcJob* dj = ar.push(t16);
+            const int nj = (int)t16.size();
+            TcArgs ta{dj, nullptr, nullptr, nb, nt};
+            ta.p16 = p16;
+            ops.push_back({[=](cudaStream_t s) { return tc_gemm_f16_launch(ta, nj, s); }, C_UPD16, 2 * f3 * nj});
+        }
+    }
+    return MP_OK;
+}
+
+static mp_status potrf_run(mp_handle* h, mp_matrix* A, const uint8_t* km, const uint8_t* cm, int64_t* info,
+                           FlopCount* fc_out) {
+    if (!h || !A || !km || !cm) return MP_ERR_ARG;
+    if (h->broken) FAIL(h, MP_ERR_STATE, "handle unusable after an earlier CUDA failure");
+    if (!A->bound || !A->generated) FAIL(h, MP_ERR_STATE, "matrix not generated");
+    if (h->nranks > 1) FAIL(h, MP_ERR_UNSUPPORTED, "multi-rank factorisation not in this build");
+    const int nt = A->nt;
+    for (int k = 0; k < nt; ++k)
+        for (int m = k; m < nt; ++m) {
+            const size_t i = (size_t)m * nt + k;
+            if (km[i] > MP_FP16 || cm[i] > MP_FP16 || (m == k && km[i] != MP_FP64))
+                FAIL(h, MP_ERR_ARG, "bad map entry at (%d,%d)", m, k);
+            if (m > k && A->st(m, k) != (km[i] == MP_FP64 ? MP_FP64 : MP_FP32))
+                FAIL(h, MP_ERR_ARG, "kernel map inconsistent with the bound storage map at (%d,%d)", m, k);
+            if (m > k && cm[i] < A->st(m, k)) FAIL(h, MP_ERR_ARG, "comm precision above storage at (%d,%d)", m, k);
+        }
+    const int big = INT_MAX;
+    CK(h, cudaMemcpyAsync(h->d_info, &big, sizeof(int), cudaMemcpyHostToDevice, h->stream));
+    Arena ar;
+    ar.dev_base = A->ws + A->R.ctrl;
+    std::vector<Op> ops;
+    FlopCount fc;
+    if (mp_status s = plan_potrf(h, A, km, cm, ar, ops, fc)) return s;
+    if (mp_status s = run_plan(h, A, ar, ops)) return s;
+    int hinfo = 0;
+    CK(h, cudaMemcpyAsync(&hinfo, h->d_info, sizeof(int), cudaMemcpyDeviceToHost, h->stream));
+    CK(h, cudaStreamSynchronize(h->stream));
+    A->kmap.assign(km, km + (size_t)nt * nt);
+    A->cmap.assign(cm, cm + (size_t)nt * nt);
+    if (fc_out) *fc_out = fc;
+    if (hinfo != big) {
+        if (info) *info = hinfo;
+        A->factored = false;
+        FAIL(h, MP_ERR_NOT_SPD, "not positive definite at column %d", hinfo);
+    }
+    if (info) *info = 0;
+    A->factored = true;
+    return MP_OK;
+}
+
+mp_status mp_tile_potrf(mp_handle* h, mp_matrix* A, const uint8_t* kernel_prec, const uint8_t* comm_prec,
+                        int64_t* info) {
+    return potrf_run(h, A, kernel_prec, comm_prec, info, nullptr);
+}
+
+// ------------------------------------------------------------------ (4) log-likelihood
+mp_status mp_loglik(mp_handle* h, const mp_matrix* Lc, const double* d_z, double* loglik, double* logdet,
+                    double* quad) {
+    mp_matrix* A = const_cast<mp_matrix*>(Lc);
+    if (!h || !A || !d_z) return MP_ERR_ARG;
+    if (h->broken) FAIL(h, MP_ERR_STATE, "handle unusable after an earlier CUDA failure");
+    if (!A->factored) FAIL(h, MP_ERR_STATE, "matrix not factored");
+    if (h->nranks > 1) FAIL(h, MP_ERR_UNSUPPORTED, "multi-rank solve not in this build");
+    const int nt = A->nt, nb = A->nb;
+    const int64_t n = A->n;
+    double* r = A->at<double>(A->R.vec_r);
+    double* y = A->at<double>(A->R.vec_y);
+    double* part = A->at<double>(A->R.partials);
+    const int chunk = 4096;
+    const int nchunks = (int)((n + chunk - 1) / chunk);
+    CK(h, cudaMemsetAsync(r, 0, (size_t)nt * nb * 8, h->stream));
+    CK(h, cudaMemcpyAsync(r, d_z, (size_t)n * 8, cudaMemcpyDeviceToDevice, h->stream));
+    Arena ar;
+    ar.dev_base = A->ws + A->R.ctrl;
+    std::vector<Op> ops;
+    std::vector<const double*> diag;
+    std::vector<int> nreal;
+    for (int k = 0; k < nt; ++k) {
+        const double* Lkk = (const double*)A->tile(k, k);
+        diag.push_back(Lkk);
+        nreal.push_back((int)std::min<int64_t>(nb, n - (int64_t)k * nb));
+        double* rk = r + (size_t)k * nb;
+        double* yk = y + (size_t)k * nb;
+        ops.push_back({[=](cudaStream_t s) { return trsv_tile_launch(Lkk, nb, rk, yk, s); }, C_SOLVE, 0});
+        std::vector<GemvTile> gv;
+        for (int m = k + 1; m < nt; ++m) gv.push_back(GemvTile{A->tile(m, k), A->st(m, k), 0, r + (size_t)m * nb});
+        if (!gv.empty()) {
+            GemvTile* dg = ar.push(gv);
+            const int ng = (int)gv.size();
+            ops.push_back({[=](cudaStream_t s) { return gemv_sub_launch(dg, ng, yk, nb, s); }, C_SOLVE, 0});
+        }
+    }
+    const double* const* d_diag = ar.push(diag);
+    const int* d_nreal = ar.push(nreal);
+    ops.push_back({[=](cudaStream_t s) { return logdiag_launch(d_diag, d_nreal, nt, nb, part, s); }, C_SOLVE, 0});
+    ops.push_back({[=](cudaStream_t s) { return sumsq_chunks_launch(y, n, chunk, part + nt, s); }, C_SOLVE, 0});
+    if (mp_status s = run_plan(h, A, ar, ops)) return s;
+    std::vector<double> hp(nt + nchunks);
+    CK(h, cudaMemcpyAsync(hp.data(), part, hp.size() * 8, cudaMemcpyDeviceToHost, h->stream));
+    CK(h, cudaStreamSynchronize(h->stream));
+    double ld = 0.0, q = 0.0;
+    for (int k = 0; k < nt; ++k) ld += hp[k];
+    ld *= 2.0;
+    for (int c = 0; c < nchunks; ++c) q += hp[nt + c];
+    const double ll = -0.5 * (double)n * std::log(2.0 * M_PI) - 0.5 * ld - 0.5 * q;
+    if (loglik) *loglik = ll;
+    if (logdet) *logdet = ld;
+    if (quad) *quad = q;
+    return MP_OK;
+}
+
+// ------------------------------------------------------------------ one evaluation
+static void band_kernel_map(int nt, const double* s, double u_req, const double* eps, std::vector<uint8_t>& km) {
+    // reading C21: two-level rule, then the narrowest band holding every FP64 tile
+    std::vector<uint8_t> two((size_t)nt * nt);
+    const double e2[3] = {eps ? eps[0] : std::ldexp(1.0, -52), eps ? eps[1] : std::ldexp(1.0, -23), HUGE_VAL};
+    mp_precision_map(nt, s, u_req, e2, MP_COMM_TTC, two.data(), nullptr, nullptr);
+    int b = 1;
+    for (int k = 0; k < nt; ++k)
+        for (int m = k + 1; m < nt; ++m)
+            if (two[(size_t)m * nt + k] == MP_FP64) b = std::max(b, m - k + 1);
+    km.assign((size_t)nt * nt, 255);
+    for (int k = 0; k < nt; ++k)
+        for (int m = k; m < nt; ++m) km[(size_t)m * nt + k] = (m - k < b) ? MP_FP64 : MP_FP32;
+}
+
+mp_status mp_eval(mp_handle* h, mp_matrix* A, const double* x, const double* y, const double* z, int inputs_on_host,
+                  const double theta[3], double u_req, const double* eps, mp_comm_policy policy, mp_map_mode mode,
+                  const uint8_t* user_kernel_prec, mp_eval_report* rep) {
+    if (!h || !A || !x || !y || !z || !rep) return MP_ERR_ARG;
+    if (!A->bound) FAIL(h, MP_ERR_STATE, "bind a worst-case workspace (mp_matrix_bytes with NULL) first");
+    if (mp_status s = check_theta(h, theta)) return s;
+    memset(rep, 0, sizeof *rep);
+    const int nt = A->nt;
+    const int64_t n = A->n;
+    const size_t NN = (size_t)nt * nt;
+    const int64_t l0 = h->launches;
+    cudaEvent_t* ev = h->ev;
+    CK(h, cudaEventRecord(ev[0], h->stream));
+    // inputs: x, y, z live in the map-independent `inputs` region for the whole evaluation
+    const size_t nvec = (size_t)nt * A->nb;
+    double* xyz = A->at<double>(A->R.inputs);
+    const cudaMemcpyKind kind = inputs_on_host ? cudaMemcpyHostToDevice : cudaMemcpyDeviceToDevice;
+    CK(h, cudaMemcpyAsync(xyz, x, n * 8, kind, h->stream));
+    CK(h, cudaMemcpyAsync(xyz + nvec, y, n * 8, kind, h->stream));
+    CK(h, cudaMemcpyAsync(xyz + 2 * nvec, z, n * 8, kind, h->stream));
+    const double* dx = xyz;
+    const double* dy = xyz + nvec;
+    const double* dz = xyz + 2 * nvec;
+    void* ws = A->ws;
+    const size_t wsb = A->ws_bytes;
+    std::vector<double> s(NN, 0.0);
+    std::vector<uint8_t> km(NN, 255), sm(NN, 255), cm(NN, 255);
+    if (mode == MP_MAP_ADAPTIVE || mode == MP_MAP_BAND) {
+        if (mp_status st = mp_matern_gen(h, A, dx, dy, theta, nullptr, s.data())) return st;
+    }
+    CK(h, cudaEventRecord(ev[1], h->stream));
+    mp_status st = MP_OK;
+    switch (mode) {
+        case MP_MAP_ADAPTIVE:
+            st = mp_precision_map(nt, s.data(), u_req, eps, policy, km.data(), sm.data(), cm.data());
+            break;
+        case MP_MAP_BAND:
+            band_kernel_map(nt, s.data(), u_req, eps, km);
+            st = mp_precision_map(nt, nullptr, u_req, eps, policy, km.data(), sm.data(), cm.data());
+            break;
+        case MP_MAP_FP64:
+        case MP_MAP_EXTREME:
+            for (int k = 0; k < nt; ++k)
+                for (int m = k; m < nt; ++m)
+                    km[(size_t)m * nt + k] = (m == k || mode == MP_MAP_FP64) ? MP_FP64 : MP_FP16;
+            st = mp_precision_map(nt, nullptr, u_req, eps, policy, km.data(), sm.data(), cm.data());
+            break;
+        case MP_MAP_USER:
+            if (!user_kernel_prec) return MP_ERR_ARG;
+            km.assign(user_kernel_prec, user_kernel_prec + NN);
+            st = mp_precision_map(nt, nullptr, u_req, eps, policy, km.data(), sm.data(), cm.data());
+            break;
+        default:
+            return MP_ERR_ARG;
+    }
+    if (st) FAIL(h, st, "precision map failed");
+    if (mp_status b = mp_matrix_bind(A, sm.data(), ws, wsb)) return b;
+    if (mp_status g = mp_matern_gen(h, A, dx, dy, theta, sm.data(), nullptr)) return g;
+    CK(h, cudaEventRecord(ev[2], h->stream));
+    FlopCount fc;
+    int64_t info = 0;
+    mp_status pst = potrf_run(h, A, km.data(), cm.data(), &info, &fc);
+    CK(h, cudaEventRecord(ev[3], h->stream));
+    rep->info = info;
+    for (int k = 0; k < nt; ++k)
+        for (int m = k + 1; m < nt; ++m) {
+            const size_t i = (size_t)m * nt + k;
+            rep->tiles[km[i]]++;
+            if (cm[i] > sm[i]) rep->stc_tiles++;
+        }
+    for (int c = 0; c < 3; ++c) rep->flops_update[c] = fc.upd[c];
+    rep->flops_potrf = fc.potrf + fc.trsm;
+    if (pst == MP_ERR_NOT_SPD) {
+        rep->loglik = -HUGE_VAL;
+        rep->gpu_launches = h->launches - l0;
+        return pst;
+    }
+    if (pst) return pst;
+    if (mp_status l = mp_loglik(h, A, dz, &rep->loglik, &rep->logdet, &rep->quad)) return l;
+    CK(h, cudaEventRecord(ev[4], h->stream));
+    CK(h, cudaEventSynchronize(ev[4]));
+    float t01, t12, t23, t34, t04;
+    cudaEventElapsedTime(&t01, ev[0], ev[1]);
+    cudaEventElapsedTime(&t12, ev[1], ev[2]);
+    cudaEventElapsedTime(&t23, ev[2], ev[3]);
+    cudaEventElapsedTime(&t34, ev[3], ev[4]);
+    cudaEventElapsedTime(&t04, ev[0], ev[4]);
+    rep->t_map_ms = 0;
+    rep->t_gen_ms = t01 + t12;
+    rep->t_potrf_ms = t23;
+    rep->t_solve_ms = t34;
+    rep->t_total_ms = t04;
+    rep->gpu_launches = h->launches - l0;
+    return MP_OK;
+}
+
+}  // extern "C"

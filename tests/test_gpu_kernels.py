@@ -1,0 +1,80 @@
+"""Kernel-level GPU checks through the C-ABI test hooks (include/mpgeo_test.h)."""
+import ctypes as C
+
+import mpmath
+import numpy as np
+import pytest
+
+pytestmark = pytest.mark.gpu
+
+
+@pytest.fixture(scope="module")
+def lib():
+    import torch
+    assert torch.cuda.is_available()
+    from paper_conf_cluster_caoalgkb23_b200._lib import lib
+    return lib
+
+
+def dev(a):
+    import torch
+    return torch.from_numpy(np.ascontiguousarray(a)).cuda()
+
+
+@pytest.mark.parametrize("nu", [0.3, 0.5, 0.8, 1.0, 1.5, 1.7, 3.7, 12.3])
+def test_bessel_k_device_vs_mpmath(lib, nu):
+    mpmath.mp.dps = 30
+    x = np.concatenate([np.logspace(-5, 2.2, 120), [1.9999999999, 2.0, 2.0000000001]])
+    dx = dev(x)
+    out = dev(np.zeros_like(x))
+    assert lib.mp_test_bessel_k(nu, C.c_void_p(dx.data_ptr()), C.c_void_p(out.data_ptr()), x.size) == 0
+    got = out.cpu().numpy()
+    for xi, g in zip(x, got):
+        ref = float(mpmath.besselk(nu, xi))
+        assert abs(g - ref) <= 4e-15 * (1 + xi) * abs(ref), (nu, xi, g, ref)
+
+
+def run_dgemm(lib, A, B, Cm, lower=0, alpha=-1.0, beta=1.0, rnd=0, cf32=0):
+    M, K = A.shape
+    N = B.shape[0]
+    dA, dB, dC = dev(A), dev(B), dev(Cm)
+    st = lib.mp_test_dgemm(C.c_void_p(dA.data_ptr()), C.c_void_p(dB.data_ptr()), C.c_void_p(dC.data_ptr()),
+                           M, N, K, K, K, Cm.shape[1], lower, alpha, beta, rnd, cf32)
+    assert st == 0
+    return dC.cpu().numpy()
+
+
+@pytest.mark.parametrize("M,N,K", [(128, 128, 16), (300, 200, 144), (2048, 256, 2048), (16, 48, 32)])
+def test_dgemm_update_fp64(lib, M, N, K):
+    rng = np.random.default_rng(M + N + K)
+    A, B, Cm = rng.standard_normal((M, K)), rng.standard_normal((N, K)), rng.standard_normal((M, N))
+    got = run_dgemm(lib, A, B, Cm)
+    ref = Cm - A @ B.T
+    assert np.max(np.abs(got - ref)) <= 1e-15 * K * 8
+
+
+def test_dgemm_overwrite_and_lower(lib):
+    rng = np.random.default_rng(1)
+    A, B, Cm = rng.standard_normal((400, 64)), rng.standard_normal((400, 64)), rng.standard_normal((400, 400))
+    got = run_dgemm(lib, A, B, Cm, alpha=1.0, beta=0.0)
+    assert np.max(np.abs(got - A @ B.T)) <= 1e-13
+    got = run_dgemm(lib, A, B, Cm, lower=1)
+    ref = Cm - A @ B.T
+    for bi in range(4):
+        for bj in range(4):
+            blk = (slice(bi * 128, (bi + 1) * 128), slice(bj * 128, (bj + 1) * 128))
+            if bj <= bi:
+                assert np.max(np.abs(got[blk] - ref[blk])) <= 1e-13
+            else:
+                assert np.array_equal(got[blk], Cm[blk])  # strictly upper CTA tiles untouched
+
+
+@pytest.mark.parametrize("rnd,npdt", [(1, np.float32), (2, np.float16)])
+def test_dgemm_rounded_operands_fp32_c(lib, rnd, npdt):
+    rng = np.random.default_rng(rnd)
+    A, B = rng.standard_normal((256, 128)), rng.standard_normal((256, 128))
+    Cm = rng.standard_normal((256, 256)).astype(np.float32)
+    got = run_dgemm(lib, A, B, Cm, rnd=rnd, cf32=1)
+    Ar, Br = A.astype(npdt).astype(np.float64), B.astype(npdt).astype(np.float64)
+    ref = (Cm.astype(np.float64) - Ar @ Br.T).astype(np.float32)
+    assert np.max(np.abs(got.astype(np.float64) - ref)) <= 2 * np.max(np.abs(ref)) * 2.0**-24

@@ -1,0 +1,235 @@
+"""Parity of the CUDA path (through the C ABI) against the CPU oracle.
+
+Tolerances (BASELINE.json north_star):
+  all-FP64: ||A - L L^T||_F / ||A||_F <= 1e-13, l relative error <= 1e-10;
+  mixed precision: l relative error <= 1e-5 vs the FP64 oracle; precision maps bit-exact.
+"""
+import math
+
+import numpy as np
+import pytest
+
+import synth
+from oracle import FP16, FP64
+from oracle.cholesky import residual, tile_cholesky
+from oracle.loglik import loglik as oracle_loglik, loglik_from_factor
+from oracle.precision import all_fp64_maps, comm_map, extreme_map, precision_maps, storage_map
+from oracle.tiles import assemble, gen_lower_tiles, num_tiles, tile_range, tile_sqnorms
+from tests.gpu_helpers import gpu_factor_dense, near_tie_guard, to_dev
+
+pytestmark = pytest.mark.gpu
+
+
+@pytest.fixture(scope="module")
+def mp():
+    import torch
+    assert torch.cuda.is_available(), "the -m gpu tests need a GPU"
+    import paper_conf_cluster_caoalgkb23_b200 as mp
+    return mp
+
+
+@pytest.fixture(scope="module")
+def handle(mp):
+    return mp.Handle(0)
+
+
+def stepwise(mp, handle, x, y, z, theta, nb, maps=None, u_req=1e-9):
+    """gen pass 1 -> map -> bind -> gen pass 2 -> potrf -> loglik through the four ABI calls."""
+    n = x.shape[0]
+    M = mp.Matrix(handle, n, nb, None)
+    dx, dy, dz = to_dev(x), to_dev(y), to_dev(z)
+    s = M.matern_gen(dx, dy, theta)
+    if maps is None:
+        km, sm, cm = mp.precision_map(s, u_req)
+    else:
+        km, sm, cm = maps
+    M.bind(sm)
+    M.matern_gen(dx, dy, theta, sm)
+    info = M.potrf(km, cm)
+    assert info == 0
+    ll = M.loglik(dz)
+    return M, s, (km, sm, cm), ll
+
+
+@pytest.mark.parametrize("n,nb,theta", [(1600, 400, (1.0, 0.1, 0.5)), (2500, 384, (1.3, 0.05, 0.8)),
+                                         (900, 256, (0.7, 0.2, 1.5))])
+def test_generation_tiles_and_norms(mp, handle, n, nb, theta):
+    x, y = synth.locations(n, 0)
+    M = mp.Matrix(handle, n, nb, None)
+    dx, dy = to_dev(x), to_dev(y)
+    s = M.matern_gen(dx, dy, theta)
+    nt = num_tiles(n, nb)
+    tiles = gen_lower_tiles(x, y, theta, nb)
+    so = tile_sqnorms(tiles, nt)
+    low = np.tril(np.ones((nt, nt), bool))
+    assert np.max(np.abs(s[low] - so[low]) / so[low]) <= 1e-13
+    M.matern_gen(dx, dy, theta, np.zeros((nt, nt), np.uint8))
+    tol = 1e-15 if theta[2] == 0.5 else 2e-13
+    for (m, k), t in tiles.items():
+        g = M.tile(m, k)
+        r = t.shape[0]
+        c = t.shape[1]
+        assert np.max(np.abs(g[:r, :c] - t)) <= tol * theta[0] * 4
+        pad = g.copy()
+        pad[:r, :c] = 0
+        expect = np.zeros_like(pad)
+        if m == k:
+            for i in range(r, nb):
+                expect[i, i] = 1.0
+        assert np.array_equal(pad, expect)
+
+
+def test_generation_fp32_storage(mp, handle):
+    n, nb, theta = 1024, 256, (1.0, 0.05, 0.5)
+    x, y = synth.locations(n, 4)
+    M = mp.Matrix(handle, n, nb, None)
+    nt = M.nt
+    sm = np.full((nt, nt), 255, np.uint8)
+    for k in range(nt):
+        for m in range(k, nt):
+            sm[m, k] = 0 if m == k else 1
+    M.bind(sm)
+    M.matern_gen(to_dev(x), to_dev(y), theta, sm)
+    t = gen_lower_tiles(x, y, theta, nb)[3, 1]
+    assert np.array_equal(M.tile(3, 1), t.astype(np.float32).astype(np.float64))
+
+
+def test_map_from_gpu_norms_bit_exact(mp, handle):
+    n, nb, u_req = 10000, 512, 1e-9
+    x, y = synth.locations(n, 0)
+    theta = (1.0, 0.03, 0.5)
+    M = mp.Matrix(handle, n, nb, None)
+    s = M.matern_gen(to_dev(x), to_dev(y), theta)
+    so = tile_sqnorms(gen_lower_tiles(x, y, theta, nb), M.nt)
+    near_tie_guard(so, M.nt, u_req)
+    got = mp.precision_map(s, u_req)
+    ref = precision_maps(so, u_req)
+    low = np.tril(np.ones((M.nt, M.nt), bool))
+    for g, r in zip(got, ref):
+        assert np.array_equal(g[low], r[low])
+    assert len(set(got[0][low].tolist())) == 3  # the case exercises all three classes
+
+
+@pytest.mark.parametrize("n,nb,theta", [(1600, 400, (1.0, 0.1, 0.5)), (4900, 512, (1.0, 0.1, 0.5)),
+                                         (3600, 1024, (1.5, 0.07, 1.0))])
+def test_fp64_path_vs_oracle(mp, handle, n, nb, theta):
+    x, y = synth.locations(n, 0)
+    z = synth.normal_vector(n, 1)
+    nt = num_tiles(n, nb)
+    M, _, _, (ll, ld, q) = stepwise(mp, handle, x, y, z, theta, nb, maps=all_fp64_maps(nt))
+    ref = oracle_loglik(x, y, z, theta, nb)
+    L = gpu_factor_dense(M, n)
+    Lo = np.tril(assemble(ref["factor"], n, nb))
+    assert np.max(np.abs(L - Lo)) <= 1e-12 * theta[0]
+    assert residual(ref["tiles"], {key: M.tile(*key)[: t.shape[0], : t.shape[1]] for key, t in ref["tiles"].items()},
+                    n, nb) <= 1e-13
+    assert abs(ll - ref["loglik"]) <= 1e-10 * abs(ref["loglik"])
+    assert abs(ld - ref["logdet"]) <= 1e-10 * abs(ref["logdet"])
+    assert abs(q - ref["quad"]) <= 1e-10 * abs(ref["quad"])
+
+
+def test_config1_via_mp_eval_host_and_device_inputs(mp, handle):
+    """Config 1 (BASELINE.json configs[0]): n=1600, 40x40 grid, theta=(1,0.1,0.5), tile 400, all FP64."""
+    n, nb, theta = 1600, 400, (1.0, 0.1, 0.5)
+    x, y = synth.locations(n, 0)
+    z = synth.normal_vector(n, 1)
+    ref = oracle_loglik(x, y, z, theta, nb)
+    ev = mp.Evaluator(n, nb, handle=handle)
+    r1 = ev.eval(x, y, z, theta, mode=mp.MP_MAP_FP64)
+    r2 = ev.eval(to_dev(x), to_dev(y), to_dev(z), theta, mode=mp.MP_MAP_FP64)
+    r3 = ev.eval(x, y, z, theta, mode=mp.MP_MAP_ADAPTIVE)  # the rule also gives all FP64 here
+    assert r1.loglik == r2.loglik == r3.loglik  # deterministic, input location irrelevant
+    assert abs(r1.loglik - ref["loglik"]) <= 1e-10 * abs(ref["loglik"])
+    assert r3.tiles[1] == 0 and r3.tiles[2] == 0
+    assert r1.gpu_launches > 0
+
+
+def test_kms_closed_form_large(mp, handle):
+    from tests.test_oracle_cholesky import kms_closed_form
+    n, nb, delta, beta, sigma2 = 12000, 1024, 1e-4, 0.02, 1.2
+    x, y = synth.collinear_locations(n, delta)
+    z = synth.normal_vector(n, 3)
+    rho = math.exp(-delta / beta)
+    ld_ref = n * math.log(sigma2) + (n - 1) * math.log(1 - rho * rho)
+    q_ref = (z[0] ** 2 + z[-1] ** 2 + (1 + rho * rho) * float(np.sum(z[1:-1] ** 2))
+             - 2 * rho * float(np.sum(z[:-1] * z[1:]))) / (sigma2 * (1 - rho * rho))
+    ll_ref = -0.5 * n * math.log(2 * math.pi) - 0.5 * ld_ref - 0.5 * q_ref
+    ev = mp.Evaluator(n, nb, handle=handle)
+    r = ev.eval(x, y, z, (sigma2, beta, 0.5), mode=mp.MP_MAP_FP64)
+    assert abs(r.logdet - ld_ref) <= 1e-10 * abs(ld_ref)
+    assert abs(r.quad - q_ref) <= 1e-10 * abs(q_ref)
+    assert abs(r.loglik - ll_ref) <= 1e-10 * abs(ll_ref)
+
+
+@pytest.mark.parametrize("beta", [0.03, 0.1])
+def test_mixed_precision_path(mp, handle, beta):
+    n, nb, u_req = 10000, 512, 1e-9
+    theta = (1.0, beta, 0.5)
+    x, y = synth.locations(n, 0)
+    z = synth.normal_vector(n, 1)
+    ref = oracle_loglik(x, y, z, theta, nb)
+    nt = num_tiles(n, nb)
+    so = tile_sqnorms(ref["tiles"], nt)
+    near_tie_guard(so, nt, u_req)
+    maps = precision_maps(so, u_req)
+    emu = oracle_loglik(x, y, z, theta, nb, maps=maps)
+    ev = mp.Evaluator(n, nb, handle=handle)
+    r = ev.eval(x, y, z, theta, u_req=u_req)
+    km, sm, cm = ev.M.maps()
+    low = np.tril(np.ones((nt, nt), bool))
+    for g, o in zip((km, sm, cm), maps):
+        assert np.array_equal(g[low], o[low])
+    err = abs(r.loglik - ref["loglik"]) / abs(ref["loglik"])
+    assert err <= 1e-5  # north-star MP tolerance
+    assert err <= 1e-8  # regression bound (survey emulation: 5e-11 .. 7e-10)
+    assert abs(r.loglik - emu["loglik"]) <= 1e-8 * abs(emu["loglik"])
+
+
+def test_extreme_map_stc_and_ttc(mp, handle):
+    """P:294 extreme FP64/FP16 map: AUTO -> every communication STC; TTC keeps storage precision."""
+    n, nb, theta = 4096, 512, (1.0, 0.03, 0.5)
+    x, y = synth.locations(n, 2)
+    z = synth.normal_vector(n, 1)
+    nt = num_tiles(n, nb)
+    km = extreme_map(nt, FP16)
+    ev = mp.Evaluator(n, nb, handle=handle)
+    out = {}
+    for pol in (mp.MP_COMM_AUTO, mp.MP_COMM_TTC):
+        r = ev.eval(x, y, z, theta, mode=mp.MP_MAP_EXTREME, policy=pol)
+        emu = oracle_loglik(x, y, z, theta, nb, maps=(km, storage_map(km), comm_map(km, pol)))
+        assert abs(r.loglik - emu["loglik"]) <= 1e-6 * abs(emu["loglik"])
+        out[pol] = r
+    assert out[mp.MP_COMM_AUTO].stc_tiles == nt * (nt - 1) // 2
+    assert out[mp.MP_COMM_TTC].stc_tiles == 0
+
+
+def test_not_spd_reports_info(mp, handle):
+    n, nb = 700, 256
+    M = mp.Matrix(handle, n, nb, None)
+    nt = M.nt
+    a = np.eye(nt * nb)
+    a[517, 517] = -2.0
+    for k in range(nt):
+        for m in range(k, nt):
+            M.set_tile(m, k, a[m * nb:(m + 1) * nb, k * nb:(k + 1) * nb])
+    km, sm, cm = all_fp64_maps(nt)
+    assert M.potrf(km, cm) == 518
+
+
+def test_user_matrix_factor_matches_lapack(mp, handle):
+    """Factor a random SPD matrix given through mp_matrix_set_tile (no Matérn)."""
+    n, nb = 1000, 208
+    rng = np.random.default_rng(7)
+    G = rng.standard_normal((n, n))
+    A = G @ G.T / n + np.eye(n)
+    M = mp.Matrix(handle, n, nb, None)
+    nt = M.nt
+    Ap = np.eye(nt * nb)
+    Ap[:n, :n] = A
+    for k in range(nt):
+        for m in range(k, nt):
+            M.set_tile(m, k, Ap[m * nb:(m + 1) * nb, k * nb:(k + 1) * nb])
+    km, sm, cm = all_fp64_maps(nt)
+    assert M.potrf(km, cm) == 0
+    L = gpu_factor_dense(M, n)
+    assert np.max(np.abs(L - np.linalg.cholesky(A))) <= 1e-12
