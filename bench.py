@@ -1,0 +1,356 @@
+#!/usr/bin/env python
+"""bench.py — Tflop/s and joules per Matérn log-likelihood evaluation (BASELINE.json metric).
+
+One "step" = one whole evaluation l(theta) of Eq. (1): Matérn tile generation with tile
+norms, the precision maps (Alg. 2), the mixed-precision tile Cholesky
+(Alg. 1) and the log-determinant + forward solve — every row of SURVEY.md §8(a) — through the
+C ABI (mp_eval).  Tflop/s = (n^3/3) / T_eval.
+
+Default (N=1): config 3 of BASELINE.json, n = 160,000 (400 x 400 jittered grid, Morton order),
+nb = 2048, theta = (1, 0.03, 0.5), adaptive FP64/FP32/FP16 map at u_req = 1e-9 — the largest
+configuration that fits one B200 (config 4, n = 360k, needs 320 GB).  The matrix (~68 GB) is far
+larger than L2, so no explicit flush is needed between steps.
+
+  python bench.py [--gpus N] [--steps K] [--warmup W] [--config c3] [--map adaptive]
+  python bench.py --impl reference ...   # the CPU oracle on a bounded sample (the reference arm)
+
+N > 1 (torchrun): each rank evaluates its own replica (weak scaling, no collective on the data
+path; the Monte-Carlo MLE study of P:264 is embarrassingly parallel over replicas); time is the
+max over ranks and value is the flops of all ranks / that time.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import math
+import os
+import statistics
+import subprocess
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+CONFIGS = {
+    "c1": dict(n=1600, nb=400, theta=(1.0, 0.1, 0.5), map="fp64"),
+    "c2": dict(n=40000, nb=2048, theta=(1.0, 0.03, 0.5), map="band"),
+    "c3": dict(n=160000, nb=2048, theta=(1.0, 0.03, 0.5), map="adaptive"),
+    "c5": dict(n=250000, nb=2048, theta=(1.0, 0.03, 0.5), map="adaptive"),
+}
+METRIC = "Tflop/s & joules per MLE log-likelihood eval (n=360k) at 1/2/4/8 B200"
+FP64_NOMINAL, BF16_NOMINAL = 40.0, 2250.0  # TFLOP/s dense, B200 datasheet (ratio used for the FP64 peak)
+
+
+def measured_peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        d = json.load(open(p))
+        return d, "measured"
+    return {"hbm_gbs": 6650.0, "bf16_tflops": 1590.0, "bf16_tflops_sustained": 1400.0}, "fallback"
+
+
+class ClockSampler:
+    """nvidia-smi clocks / throttle reasons sampled during the timed region."""
+
+    FIELDS = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
+              "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+              "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, device: int):
+        self.device = device
+        self.rows = []
+        self.proc = None
+
+    def start(self):
+        try:
+            self.proc = subprocess.Popen(["nvidia-smi", "-i", str(self.device), f"--query-gpu={self.FIELDS}",
+                                          "--format=csv,noheader,nounits", "-lms", "200"],
+                                         stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            threading.Thread(target=self._read, daemon=True).start()
+        except (OSError, FileNotFoundError):
+            self.proc = None
+
+    def _read(self):
+        for line in self.proc.stdout:
+            parts = [p.strip() for p in line.split(",")]
+            if len(parts) >= 9:
+                self.rows.append(parts)
+
+    def stop(self):
+        if self.proc:
+            self.proc.terminate()
+            try:
+                self.proc.wait(timeout=5)
+            except subprocess.TimeoutExpired:
+                self.proc.kill()
+        sm = [float(r[1]) for r in self.rows if r[1].replace(".", "").isdigit()]
+        mx = [float(r[2]) for r in self.rows if r[2].replace(".", "").isdigit()]
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        reasons = sorted({names[i] for r in self.rows for i in range(4) if r[5 + i].lower() == "active"})
+        return {"sm_mhz": statistics.median(sm) if sm else None, "sm_max_mhz": max(mx) if mx else None,
+                "reasons": reasons, "samples": len(self.rows)}
+
+
+def nvml_energy_mj(device: int):
+    try:
+        import pynvml
+        pynvml.nvmlInit()
+        h = pynvml.nvmlDeviceGetHandleByIndex(device)
+        return float(pynvml.nvmlDeviceGetTotalEnergyConsumption(h))
+    except Exception:
+        return None
+
+
+def cublas_dgemm_tflops(seconds=1.5):
+    """Context only: cuBLAS DGEMM 8192^3 back to back (not the roofline denominator)."""
+    import torch
+    a = torch.randn(8192, 8192, dtype=torch.float64, device="cuda")
+    b = torch.randn(8192, 8192, dtype=torch.float64, device="cuda")
+    torch.matmul(a, b)
+    torch.cuda.synchronize()
+    s, e = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    it = 0
+    s.record()
+    t0 = time.time()
+    while time.time() - t0 < seconds:
+        torch.matmul(a, b)
+        it += 1
+    e.record()
+    torch.cuda.synchronize()
+    return 2 * 8192**3 * it / (s.elapsed_time(e) / 1e3) / 1e12
+
+
+# --------------------------------------------------------------------------- oracle (CPU) leg
+def oracle_sample_eval(n=10000, nb=512, theta=(1.0, 0.03, 0.5), u_req=1e-9, map_mode="adaptive"):
+    """One oracle evaluation as it stands (generation + norms + maps + tile Cholesky + Eq. (1))."""
+    import synth
+    from oracle.loglik import loglik as oracle_loglik
+    from oracle.precision import precision_maps
+    from oracle.tiles import gen_lower_tiles, num_tiles, tile_sqnorms
+
+    x, y = synth.locations(n, 0)
+    z = synth.normal_vector(n, 1)
+    t0 = time.perf_counter()
+    if map_mode == "fp64":
+        oracle_loglik(x, y, z, theta, nb)
+    else:
+        s = tile_sqnorms(gen_lower_tiles(x, y, theta, nb), num_tiles(n, nb))
+        oracle_loglik(x, y, z, theta, nb, maps=precision_maps(s, u_req))
+    return time.perf_counter() - t0
+
+
+def cpu_cores():
+    try:
+        from threadpoolctl import threadpool_info
+        th = [i.get("num_threads", 0) for i in threadpool_info() if i.get("user_api") == "blas"]
+        return max(th) if th else os.cpu_count()
+    except Exception:
+        return os.cpu_count()
+
+
+def cpu_baseline(map_mode):
+    n_s, nb_s = 10000, 512
+    t = oracle_sample_eval(n_s, nb_s, map_mode=map_mode)
+    return {"value": (n_s**3 / 3) / t / 1e12, "unit": "Tflop/s", "cores": cpu_cores(), "kind": "oracle",
+            "sample": f"1 oracle evaluation at n={n_s} (100x100 grid), nb={nb_s}, {map_mode} map, same theta/recipe "
+                      f"as the workload: NumPy/SciPy FP64 generation+norms+maps+tile Cholesky+Eq.(1); {t:.1f} s",
+            "seconds": t}
+
+
+def run_reference(args, cfg, world, rank):
+    if rank != 0:
+        return
+    steps, times = args.steps, []
+    for i in range(args.warmup + args.steps):
+        t = oracle_sample_eval(map_mode=cfg["map"])
+        if i >= args.warmup:
+            times.append(t)
+    n_s = 10000
+    T = sum(times)
+    val = steps * (n_s**3 / 3) / T / 1e12
+    cores = cpu_cores()
+    out = {"impl": "reference", "metric": METRIC, "value": val, "unit": "Tflop/s", "n_gpus": world, "steps": steps,
+           "warmup": args.warmup, "ms_per_step": 1e3 * T / steps, "higher_is_better": True, "scaling": "weak",
+           "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+           "config": {"workload": f"{args.config} sample: n=10000 nb=512 (bounded oracle sample)",
+                      "map": cfg["map"], "theta": list(cfg["theta"])},
+           "cpu_baseline": {"value": val, "unit": "Tflop/s", "cores": cores, "kind": "oracle",
+                            "sample": "each step = 1 oracle evaluation at n=10000, nb=512 (CPU, NumPy/SciPy FP64)"},
+           "e2e": {"value": val, "unit": "Tflop/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(out), flush=True)
+
+
+# --------------------------------------------------------------------------- GPU leg
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=3)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--config", default="c3", choices=sorted(CONFIGS))
+    ap.add_argument("--map", default=None, choices=["adaptive", "fp64", "band", "extreme"])
+    ap.add_argument("--policy", default="auto", choices=["auto", "ttc"])
+    ap.add_argument("--u-req", type=float, default=1e-9)
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-e2e", action="store_true")
+    args = ap.parse_args()
+    cfg = dict(CONFIGS[args.config])
+    if args.map:
+        cfg["map"] = args.map
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    if args.impl == "reference":
+        return run_reference(args, cfg, world, rank)
+    if args.warmup < 3:
+        print("note: --warmup raised to 3 (timing rules)", file=sys.stderr)
+        args.warmup = 3
+
+    import numpy as np
+    import torch
+
+    import paper_conf_cluster_caoalgkb23_b200 as mp
+    import synth
+
+    torch.cuda.set_device(local)
+    dist = None
+    if world > 1:
+        import torch.distributed as dist
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    n, nb, theta = cfg["n"], cfg["nb"], cfg["theta"]
+    mode = {"adaptive": mp.MP_MAP_ADAPTIVE, "fp64": mp.MP_MAP_FP64, "band": mp.MP_MAP_BAND,
+            "extreme": mp.MP_MAP_EXTREME}[cfg["map"]]
+    policy = mp.MP_COMM_AUTO if args.policy == "auto" else mp.MP_COMM_TTC
+    x, y = synth.locations(n, seed=rank)
+    z = synth.normal_vector(n, seed=1 + rank)
+    dx, dy, dz = (torch.from_numpy(a).cuda() for a in (x, y, z))
+    hx, hy, hz = (torch.from_numpy(a).pin_memory() for a in (x, y, z))
+    ev = mp.Evaluator(n, nb, device=local)
+    h = ev.handle
+    stream = h.stream
+
+    def step(on_host=False):
+        if on_host:
+            return ev.eval(hx.numpy(), hy.numpy(), hz.numpy(), theta, u_req=args.u_req, mode=mode, policy=policy)
+        return ev.eval(dx, dy, dz, theta, u_req=args.u_req, mode=mode, policy=policy)
+
+    for _ in range(args.warmup):
+        rep = step()
+    torch.cuda.synchronize()
+
+    def barrier():
+        if dist:
+            dist.barrier()
+        torch.cuda.synchronize()
+
+    # ---- timed region: K evaluations, inputs resident in HBM
+    clocks = ClockSampler(local)
+    barrier()
+    e0_mj = nvml_energy_mj(local)
+    clocks.start()
+    h.set_profiling(True)
+    l0 = h.launches
+    ev_s, ev_e = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    ev_s.record(stream)
+    reps = []
+    for _ in range(args.steps):
+        reps.append(step())
+    ev_e.record(stream)
+    barrier()
+    e1_mj = nvml_energy_mj(local)
+    ck = clocks.stop()
+    launches = h.launches - l0
+    prof = h.profile()
+    h.set_profiling(False)
+    t_ms = ev_s.elapsed_time(ev_e)
+    if dist:
+        t = torch.tensor([t_ms], device="cuda")
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        t_ms = float(t.item())
+    joules = None if e0_mj is None or e1_mj is None else (e1_mj - e0_mj) / 1e3
+    if dist and joules is not None:
+        t = torch.tensor([joules], device="cuda", dtype=torch.float64)
+        dist.all_reduce(t)
+        joules = float(t.item())
+    flops_eval = n**3 / 3.0
+    value = world * args.steps * flops_eval / (t_ms / 1e3) / 1e12
+
+    # ---- e2e: same metric through mp_eval with pinned HOST inputs (H2D inside the call) and the
+    # results (norms, info, partial sums, scalars) read back to the host every step
+    e2e = None
+    if not args.no_e2e:
+        barrier()
+        es, ee = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        es.record(stream)
+        for _ in range(args.steps):
+            step(on_host=True)
+        ee.record(stream)
+        barrier()
+        te = es.elapsed_time(ee)
+        if dist:
+            t = torch.tensor([te], device="cuda")
+            dist.all_reduce(t, op=dist.ReduceOp.MAX)
+            te = float(t.item())
+        nt = ev.nt
+        chunks = (n + 4095) // 4096
+        d2h = (nt * (nt + 1) // 2) * 8 if mode in (mp.MP_MAP_ADAPTIVE, mp.MP_MAP_BAND) else 0
+        d2h += 4 + (nt + chunks) * 8
+        e2e = {"value": world * args.steps * flops_eval / (te / 1e3) / 1e12, "unit": "Tflop/s",
+               "h2d_bytes_per_step": 3 * n * 8, "d2h_bytes_per_step": d2h, "ms_per_step": te / args.steps}
+
+    if rank != 0:
+        if dist:
+            dist.destroy_process_group()
+        return
+    peaks, peak_src = measured_peaks()
+    p = prof.as_dict()
+    dom = p["upd_fp64"]
+    fp64_peak = peaks["bf16_tflops_sustained"] * FP64_NOMINAL / BF16_NOMINAL
+    achieved = dom["flops"] / (dom["ms"] / 1e3) / 1e12 if dom["ms"] > 0 else 0.0
+    try:
+        cub = cublas_dgemm_tflops()
+    except Exception:
+        cub = None
+    last = reps[-1]
+    upd = list(last.flops_update)
+    roof_time_s = (upd[0] / (fp64_peak * 1e12)
+                   + upd[1] / (peaks["bf16_tflops_sustained"] * 0.5 / 3 * 1e12)
+                   + upd[2] / (peaks["bf16_tflops_sustained"] * 1e12))
+    t_upd_s = (p["upd_fp64"]["ms"] + p["upd_fp32"]["ms"] + p["upd_fp16"]["ms"]) / 1e3 / args.steps
+    out = {
+        "metric": METRIC, "value": value, "unit": "Tflop/s", "n_gpus": world, "steps": args.steps,
+        "warmup": args.warmup, "ms_per_step": t_ms / args.steps, "higher_is_better": True, "scaling": "weak",
+        "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+        "config": {"workload": f"{args.config}: n={n} ({int(math.isqrt(n))}^2 jittered grid, Morton order), nb={nb}, "
+                               f"theta={list(theta)}, {cfg['map']} map u_req={args.u_req}, comm={args.policy}",
+                   "n": n, "nb": nb, "map": cfg["map"], "policy": args.policy,
+                   "parallelism": "replicas" if world > 1 else "1 GPU",
+                   "l2": "matrix (~%.0f GB) >> 126 MB L2; no flush needed" % (n * n / 2 * 5 / 1e9)},
+        "joules_per_eval": None if joules is None else joules / args.steps,
+        "loglik": last.loglik, "tiles_fp64_fp32_fp16": list(last.tiles), "stc_tiles": last.stc_tiles,
+        "flops_update_per_class": upd,
+        "phase_ms": {"gen+map": last.t_gen_ms, "potrf": last.t_potrf_ms, "solve": last.t_solve_ms},
+        "profile": {k: {"ms_per_step": v["ms"] / args.steps, "launches_per_step": v["launches"] / args.steps,
+                        "tflops": (v["flops"] / (v["ms"] / 1e3) / 1e12) if v["ms"] > 0 and v["flops"] else None}
+                    for k, v in p.items()},
+        "update_roofline_fraction": roof_time_s / t_upd_s if t_upd_s > 0 else None,
+        "roofline": {"bound": "tensor", "kernel": "dgemm_nt_kernel (FP64 DMMA trailing update)",
+                     "achieved": achieved, "peak": fp64_peak, "unit": "TFLOP/s",
+                     "frac": achieved / fp64_peak if fp64_peak else None, "traffic": None,
+                     "peak_source": f"{peak_src} bf16_tflops_sustained x {FP64_NOMINAL}/{BF16_NOMINAL} (FP64 DMMA nominal / bf16 nominal)",
+                     "cublas_dgemm_tflops_live": cub, "frac_vs_cublas_dgemm": (achieved / cub) if cub else None},
+        "gpu_launches": launches,
+        "clocks": ck,
+        "e2e": e2e,
+    }
+    if world == 1 and not args.no_cpu_baseline:
+        out["cpu_baseline"] = cpu_baseline(cfg["map"])
+    print(json.dumps(out), flush=True)
+    if dist:
+        dist.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()
