@@ -513,7 +513,7 @@ static mp_status plan_potrf(mp_handle* h, mp_matrix* A, const uint8_t* km, const
     double* wb = A->at<double>(A->R.wbuf);
     double* wb2 = A->at<double>(A->R.wbuf2);
     int* d_info = h->d_info;
-    const bool use_tc = h->tc_mode != 0 && tc_gemm_available();
+    const bool use_tc = h->tc_mode != 0 && tc_gemm_available() && nb % 256 == 0;
     auto K = [&](int m, int k) { return km[(size_t)m * nt + k]; };
     auto C = [&](int m, int k) { return cm[(size_t)m * nt + k]; };
     const double fnb = (double)nb;

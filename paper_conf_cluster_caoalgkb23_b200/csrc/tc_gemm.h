@@ -1,6 +1,12 @@
-// K6 / K7 — tcgen05 tensor-core GEMMs for the FP32 class (3xTF32) and the FP16 class
-// (FP16 x FP16 -> FP32) trailing updates:  C_mn (FP32 tile) -= L_m L_n^T.
+// K6 / K7 — tcgen05 tensor-core GEMMs for the trailing update of FP32-class and FP16-class tiles
+// (GEMM(m,n,k) at kernel(m,n)):   C_mn (FP32 tile) -= L_mk L_nk^T
+//   FP16 class  (the paper's FP16_32): FP16 operands, FP32 accumulation in TMEM (kind::f16);
+//   FP32 class : 3xTF32 — hi = rna_tf32(a), lo = rna_tf32(a - hi), C -= hi.hi + hi.lo + lo.hi with
+//                an FP32 TMEM accumulator (kind::tf32), reading C13 in DESIGN.md.
+// Operands are the consumer-side conversions of the panel (K2), stored as [nt*nb][nb] row-major
+// caches and fetched with TMA (128-byte swizzle) into a multi-stage mbarrier pipeline.
 #pragma once
+#include <cuda.h>
 #include <cuda_fp16.h>
 #include <cuda_runtime.h>
 

@@ -78,3 +78,48 @@ def test_dgemm_rounded_operands_fp32_c(lib, rnd, npdt):
     Ar, Br = A.astype(npdt).astype(np.float64), B.astype(npdt).astype(np.float64)
     ref = (Cm.astype(np.float64) - Ar @ Br.T).astype(np.float32)
     assert np.max(np.abs(got.astype(np.float64) - ref)) <= 2 * np.max(np.abs(ref)) * 2.0**-24
+
+
+def tf32_rna(a32: np.ndarray) -> np.ndarray:
+    """cvt.rna.tf32.f32 written out: round the fp32 magnitude to 10 mantissa bits, ties away from zero."""
+    b = a32.astype(np.float32).view(np.uint32).astype(np.uint64)
+    b = ((b + 0x1000) & 0xFFFFE000).astype(np.uint32)
+    return b.view(np.float32)
+
+
+def test_tc_gemm_f16(lib):
+    assert lib.mp_tc_available() == 1
+    nb, nt = 512, 3
+    rng = np.random.default_rng(3)
+    P = (rng.standard_normal((nt * nb, nb)) * 0.1).astype(np.float16)
+    Cm = rng.standard_normal((nb, nb)).astype(np.float32)
+    dP, dC = dev(P), dev(Cm)
+    assert lib.mp_test_tc_gemm(2, C.c_void_p(dP.data_ptr()), None, C.c_void_p(dC.data_ptr()), nb, nt, 2, 0) == 0
+    got = dC.cpu().numpy().astype(np.float64)
+    Pd = P.astype(np.float64)
+    ref = Cm.astype(np.float64) - Pd[2 * nb:3 * nb] @ Pd[0:nb].T
+    err = np.max(np.abs(got - ref))
+    assert err <= 1e-5 * np.max(np.abs(ref)), err
+
+
+def test_tc_gemm_tf32x3_matches_sgemm_accuracy(lib):
+    """Reading C13 pin: 3xTF32 error vs an FP64 product <= 2x the SGEMM error on the same inputs."""
+    nb, nt = 512, 2
+    rng = np.random.default_rng(4)
+    A32 = rng.standard_normal((nt * nb, nb)).astype(np.float32)
+    hi = tf32_rna(A32)
+    lo = tf32_rna((A32 - hi).astype(np.float32))
+    Cm = np.zeros((nb, nb), np.float32)
+    dH, dL, dC = dev(hi), dev(lo), dev(Cm)
+    assert lib.mp_test_tc_gemm(1, C.c_void_p(dH.data_ptr()), C.c_void_p(dL.data_ptr()), C.c_void_p(dC.data_ptr()),
+                               nb, nt, 1, 0) == 0
+    got = -dC.cpu().numpy().astype(np.float64)
+    Ad = A32.astype(np.float64)
+    exact = Ad[nb:] @ Ad[:nb].T
+    sgemm = (A32[nb:] @ A32[:nb].T).astype(np.float64)
+    err_tc = np.linalg.norm(got - exact) / np.linalg.norm(exact)
+    err_sg = np.linalg.norm(sgemm - exact) / np.linalg.norm(exact)
+    single = (hi[nb:].astype(np.float64) @ hi[:nb].astype(np.float64).T)
+    err_1x = np.linalg.norm(single - exact) / np.linalg.norm(exact)
+    assert err_tc <= 2 * err_sg + 1e-9, (err_tc, err_sg)
+    assert err_tc < err_1x / 50  # far better than a single TF32 product
