@@ -9,12 +9,12 @@
 //
 // There is no tcgen05 kind::f64 on sm_100a; FP64 tensor-core math is the warp-level
 // mma.sync.m16n8k4.f64 (SASS DMMA).  Design:
-//   * CTA tile 128 x 128 x 16, 256 threads = 8 warps (2 x 4), warp tile 64 x 32,
+//   * CTA tile 128 x 128 x 32, 256 threads = 8 warps (2 x 4), warp tile 64 x 32,
 //     16 DMMA m16n8k4 per k4-step held in 64 FP64 accumulators per thread;
-//   * 4-stage cp.async (LDGSTS) pipeline, 16-byte chunks, zero-fill past M / N;
-//   * shared tiles are [128][16] doubles with the 16-byte chunk index XOR-swizzled
-//     by (row & 7): every fragment load (8 rows x 4 doubles per warp) is exactly
-//     two 128-byte wavefronts, the minimum for 256 bytes;
+//   * 3-stage cp.async (LDGSTS) pipeline (192 KB), 16-byte chunks, zero-fill past M / N;
+//   * shared tiles are [128][32] doubles with the 16-byte chunk index XOR-swizzled
+//     by 2*(row & 3) (see dg_swz): every fragment load is two 128-byte wavefronts, the
+//     minimum for 256 bytes; fragments are double-buffered in registers;
 //   * optional operand rounding to FP32 / FP16 (the FP32- and FP16-class GEMM of
 //     P:146 evaluated as FP64 arithmetic on rounded operands) and an FP32 C tile.
 // Jobs of one launch are laid out job-major so the CTAs resident at one time share
@@ -24,12 +24,17 @@
 
 namespace mpgeo {
 
-constexpr int DG_BM = 128, DG_BN = 128, DG_BK = 16, DG_STAGES = 4, DG_THREADS = 256;
+constexpr int DG_BM = 128, DG_BN = 128, DG_BK = 32, DG_STAGES = 3, DG_THREADS = 256;
+constexpr int DG_CH = DG_BK / 2;  // 16-byte chunks per smem row
 constexpr int DG_STAGE_ELEMS = (DG_BM + DG_BN) * DG_BK;  // doubles per stage
-constexpr int DG_SMEM = DG_STAGES * DG_STAGE_ELEMS * 8;  // 128 KB
+constexpr int DG_SMEM = DG_STAGES * DG_STAGE_ELEMS * 8;  // 192 KB
 
+// 16-byte chunk c of row r lives at chunk c ^ ((r & 3) << 1).  A DMMA fragment load reads 8 rows
+// (g = lane / 4) x 2 chunks; 64-bit shared loads are served per half-warp (g = 0..3 and 4..7), and
+// within a half-warp the 8 (row, chunk) pairs land on 8 distinct 16-byte bank groups: 2 wavefronts
+// per warp load, the minimum for 256 bytes.
 __device__ __forceinline__ int dg_swz(int row, int col) {
-    return row * DG_BK + ((((col >> 1) ^ (row & 7))) << 1) + (col & 1);
+    return row * DG_BK + ((((col >> 1) ^ ((row & 3) << 1))) << 1) + (col & 1);
 }
 
 __device__ __forceinline__ void cp_async16(void* smem, const void* gmem, bool valid) {
@@ -82,21 +87,23 @@ __global__ void __launch_bounds__(DG_THREADS, 1) dgemm_nt_kernel(DgemmArgs p) {
     const double* __restrict__ B = (const double*)jb.B;
     const int bm = bi * DG_BM, bn = bj * DG_BN;
 
-    // ---- loader: 1024 16-byte chunks per operand per stage, 4 per thread per operand
+    // ---- loader: BM x BK/2 16-byte chunks per operand per stage (zero-fill past M, N, K)
     auto load_stage = [&](int stage, int kt) {
         double* As = smem + stage * DG_STAGE_ELEMS;
         double* Bs = As + DG_BM * DG_BK;
         const int k0 = kt * DG_BK;
 #pragma unroll
-        for (int i = 0; i < 4; ++i) {
+        for (int i = 0; i < DG_BM * DG_CH / DG_THREADS; ++i) {
             const int c = tid + i * DG_THREADS;
-            const int row = c >> 3, ch = c & 7;
+            const int row = c / DG_CH, ch = c % DG_CH;
             const int ra = bm + row, rb = bn + row;
-            const bool va = ra < p.M, vb = rb < p.N;
-            const double* ga = A + (size_t)(va ? ra : 0) * p.lda + k0 + ch * 2;
-            const double* gb = B + (size_t)(vb ? rb : 0) * p.ldb + k0 + ch * 2;
-            cp_async16(As + row * DG_BK + ((ch ^ (row & 7)) << 1), ga, va);
-            cp_async16(Bs + row * DG_BK + ((ch ^ (row & 7)) << 1), gb, vb);
+            const bool kv = k0 + ch * 2 < p.K;  // K is even: a chunk is all-in or all-out
+            const bool va = ra < p.M && kv, vb = rb < p.N && kv;
+            const double* ga = va ? A + (size_t)ra * p.lda + k0 + ch * 2 : A;
+            const double* gb = vb ? B + (size_t)rb * p.ldb + k0 + ch * 2 : B;
+            const int sw = (ch ^ ((row & 3) << 1)) << 1;
+            cp_async16(As + row * DG_BK + sw, ga, va);
+            cp_async16(Bs + row * DG_BK + sw, gb, vb);
         }
     };
 
@@ -108,7 +115,7 @@ __global__ void __launch_bounds__(DG_THREADS, 1) dgemm_nt_kernel(DgemmArgs p) {
 #pragma unroll
             for (int r = 0; r < 4; ++r) acc[i][j][r] = 0.0;
 
-    const int KT = p.K / DG_BK;
+    const int KT = (p.K + DG_BK - 1) / DG_BK;  // zero-filled past K
 #pragma unroll
     for (int s = 0; s < DG_STAGES - 1; ++s) {
         if (s < KT) load_stage(s, s);
@@ -125,22 +132,27 @@ __global__ void __launch_bounds__(DG_THREADS, 1) dgemm_nt_kernel(DgemmArgs p) {
         }
         const double* As = smem + (kt % DG_STAGES) * DG_STAGE_ELEMS;
         const double* Bs = As + DG_BM * DG_BK;
-#pragma unroll
-        for (int ks = 0; ks < DG_BK / 4; ++ks) {
+        // fragments double-buffered across k4-steps: loads of step ks+1 overlap the DMMAs of ks
+        double a[2][4][2], b[2][4];
+        auto load_frag = [&](int buf, int ks) {
             const int kk = ks * 4 + t;
-            double a[4][2], b[4];
 #pragma unroll
             for (int i = 0; i < 4; ++i) {
                 const int r = wm * 64 + i * 16 + g;
-                a[i][0] = ld_op<ROUND>(As + dg_swz(r, kk));
-                a[i][1] = ld_op<ROUND>(As + dg_swz(r + 8, kk));
+                a[buf][i][0] = ld_op<ROUND>(As + dg_swz(r, kk));
+                a[buf][i][1] = ld_op<ROUND>(As + dg_swz(r + 8, kk));
             }
 #pragma unroll
-            for (int j = 0; j < 4; ++j) b[j] = ld_op<ROUND>(Bs + dg_swz(wn * 32 + j * 8 + g, kk));
+            for (int j = 0; j < 4; ++j) b[buf][j] = ld_op<ROUND>(Bs + dg_swz(wn * 32 + j * 8 + g, kk));
+        };
+        load_frag(0, 0);
+#pragma unroll
+        for (int ks = 0; ks < DG_BK / 4; ++ks) {
+            if (ks + 1 < DG_BK / 4) load_frag((ks + 1) & 1, ks + 1);
 #pragma unroll
             for (int i = 0; i < 4; ++i)
 #pragma unroll
-                for (int j = 0; j < 4; ++j) dmma_16x8x4(acc[i][j], a[i], b[j]);
+                for (int j = 0; j < 4; ++j) dmma_16x8x4(acc[i][j], a[ks & 1][i], b[ks & 1][j]);
         }
     }
     cp_async_wait<0>();
@@ -203,7 +215,7 @@ static cudaError_t launch_one(const DgemmArgs& a, long long grid, cudaStream_t s
 
 cudaError_t dgemm_nt_launch(DgemmArgs a, int njobs, int round_ops, bool c_f32, cudaStream_t s) {
     if (njobs <= 0 || a.M <= 0 || a.N <= 0 || a.K <= 0) return cudaSuccess;
-    if (a.K % DG_BK) return cudaErrorInvalidValue;
+    if (a.K % 16) return cudaErrorInvalidValue;
     a.tiles_m = (a.M + DG_BM - 1) / DG_BM;
     a.tiles_n = (a.N + DG_BN - 1) / DG_BN;
     if (a.lower) {
