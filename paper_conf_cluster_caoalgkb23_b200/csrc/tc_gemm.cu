@@ -12,7 +12,8 @@
 //                    C -= acc with 16-byte loads/stores of the row.
 // KIND 0 (FP16 class, "FP16_32"): kind::f16, BN = 256, BK = 64, 4 stages (48 KB each).
 // KIND 1 (FP32 class, 3xTF32, reading C13): kind::tf32, BN = 128, BK = 32, 3 stages of
-//   {A_hi, A_lo, B_hi, B_lo} (64 KB); per k-step three MMAs hi.hi + hi.lo + lo.hi into one accumulator.
+//   {A_hi, A_lo, B_hi, B_lo} (64 KB); per k-step three MMAs lo.hi + hi.lo + hi.hi; K is split in
+//   chunks of 64 accumulated in two ping-pong TMEM accumulators and summed by the epilogue in FP32.
 #include <cudaTypedefs.h>
 #include <stdint.h>
 #include <string.h>
@@ -41,7 +42,11 @@ struct TcCfg {
     static constexpr int STAGE_BYTES = KIND == 0 ? A_BYTES + B_BYTES : 2 * (A_BYTES + B_BYTES);
     static constexpr int STAGES = KIND == 0 ? 4 : 3;
     static constexpr int SMEM = STAGES * STAGE_BYTES + 1024;
-    static constexpr uint32_t TMEM_COLS = BN;  // power of two >= 32
+    // KIND 1: accumulate CHUNK_KB k-blocks (64 of K) per TMEM accumulator, two accumulators
+    // ping-pong; the epilogue sums the chunks in FP32 registers (round-to-nearest), which keeps
+    // the tensor core's non-RN FP32 accumulation error from growing with K (reading C13).
+    static constexpr int CHUNK_KB = KIND == 0 ? 1 << 20 : 2;
+    static constexpr uint32_t TMEM_COLS = KIND == 0 ? BN : 2 * BN;  // power of two >= 32
     // instruction descriptor: D = F32 (bit 4), A/B format (bits 7-9 / 10-12), K-major both,
     // N >> 3 (bits 17-22), M >> 4 (bits 24-28)
     static constexpr uint32_t IDESC = (1u << 4) | ((KIND == 0 ? 0u : 2u) << 7) | ((KIND == 0 ? 0u : 2u) << 10) |
@@ -121,6 +126,7 @@ __global__ void __launch_bounds__(TC_THREADS, 1) tc_gemm_kernel(const __grid_con
     extern __shared__ uint8_t smem_raw[];
     uint8_t* smem = (uint8_t*)(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
     __shared__ __align__(8) uint64_t full_bar[Cfg::STAGES], empty_bar[Cfg::STAGES], done_bar;
+    __shared__ __align__(8) uint64_t acc_full[2], acc_empty[2];
     __shared__ uint32_t tmem_slot;
 
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
@@ -138,6 +144,10 @@ __global__ void __launch_bounds__(TC_THREADS, 1) tc_gemm_kernel(const __grid_con
             mbar_init(smem_u32(&empty_bar[s]), 1);
         }
         mbar_init(smem_u32(&done_bar), 1);
+        for (int i = 0; i < 2; ++i) {
+            mbar_init(smem_u32(&acc_full[i]), 1);
+            mbar_init(smem_u32(&acc_empty[i]), 4);  // one arrive per epilogue warp
+        }
         asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
         asm volatile("prefetch.tensormap [%0];" ::"l"((uint64_t)&p.a) : "memory");
         asm volatile("prefetch.tensormap [%0];" ::"l"((uint64_t)&p.b) : "memory");
@@ -178,48 +188,90 @@ __global__ void __launch_bounds__(TC_THREADS, 1) tc_gemm_kernel(const __grid_con
         for (int kb = 0; kb < KB; ++kb) {
             const int s = kb % Cfg::STAGES;
             const uint32_t ph = (uint32_t)(kb / Cfg::STAGES) & 1u;
+            const int chunk = kb / Cfg::CHUNK_KB, kin = kb % Cfg::CHUNK_KB;
+            const uint32_t abuf = (uint32_t)(chunk & 1);
+            const uint32_t dacc = KIND == 0 ? tmem : tmem + abuf * Cfg::BN;
+            if (KIND == 1 && kin == 0) {  // wait until the epilogue drained this accumulator
+                mbar_wait(smem_u32(&acc_empty[abuf]), ((uint32_t)(chunk >> 1) & 1u) ^ 1u);
+                tc_fence_after();
+            }
             mbar_wait(smem_u32(&full_bar[s]), ph);
             tc_fence_after();
             const uint32_t base = smem_u32(smem + s * Cfg::STAGE_BYTES);
 #pragma unroll
             for (int k = 0; k < Cfg::BK / Cfg::UK; ++k) {
                 const uint32_t koff = k * 32;  // bytes along K inside the 128-byte swizzle atom
-                const uint32_t acc = (kb | k) != 0;
+                const uint32_t acc = (kin | k) != 0;
                 if (KIND == 0) {
-                    tc_mma<0>(tmem, desc_sw128(base + koff), desc_sw128(base + Cfg::A_BYTES + koff), acc);
+                    tc_mma<0>(dacc, desc_sw128(base + koff), desc_sw128(base + Cfg::A_BYTES + koff), acc);
                 } else {
                     const uint64_t ahi = desc_sw128(base + koff);
                     const uint64_t alo = desc_sw128(base + Cfg::A_BYTES + koff);
                     const uint64_t bhi = desc_sw128(base + 2 * Cfg::A_BYTES + koff);
                     const uint64_t blo = desc_sw128(base + 2 * Cfg::A_BYTES + Cfg::B_BYTES + koff);
-                    tc_mma<1>(tmem, alo, bhi, acc);  // small terms first
-                    tc_mma<1>(tmem, ahi, blo, 1u);
-                    tc_mma<1>(tmem, ahi, bhi, 1u);
+                    tc_mma<1>(dacc, alo, bhi, acc);  // small terms first
+                    tc_mma<1>(dacc, ahi, blo, 1u);
+                    tc_mma<1>(dacc, ahi, bhi, 1u);
                 }
             }
             tc_commit(smem_u32(&empty_bar[s]));
+            if (KIND == 1 && (kin == Cfg::CHUNK_KB - 1 || kb == KB - 1)) tc_commit(smem_u32(&acc_full[abuf]));
         }
-        tc_commit(smem_u32(&done_bar));
+        if (KIND == 0) tc_commit(smem_u32(&done_bar));
     } else if (warp >= 4) {
         // ---------------- epilogue: C -= acc
-        mbar_wait(smem_u32(&done_bar), 0);
-        tc_fence_after();
         const int q = warp - 4;
         const int row = bi * TC_BM + q * 32 + lane;
         float* crow = jb.C + (size_t)row * p.nb + bj * Cfg::BN;
+        const uint32_t tl = (uint32_t)(q * 32) << 16;
+        if (KIND == 0) {
+            mbar_wait(smem_u32(&done_bar), 0);
+            tc_fence_after();
 #pragma unroll 1
-        for (int c0 = 0; c0 < Cfg::BN; c0 += 32) {
-            uint32_t r[32];
-            tmem_ld32(tmem + ((uint32_t)(q * 32) << 16) + (uint32_t)c0, r);
-            float4* cp = (float4*)(crow + c0);
+            for (int c0 = 0; c0 < Cfg::BN; c0 += 32) {
+                uint32_t r[32];
+                tmem_ld32(tmem + tl + (uint32_t)c0, r);
+                float4* cp = (float4*)(crow + c0);
 #pragma unroll
-            for (int v = 0; v < 8; ++v) {
-                float4 c = cp[v];
-                c.x -= __uint_as_float(r[4 * v + 0]);
-                c.y -= __uint_as_float(r[4 * v + 1]);
-                c.z -= __uint_as_float(r[4 * v + 2]);
-                c.w -= __uint_as_float(r[4 * v + 3]);
-                cp[v] = c;
+                for (int v = 0; v < 8; ++v) {
+                    float4 c = cp[v];
+                    c.x -= __uint_as_float(r[4 * v + 0]);
+                    c.y -= __uint_as_float(r[4 * v + 1]);
+                    c.z -= __uint_as_float(r[4 * v + 2]);
+                    c.w -= __uint_as_float(r[4 * v + 3]);
+                    cp[v] = c;
+                }
+            }
+        } else {
+            float sum[Cfg::BN];
+#pragma unroll
+            for (int i = 0; i < Cfg::BN; ++i) sum[i] = 0.f;
+            const int nchunks = (KB + Cfg::CHUNK_KB - 1) / Cfg::CHUNK_KB;
+#pragma unroll 1
+            for (int c = 0; c < nchunks; ++c) {
+                const uint32_t abuf = (uint32_t)(c & 1);
+                mbar_wait(smem_u32(&acc_full[abuf]), (uint32_t)(c >> 1) & 1u);
+                tc_fence_after();
+#pragma unroll
+                for (int c0 = 0; c0 < Cfg::BN; c0 += 32) {
+                    uint32_t r[32];
+                    tmem_ld32(tmem + tl + abuf * Cfg::BN + (uint32_t)c0, r);
+#pragma unroll
+                    for (int v = 0; v < 32; ++v) sum[c0 + v] += __uint_as_float(r[v]);
+                }
+                tc_fence_before();
+                __syncwarp();
+                if (lane == 0) asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(&acc_empty[abuf])) : "memory");
+            }
+#pragma unroll
+            for (int c0 = 0; c0 < Cfg::BN; c0 += 4) {
+                float4* cp = (float4*)(crow + c0);
+                float4 cv = *cp;
+                cv.x -= sum[c0];
+                cv.y -= sum[c0 + 1];
+                cv.z -= sum[c0 + 2];
+                cv.w -= sum[c0 + 3];
+                *cp = cv;
             }
         }
     }
