@@ -67,6 +67,9 @@ struct mp_handle {
     cudaEvent_t ev[8] = {};
     bool broken = false;
     int tc_mode = 1;  // 1: tcgen05 kernels for FP32/FP16 classes when available, 0: DMMA emulation
+    int lookahead = 1;  // 1: panel k+1 on the high-priority panel stream overlaps update k
+    cudaStream_t pstream = nullptr;
+    std::vector<cudaEvent_t> sync_ev;
     // profiling (mp_set_profiling): event pairs per launch, resolved in mp_get_profile
     bool profiling = false;
     std::vector<cudaEvent_t> prof_pool;
@@ -158,10 +161,11 @@ static Regions layout(const mp_matrix* A, const uint8_t* storage) {
     R.ltilde = take(nb2 * 8);
     R.wbuf = take((size_t)POTRF_IB * POTRF_IB * 8);
     R.wbuf2 = take((size_t)ceil_div(A->nb, POTRF_IB) * POTRF_IB * POTRF_IB * 8);
-    R.p64 = take((size_t)nt * nb2 * 8);
-    R.p16 = take((size_t)nt * nb2 * 2);
-    R.phi = take((size_t)nt * nb2 * 4);
-    R.plo = take((size_t)nt * nb2 * 4);
+    // two sets of panel buffers (panel parity) so panel k+1 can be produced while update k reads panel k
+    R.p64 = take(2 * (size_t)nt * nb2 * 8);
+    R.p16 = take(2 * (size_t)nt * nb2 * 2);
+    R.phi = take(2 * (size_t)nt * nb2 * 4);
+    R.plo = take(2 * (size_t)nt * nb2 * 4);
     R.tile_off.assign((size_t)nt * nt, SIZE_MAX);
     for (int k = 0; k < nt; ++k)
         for (int m = k; m < nt; ++m)
@@ -194,7 +198,12 @@ struct Op {
     std::function<cudaError_t(cudaStream_t)> fn;
     int cls;
     double flops;
+    int stream = 0;  // 0: the handle's stream, 1: the high-priority panel stream (lookahead)
+    int kind = 0;    // 0: launch, 1: record event `ev` on `stream`, 2: make `stream` wait for `ev`
+    int ev = -1;
 };
+static Op op_record(int stream, int ev) { Op o{nullptr, 0, 0}; o.stream = stream; o.kind = 1; o.ev = ev; return o; }
+static Op op_wait(int stream, int ev) { Op o{nullptr, 0, 0}; o.stream = stream; o.kind = 2; o.ev = ev; return o; }
 enum { C_UPD64 = 0, C_UPD32 = 1, C_UPD16 = 2, C_POTRF = 3, C_TRSM = 4, C_CONV = 5, C_GEN = 6, C_SOLVE = 7 };
 
 static cudaEvent_t prof_event(mp_handle* h) {
@@ -211,15 +220,31 @@ static mp_status run_plan(mp_handle* h, mp_matrix* A, Arena& ar, std::vector<Op>
         FAIL(h, MP_ERR_NOMEM, "control arena overflow (%zu > %zu)", ar.host.size(), A->R.ctrl_bytes);
     if (!ar.host.empty())
         CK(h, cudaMemcpyAsync(ar.dev_base, ar.host.data(), ar.host.size(), cudaMemcpyHostToDevice, h->stream));
+    int max_ev = -1;
+    for (auto& op : ops) max_ev = std::max(max_ev, op.ev);
+    while ((int)h->sync_ev.size() <= max_ev) {
+        cudaEvent_t e;
+        CK(h, cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
+        h->sync_ev.push_back(e);
+    }
     for (auto& op : ops) {
+        cudaStream_t st = op.stream ? h->pstream : h->stream;
+        if (op.kind == 1) {
+            CK(h, cudaEventRecord(h->sync_ev[op.ev], st));
+            continue;
+        }
+        if (op.kind == 2) {
+            CK(h, cudaStreamWaitEvent(st, h->sync_ev[op.ev], 0));
+            continue;
+        }
         if (h->profiling) {
             cudaEvent_t e0 = prof_event(h), e1 = prof_event(h);
-            CK(h, cudaEventRecord(e0, h->stream));
-            CK(h, op.fn(h->stream));
-            CK(h, cudaEventRecord(e1, h->stream));
+            CK(h, cudaEventRecord(e0, st));
+            CK(h, op.fn(st));
+            CK(h, cudaEventRecord(e1, st));
             h->prof_pending.push_back(ProfRec{e0, e1, op.cls, op.flops});
         } else {
-            CK(h, op.fn(h->stream));
+            CK(h, op.fn(st));
         }
         h->launches++;
     }
@@ -251,6 +276,7 @@ mp_status mp_init(int device, int rank, int nranks, int P, int Q, const uint8_t*
     h->P = P;
     h->Q = Q;
     if (const char* e = getenv("MPGEO_TC")) h->tc_mode = atoi(e);
+    if (const char* e = getenv("MPGEO_LOOKAHEAD")) h->lookahead = atoi(e);
     auto fail = [&](mp_status s) {
         if (h->own_stream && h->stream) cudaStreamDestroy(h->stream);
         delete h;
@@ -263,6 +289,11 @@ mp_status mp_init(int device, int rank, int nranks, int P, int Q, const uint8_t*
     } else {
         if (cudaStreamCreateWithFlags(&h->stream, cudaStreamNonBlocking) != cudaSuccess) return fail(MP_ERR_CUDA);
         h->own_stream = true;
+    }
+    {
+        int lo = 0, hi = 0;
+        cudaDeviceGetStreamPriorityRange(&lo, &hi);
+        if (cudaStreamCreateWithPriority(&h->pstream, cudaStreamNonBlocking, hi) != cudaSuccess) return fail(MP_ERR_CUDA);
     }
     if (cudaMalloc(&h->d_info, sizeof(int)) != cudaSuccess) return fail(MP_ERR_CUDA);
     for (auto& e : h->ev)
@@ -286,6 +317,9 @@ mp_status mp_finalize(mp_handle* h) {
         if (e) cudaEventDestroy(e);
     for (auto& e : h->prof_pool)
         if (e) cudaEventDestroy(e);
+    for (auto& e : h->sync_ev)
+        if (e) cudaEventDestroy(e);
+    if (h->pstream) cudaStreamDestroy(h->pstream);
     if (h->d_info) cudaFree(h->d_info);
     if (h->own_stream) cudaStreamDestroy(h->stream);
     delete h;
@@ -503,12 +537,12 @@ struct FlopCount {
 
 static mp_status plan_potrf(mp_handle* h, mp_matrix* A, const uint8_t* km, const uint8_t* cm, Arena& ar,
                             std::vector<Op>& ops, FlopCount& fc) {
-    const int nt = A->nt, nb = A->nb, IB = POTRF_IB;
+    const int nt = A->nt, nb = A->nb, IB = POTRF_IB, OB = 4 * POTRF_IB;
     const size_t nb2 = A->nb2();
-    double* p64 = A->at<double>(A->R.p64);
-    __half* p16 = A->at<__half>(A->R.p16);
-    float* phi = A->at<float>(A->R.phi);
-    float* plo = A->at<float>(A->R.plo);
+    double* const p64b = A->at<double>(A->R.p64);
+    __half* const p16b = A->at<__half>(A->R.p16);
+    float* const phib = A->at<float>(A->R.phi);
+    float* const plob = A->at<float>(A->R.plo);
     double* ltil = A->at<double>(A->R.ltilde);
     double* wb = A->at<double>(A->R.wbuf);
     double* wb2 = A->at<double>(A->R.wbuf2);
@@ -518,6 +552,10 @@ static mp_status plan_potrf(mp_handle* h, mp_matrix* A, const uint8_t* km, const
     auto C = [&](int m, int k) { return cm[(size_t)m * nt + k]; };
     const double fnb = (double)nb;
 
+    // per step: panel(k) = POTRF + TRSM + conversion; next(k) = the update of column k+1 (what
+    // panel k+1 waits for); rest(k) = the rest of the trailing update
+    std::vector<std::vector<Op>> pan(nt), nxt(nt), rst(nt);
+    std::vector<Op>* cur = nullptr;
     auto gemm = [&](std::vector<GemmJob>& jobs, int M, int N, int Kd, int lda, int ldb, int ldc, int lower,
                     double alpha, double beta, int round, bool cf32, int cls, double flops_per_job) {
         if (jobs.empty()) return;
@@ -534,28 +572,48 @@ static mp_status plan_potrf(mp_handle* h, mp_matrix* A, const uint8_t* km, const
         g.alpha = alpha;
         g.beta = beta;
         const int nj = (int)jobs.size();
-        ops.push_back({[=](cudaStream_t s) { return dgemm_nt_launch(g, nj, round, cf32, s); }, cls, flops_per_job * nj});
+        cur->push_back({[=](cudaStream_t s) { return dgemm_nt_launch(g, nj, round, cf32, s); }, cls, flops_per_job * nj});
     };
 
     for (int k = 0; k < nt; ++k) {
-        // ---- 1. DPOTRF(k,k), FP64
+        const size_t set = h->lookahead ? (size_t)(k & 1) : 0;
+        double* p64 = p64b + set * nt * nb2;
+        __half* p16 = p16b + set * nt * nb2;
+        float* phi = phib + set * nt * nb2;
+        float* plo = plob + set * nt * nb2;
+        cur = &pan[k];
+        // ---- 1. DPOTRF(k,k), FP64: two-level blocking — 128-column blocks
+        //      (diagonal block Cholesky + inverse, block column as GEMM with the inverse, update
+        //      inside the 512-column outer block), then one K = 512 SYRK per outer block.
         if (A->mine(k, k)) {
             double* Akk = (double*)A->tile(k, k);
-            for (int j0 = 0; j0 < nb; j0 += IB) {
-                const int jb = std::min(IB, nb - j0);
-                double* blk = Akk + (size_t)j0 * nb + j0;
-                const int col0 = k * nb + j0;
-                ops.push_back({[=](cudaStream_t s) { return potrf_diag_block_launch(blk, nb, jb, wb, col0, d_info, s); }, C_POTRF, (double)jb * jb * jb / 3.0});
-                const int rest = nb - j0 - jb;
-                if (rest > 0) {
-                    double* X = Akk + (size_t)(j0 + jb) * nb + j0;
+            for (int J0 = 0; J0 < nb; J0 += OB) {
+                const int Jend = std::min(nb, J0 + OB), Jb = Jend - J0;
+                for (int j0 = J0; j0 < Jend; j0 += IB) {
+                    const int jb = std::min(IB, Jend - j0), jend = j0 + jb;
+                    double* blk = Akk + (size_t)j0 * nb + j0;
+                    const int col0 = k * nb + j0;
+                    cur->push_back({[=](cudaStream_t s) { return potrf_diag_block_launch(blk, nb, jb, wb, col0, d_info, s); },
+                                   C_POTRF, (double)jb * jb * jb / 3.0});
+                    const int rest = nb - jend;
+                    if (rest <= 0) continue;
+                    double* X = Akk + (size_t)jend * nb + j0;
                     std::vector<GemmJob> j1{GemmJob{X, wb, X}};
                     gemm(j1, rest, jb, jb, nb, IB, nb, 0, 1.0, 0.0, P64, false, C_POTRF, (double)rest * jb * jb);
-                    std::vector<GemmJob> j2{GemmJob{X, X, Akk + (size_t)(j0 + jb) * nb + j0 + jb}};
-                    gemm(j2, rest, rest, jb, nb, nb, nb, 1, -1.0, 1.0, P64, false, C_POTRF, (double)rest * rest * jb);
+                    if (Jend > jend) {
+                        std::vector<GemmJob> j2{GemmJob{X, X, Akk + (size_t)jend * nb + jend}};
+                        gemm(j2, rest, Jend - jend, jb, nb, nb, nb, 0, -1.0, 1.0, P64, false, C_POTRF,
+                             2.0 * rest * (Jend - jend) * jb);
+                    }
+                }
+                const int rest = nb - Jend;
+                if (rest > 0) {
+                    double* Y = Akk + (size_t)Jend * nb + J0;
+                    std::vector<GemmJob> j3{GemmJob{Y, Y, Akk + (size_t)Jend * nb + Jend}};
+                    gemm(j3, rest, rest, Jb, nb, nb, nb, 1, -1.0, 1.0, P64, false, C_POTRF, (double)rest * rest * Jb);
                 }
             }
-            ops.push_back({[=](cudaStream_t s) { return zero_upper_launch(Akk, nb, s); }, C_POTRF, 0});
+            cur->push_back({[=](cudaStream_t s) { return zero_upper_launch(Akk, nb, s); }, C_POTRF, 0});
             fc.potrf += fnb * fnb * fnb / 3.0;
         }
         if (k == nt - 1) break;
@@ -563,8 +621,8 @@ static mp_status plan_potrf(mp_handle* h, mp_matrix* A, const uint8_t* km, const
         {
             double* Akk = (double*)A->tile(k, k);
             const int pc = C(k, k);
-            ops.push_back({[=](cudaStream_t s) { return round_copy_launch(Akk, ltil, (int64_t)nb2, pc, s); }, C_TRSM, 0});
-            ops.push_back({[=](cudaStream_t s) { return trtri_blocks_launch(ltil, nb, wb2, s); }, C_TRSM, 0});
+            cur->push_back({[=](cudaStream_t s) { return round_copy_launch(Akk, ltil, (int64_t)nb2, pc, s); }, C_TRSM, 0});
+            cur->push_back({[=](cudaStream_t s) { return trtri_blocks_launch(ltil, nb, wb2, s); }, C_TRSM, 0});
         }
         // ---- 3. panel in
         std::vector<PanelTile> pin, pout;
@@ -599,33 +657,45 @@ static mp_status plan_potrf(mp_handle* h, mp_matrix* A, const uint8_t* km, const
             PanelTile* d_in = ar.push(pin);
             PanelTile* d_out = ar.push(pout);
             const int np = (int)pin.size();
-            ops.push_back({[=](cudaStream_t s) { return panel_in_launch(d_in, np, (int64_t)nb2, s); }, C_CONV, 0});
-            // ---- 4. TRSM(m,k): L_mk = A_mk L~_kk^{-T}, FP64 arithmetic (reading C12')
-            for (int j0 = 0; j0 < nb; j0 += IB) {
-                const int jb = std::min(IB, nb - j0);
-                std::vector<GemmJob> ja, jbv;
-                for (auto& t : pin) {
-                    ja.push_back(GemmJob{t.p64 + j0, wb2 + (size_t)(j0 / IB) * IB * IB, t.p64 + j0});
-                    if (j0 + jb < nb)
-                        jbv.push_back(GemmJob{t.p64 + j0, ltil + (size_t)(j0 + jb) * nb + j0, t.p64 + j0 + jb});
+            cur->push_back({[=](cudaStream_t s) { return panel_in_launch(d_in, np, (int64_t)nb2, s); }, C_CONV, 0});
+            // ---- 4. TRSM(m,k): L_mk = A_mk L~_kk^{-T}, FP64 arithmetic (reading C12'),
+            //      right-looking over 128-column blocks (X_j = X_j W_j^T) with the updates inside a
+            //      512-column outer block at K = 128 and across outer blocks at K = 512.
+            for (int J0 = 0; J0 < nb; J0 += OB) {
+                const int Jend = std::min(nb, J0 + OB), Jb = Jend - J0;
+                for (int j0 = J0; j0 < Jend; j0 += IB) {
+                    const int jb = std::min(IB, Jend - j0), jend = j0 + jb;
+                    std::vector<GemmJob> ja, jin;
+                    for (auto& t : pin) {
+                        ja.push_back(GemmJob{t.p64 + j0, wb2 + (size_t)(j0 / IB) * IB * IB, t.p64 + j0});
+                        if (Jend > jend) jin.push_back(GemmJob{t.p64 + j0, ltil + (size_t)jend * nb + j0, t.p64 + jend});
+                    }
+                    gemm(ja, nb, jb, jb, nb, IB, nb, 0, 1.0, 0.0, P64, false, C_TRSM, fnb * jb * jb);
+                    gemm(jin, nb, Jend - jend, jb, nb, nb, nb, 0, -1.0, 1.0, P64, false, C_TRSM, 2.0 * fnb * (Jend - jend) * jb);
                 }
-                gemm(ja, nb, jb, jb, nb, IB, nb, 0, 1.0, 0.0, P64, false, C_TRSM, fnb * jb * jb);
-                gemm(jbv, nb, nb - j0 - jb, jb, nb, nb, nb, 0, -1.0, 1.0, P64, false, C_TRSM, 2.0 * fnb * (nb - j0 - jb) * jb);
+                if (nb > Jend) {
+                    std::vector<GemmJob> jo;
+                    for (auto& t : pin) jo.push_back(GemmJob{t.p64 + J0, ltil + (size_t)Jend * nb + J0, t.p64 + Jend});
+                    gemm(jo, nb, nb - Jend, Jb, nb, nb, nb, 0, -1.0, 1.0, P64, false, C_TRSM, 2.0 * fnb * (nb - Jend) * Jb);
+                }
             }
             fc.trsm += np * fnb * fnb * fnb;
             // ---- 5. panel out (K2)
-            ops.push_back({[=](cudaStream_t s) { return panel_out_launch(d_out, np, (int64_t)nb2, s); }, C_CONV, 0});
+            cur->push_back({[=](cudaStream_t s) { return panel_out_launch(d_out, np, (int64_t)nb2, s); }, C_CONV, 0});
         }
-        // ---- 6. trailing update: SYRK + GEMM grouped by kernel(m,n)
+        // ---- 6. trailing update: SYRK + GEMM grouped by kernel(m,n); the tiles of
+        //      column k+1 (next) are emitted separately so panel k+1 can start as soon as they are done
+        for (int part = 0; part < 2; ++part) {
+        cur = part == 0 ? &nxt[k] : &rst[k];
         std::vector<GemmJob> syrk, g64, g32, g16;
         std::vector<TcJob> t32, t16;
         for (int m = k + 1; m < nt; ++m) {
-            if (A->mine(m, m)) {
+            if (A->mine(m, m) && ((m == k + 1) == (part == 0))) {
                 syrk.push_back(GemmJob{p64 + (size_t)m * nb2, p64 + (size_t)m * nb2, A->tile(m, m)});
                 fc.upd[MP_FP64] += fnb * fnb * fnb;
             }
             for (int n = k + 1; n < m; ++n) {
-                if (!A->mine(m, n)) continue;
+                if (!A->mine(m, n) || ((n == k + 1) != (part == 0))) continue;
                 const int p = K(m, n);
                 fc.upd[p] += 2.0 * fnb * fnb * fnb;
                 if (p == MP_FP64) {
@@ -646,16 +716,45 @@ static mp_status plan_potrf(mp_handle* h, mp_matrix* A, const uint8_t* km, const
             TcJob* dj = ar.push(t32);
             const int nj = (int)t32.size();
             TcArgs ta{dj, phi, plo, nb, nt};
-            ops.push_back({[=](cudaStream_t s) { return tc_gemm_tf32x3_launch(ta, nj, s); }, C_UPD32, 2 * f3 * nj});
+            cur->push_back({[=](cudaStream_t s) { return tc_gemm_tf32x3_launch(ta, nj, s); }, C_UPD32, 2 * f3 * nj});
         }
         if (!t16.empty()) {
             TcJob* dj = ar.push(t16);
             const int nj = (int)t16.size();
             TcArgs ta{dj, nullptr, nullptr, nb, nt};
             ta.p16 = p16;
-            ops.push_back({[=](cudaStream_t s) { return tc_gemm_f16_launch(ta, nj, s); }, C_UPD16, 2 * f3 * nj});
+            cur->push_back({[=](cudaStream_t s) { return tc_gemm_f16_launch(ta, nj, s); }, C_UPD16, 2 * f3 * nj});
         }
+        }  // part
     }
+    // ---- assemble the schedule
+    if (!h->lookahead) {
+        for (int k = 0; k < nt; ++k)
+            for (auto* v : {&pan[k], &nxt[k], &rst[k]})
+                for (auto& o : *v) ops.push_back(std::move(o));
+        return MP_OK;
+    }
+    // events: 0 = start; 1 + 2k = panel k done; 2 + 2k = column k+1 updated
+    auto on = [&](std::vector<Op>& v, int stream) {
+        for (auto& o : v) {
+            o.stream = stream;
+            ops.push_back(std::move(o));
+        }
+    };
+    ops.push_back(op_record(0, 0));
+    ops.push_back(op_wait(1, 0));
+    on(pan[0], 1);
+    ops.push_back(op_record(1, 1));
+    for (int k = 0; k + 1 < nt; ++k) {
+        ops.push_back(op_wait(0, 1 + 2 * k));
+        on(nxt[k], 0);
+        ops.push_back(op_record(0, 2 + 2 * k));
+        ops.push_back(op_wait(1, 2 + 2 * k));
+        on(pan[k + 1], 1);
+        ops.push_back(op_record(1, 1 + 2 * (k + 1)));
+        on(rst[k], 0);
+    }
+    ops.push_back(op_wait(0, 1 + 2 * (nt - 1)));
     return MP_OK;
 }
 

@@ -1,9 +1,16 @@
-// K3 helpers — FP64 Cholesky and triangular inverse of one <=128 x 128 diagonal block in
-// shared memory.  The tile DPOTRF of Algorithm 1 ("D" = FP64 on diagonal tiles,
-// P:146) and the panel TRSM are blocked right-looking loops over 128-column
-// blocks whose bulk work is the DMMA GEMM (dgemm_dmma.cu); only these small sequential
-// pieces live here.  The inverse W = L_bb^{-1} turns each block's triangular solve into a
-// 128-wide GEMM (X_b = A_b W^T), the usual GPU treatment of small diagonal blocks.
+// K3 helpers — FP64 Cholesky and triangular inverse of one <= 128 x 128 diagonal block held in
+// shared memory.  The tile DPOTRF of Algorithm 1 ("D" = FP64 on diagonal tiles)
+// and the panel TRSM are blocked right-looking loops whose bulk work is the DMMA GEMM
+// (dgemm_dmma.cu); only these small sequential pieces live here.  The inverse W = L_bb^{-1} turns
+// each block's triangular solve into a 128-wide GEMM (X_b = A_b W^T).
+//
+// One 128 x 129 FP64 smem array holds the block: L in the lower triangle, W^T in the strictly
+// upper triangle, diag(W) in a side array, so L and W (264 KB together) fit in 132 KB.
+//   Cholesky: right-looking, ONE barrier per column — the update of step c uses the unscaled
+//     column c and 1/pivot; the column is scaled by 1/sqrt(pivot) during step c+1, when nobody
+//     reads it any more.
+//   Inverse:  Gauss-Jordan on [L | I]: for p, row p of W is final after dividing by L_pp and every
+//     row i > p subtracts L_ip times it (n^3/6 FMAs spread over all threads, 2 barriers per p).
 #include <math.h>
 
 #include "common.cuh"
@@ -11,90 +18,108 @@
 
 namespace mpgeo {
 
-constexpr int PB = POTRF_IB;     // 128
-constexpr int PLD = PB + 1;      // padded smem leading dimension
-constexpr int PT = 256;          // threads
-constexpr int P_SMEM = PB * PLD * 8;
+constexpr int PB = POTRF_IB;  // 128
+constexpr int PLD = PB + 1;   // padded smem leading dimension
+constexpr int PT = 256;       // threads
+constexpr int P_SMEM = PB * PLD * 8 + 3 * PB * 8;
 
-// In-place inverse of the jb x jb lower-triangular S (ld PLD) by columns, last to first:
-// L = [[l, 0], [x, L2]]  ->  L^{-1} = [[1/l, 0], [-(L2^{-1} x)/l, L2^{-1}]].
-__device__ void smem_trtri_lower(double* S, int jb, double* tmp) {
+// Cholesky of S[0:n, 0:n] (lower) in place; pivots checked against `info`.
+__device__ void smem_cholesky(double* S, double* piv, int n, int col0, int* info) {
     const int tid = threadIdx.x;
-    for (int j = jb - 1; j >= 0; --j) {
-        // tmp[i] = sum_{p=j+1..i} Winv[i][p] * x[p], x = S[j+1:, j] (old values)
-        for (int i = j + 1 + tid; i < jb; i += PT) {
-            double s = 0.0;
-            for (int p = j + 1; p <= i; ++p) s = fma(S[i * PLD + p], S[p * PLD + j], s);
-            tmp[i] = s;
+    const int tx = tid & 15, ty = tid >> 4;
+    for (int c = 0; c < n; ++c) {
+        const double d = S[c * PLD + c];
+        if (tid == 0) {
+            if (!(d > 0.0)) atomicMin(info, col0 + c + 1);
+            piv[c] = sqrt(d);
+        }
+        if (c > 0) {  // finalise column c-1 (no longer read by anyone)
+            const double inv = 1.0 / piv[c - 1];
+            for (int i = c + tid; i < n; i += PT) S[i * PLD + c - 1] *= inv;
+        }
+        const double ip = 1.0 / d;
+        for (int i = c + 1 + ty; i < n; i += 16) {
+            const double lic = S[i * PLD + c] * ip;
+            for (int j = c + 1 + tx; j <= i; j += 16) S[i * PLD + j] = fma(-lic, S[j * PLD + c], S[i * PLD + j]);
         }
         __syncthreads();
-        const double inv = 1.0 / S[j * PLD + j];
-        for (int i = j + 1 + tid; i < jb; i += PT) S[i * PLD + j] = -inv * tmp[i];
+    }
+    for (int c = tid; c < n; c += PT) S[c * PLD + c] = piv[c];
+    __syncthreads();
+}
+
+// W = L^{-1} by Gauss-Jordan; W[i][c] (c < i) stored at S[c][i], W[i][i] in wd[i].
+__device__ void smem_trtri_gj(double* S, double* wd, double* rowp, int n) {
+    const int tid = threadIdx.x;
+    for (int idx = tid; idx < n * n; idx += PT) {
+        const int r = idx / n, c = idx - r * n;
+        if (c > r) S[r * PLD + c] = 0.0;  // W starts as I (strict part)
+    }
+    for (int i = tid; i < n; i += PT) wd[i] = 1.0;
+    __syncthreads();
+    for (int p = 0; p < n; ++p) {
+        // row p of W: entries c < p at S[c][p], diagonal wd[p]; scale by 1/L_pp into rowp
+        const double ip = 1.0 / S[p * PLD + p];
+        for (int c = tid; c <= p; c += PT) rowp[c] = (c < p ? S[c * PLD + p] : wd[p]) * ip;
         __syncthreads();
-        if (tid == 0) S[j * PLD + j] = inv;
+        for (int c = tid; c <= p; c += PT) {
+            if (c < p) S[c * PLD + p] = rowp[c];
+            else wd[p] = rowp[p];
+        }
+        // rows i > p: W[i][c] -= L_ip * W[p][c], c <= p   (i fastest: conflict-free S[c][i])
+        const int rows = n - p - 1;
+        const int work = rows * (p + 1);
+        for (int w = tid; w < work; w += PT) {
+            const int c = w / rows, i = p + 1 + (w - c * rows);
+            const double l = S[i * PLD + p];
+            if (c < i) S[c * PLD + i] = fma(-l, rowp[c], S[c * PLD + i]);
+        }
         __syncthreads();
+    }
+}
+
+__device__ void write_block(const double* S, const double* wd, int n, double* A, int lda, double* W) {
+    const int tid = threadIdx.x;
+    for (int idx = tid; idx < n * n; idx += PT) {
+        const int r = idx / n, c = idx - r * n;
+        if (A) A[(size_t)r * lda + c] = (c <= r) ? S[r * PLD + c] : 0.0;
+        if (W) W[r * PB + c] = (c < r) ? S[c * PLD + r] : (c == r ? wd[r] : 0.0);
     }
 }
 
 __global__ void __launch_bounds__(PT, 1)
     potrf_diag_block_kernel(double* A, int lda, int jb, double* W, int col0, int* info) {
     extern __shared__ double S[];
-    double* tmp = S + PB * PLD;
+    double* piv = S + PB * PLD;
+    double* wd = piv + PB;
+    double* rowp = wd + PB;
     const int tid = threadIdx.x;
     for (int idx = tid; idx < jb * jb; idx += PT) {
         const int r = idx / jb, c = idx - r * jb;
-        S[r * PLD + c] = (c <= r) ? A[(size_t)r * lda + c] : 0.0;
+        if (c <= r) S[r * PLD + c] = A[(size_t)r * lda + c];
     }
     __syncthreads();
-    const int tx = tid & 15, ty = tid >> 4;
-    for (int c = 0; c < jb; ++c) {
-        if (tid == 0) {
-            const double d = S[c * PLD + c];
-            if (!(d > 0.0)) atomicMin(info, col0 + c + 1);
-            S[c * PLD + c] = sqrt(d);
-        }
-        __syncthreads();
-        const double inv = 1.0 / S[c * PLD + c];
-        for (int i = c + 1 + tid; i < jb; i += PT) S[i * PLD + c] *= inv;
-        __syncthreads();
-        for (int i = c + 1 + ty; i < jb; i += 16) {
-            const double lic = S[i * PLD + c];
-            for (int j = c + 1 + tx; j <= i; j += 16) S[i * PLD + j] = fma(-lic, S[j * PLD + c], S[i * PLD + j]);
-        }
-        __syncthreads();
-    }
-    // L back to the tile (upper part of the block zeroed)
-    for (int idx = tid; idx < jb * jb; idx += PT) {
-        const int r = idx / jb, c = idx - r * jb;
-        A[(size_t)r * lda + c] = (c <= r) ? S[r * PLD + c] : 0.0;
-    }
-    __syncthreads();
-    smem_trtri_lower(S, jb, tmp);
-    for (int idx = tid; idx < jb * jb; idx += PT) {
-        const int r = idx / jb, c = idx - r * jb;
-        W[r * PB + c] = (c <= r) ? S[r * PLD + c] : 0.0;
-    }
+    smem_cholesky(S, piv, jb, col0, info);
+    smem_trtri_gj(S, wd, rowp, jb);
+    write_block(S, wd, jb, A, lda, W);
 }
 
 __global__ void __launch_bounds__(PT, 1) trtri_blocks_kernel(const double* L, int nb, double* W) {
     extern __shared__ double S[];
-    double* tmp = S + PB * PLD;
+    double* wd = S + PB * PLD + PB;
+    double* rowp = wd + PB;
     const int b = blockIdx.x;
     const int j0 = b * PB;
     const int jb = min(PB, nb - j0);
     const double* Lb = L + (size_t)j0 * nb + j0;
-    double* Wb = W + (size_t)b * PB * PB;
     const int tid = threadIdx.x;
     for (int idx = tid; idx < jb * jb; idx += PT) {
         const int r = idx / jb, c = idx - r * jb;
-        S[r * PLD + c] = (c <= r) ? Lb[(size_t)r * nb + c] : 0.0;
+        if (c <= r) S[r * PLD + c] = Lb[(size_t)r * nb + c];
     }
     __syncthreads();
-    smem_trtri_lower(S, jb, tmp);
-    for (int idx = tid; idx < jb * jb; idx += PT) {
-        const int r = idx / jb, c = idx - r * jb;
-        Wb[r * PB + c] = (c <= r) ? S[r * PLD + c] : 0.0;
-    }
+    smem_trtri_gj(S, wd, rowp, jb);
+    write_block(S, wd, jb, nullptr, 0, W + (size_t)b * PB * PB);
 }
 
 static cudaError_t set_smem(const void* f, int bytes) {
@@ -104,25 +129,23 @@ static cudaError_t set_smem(const void* f, int bytes) {
 cudaError_t potrf_diag_block_launch(double* A, int lda, int jb, double* W, int col0, int* info,
                                     cudaStream_t s) {
     static bool init = false;
-    const int smem = P_SMEM + PB * 8;
     if (!init) {
-        cudaError_t e = set_smem((const void*)potrf_diag_block_kernel, smem);
+        cudaError_t e = set_smem((const void*)potrf_diag_block_kernel, P_SMEM);
         if (e != cudaSuccess) return e;
         init = true;
     }
-    potrf_diag_block_kernel<<<1, PT, smem, s>>>(A, lda, jb, W, col0, info);
+    potrf_diag_block_kernel<<<1, PT, P_SMEM, s>>>(A, lda, jb, W, col0, info);
     return cudaGetLastError();
 }
 
 cudaError_t trtri_blocks_launch(const double* L, int nb, double* W, cudaStream_t s) {
     static bool init = false;
-    const int smem = P_SMEM + PB * 8;
     if (!init) {
-        cudaError_t e = set_smem((const void*)trtri_blocks_kernel, smem);
+        cudaError_t e = set_smem((const void*)trtri_blocks_kernel, P_SMEM);
         if (e != cudaSuccess) return e;
         init = true;
     }
-    trtri_blocks_kernel<<<(nb + PB - 1) / PB, PT, smem, s>>>(L, nb, W);
+    trtri_blocks_kernel<<<(nb + PB - 1) / PB, PT, P_SMEM, s>>>(L, nb, W);
     return cudaGetLastError();
 }
 
