@@ -55,7 +55,7 @@ typedef enum {
     MP_ERR_ARG = 1,          /* invalid argument: sizes, theta <= 0, nu outside (0, 20], bad map */
     MP_ERR_NOT_SPD = 2,      /* POTRF met a non-positive pivot; see `info` of mp_tile_potrf */
     MP_ERR_CUDA = 3,         /* a CUDA call failed; the handle is unusable afterwards */
-    MP_ERR_NCCL = 4,         /* an NCCL call failed; the handle is unusable afterwards */
+    MP_ERR_COMM = 4,         /* peer exchange not connected / IPC mapping failed */
     MP_ERR_NOMEM = 5,        /* workspace too small for the requested layout */
     MP_ERR_UNSUPPORTED = 6,  /* configuration this build does not implement */
     MP_ERR_STATE = 7         /* call order violated (e.g. potrf before generation) */
@@ -98,13 +98,11 @@ typedef struct {
 
 /* ---------------------------------------------------------------- lifecycle */
 
-/* NCCL unique id for multi-GPU handles (rank 0 calls it and broadcasts the 128
- * bytes, e.g. with torch.distributed).  Unused when nranks == 1. */
-mp_status mp_get_unique_id(uint8_t id[128]);
-
 /* Create a handle on CUDA `device` for `rank` of `nranks` (P * Q == nranks,
- * P <= Q).  `id` may be NULL when nranks == 1.  `cuda_stream` is a cudaStream_t
- * (NULL = a stream created and owned by the handle).  *h receives the handle. */
+ * P <= Q, nranks <= 8).  `id` is reserved (pass NULL).  `cuda_stream` is a
+ * cudaStream_t (NULL = a stream created and owned by the handle).  *h receives
+ * the handle.  Multi-rank matrices exchange panel tiles through peer memory: see
+ * mp_matrix_comm_export / mp_matrix_comm_connect. */
 mp_status mp_init(int device, int rank, int nranks, int P, int Q, const uint8_t* id,
                   void* cuda_stream, mp_handle** h);
 mp_status mp_finalize(mp_handle* h);
@@ -126,6 +124,34 @@ mp_status mp_matrix_bytes(const mp_matrix* A, const uint8_t* storage_prec, size_
  * storage map (NULL = all FP64).  May be called again with a new map on the
  * same workspace (each MLE evaluation has its own map); contents are lost. */
 mp_status mp_matrix_bind(mp_matrix* A, const uint8_t* storage_prec, void* d_workspace, size_t bytes);
+
+/* Multi-rank only (nranks > 1), once per matrix, before its first use:
+ * mp_matrix_comm_export allocates this rank's exchange area (send slots in
+ * communication precision, stamps, solve vectors; library-owned device memory)
+ * and writes its 64-byte CUDA IPC handle to handle_out.  The caller all-gathers
+ * the handles (e.g. torch.distributed.all_gather_object) in rank order and
+ * passes the nranks * 64 bytes to mp_matrix_comm_connect, which maps every
+ * peer's area.  Consumers then read panel tiles directly from the producer's
+ * memory (NVLink peer loads across GPUs; same-device IPC between processes). */
+mp_status mp_matrix_comm_export(mp_matrix* A, void* handle_out);
+mp_status mp_matrix_comm_connect(mp_matrix* A, const void* all_handles);
+
+/* One transfer of the multi-rank panel exchange (host description). */
+typedef struct {
+    int32_t k;     /* panel */
+    int32_t m;     /* tile row: m == k is L~_kk (POTRF output), m > k is L_mk (TRSM output) */
+    int32_t peer;  /* producer rank for a pull, -1 for a publish */
+    int32_t prec;  /* communication precision (mp_prec) the tile travels in */
+    int32_t dir;   /* 0 = publish (this rank produces it for others), 1 = pull */
+} mp_xfer;
+
+/* Pure host: the exchange `rank` performs in an nt x nt factorisation on a P x Q grid
+ * (POTRF(k,k) -> TRSMs of column k; TRSM(m,k) -> GEMMs of row m and column m and
+ * SYRK(m,k)), given the NT*NT comm map.  Writes up to `cap` records (out may be NULL to count)
+ * and the total to *count; MP_ERR_NOMEM if cap was too small.  mp_tile_potrf executes
+ * exactly these records. */
+mp_status mp_exchange_plan(int nt, int P, int Q, int rank, const uint8_t* comm_prec, mp_xfer* out,
+                           int64_t cap, int64_t* count);
 
 /* ---------------------------------------------------------------- the path */
 

@@ -19,7 +19,7 @@ from ._lib import (EvalReport, MpError, Profile, PROF_CLASSES, lib, MP_OK, MP_ER
                    MP_COMM_TTC, MP_COMM_AUTO, MP_MAP_ADAPTIVE, MP_MAP_FP64, MP_MAP_BAND, MP_MAP_EXTREME,
                    MP_MAP_USER)
 
-__all__ = ["Handle", "Matrix", "Evaluator", "precision_map", "exact_sum", "MpError", "EvalReport"]
+__all__ = ["Handle", "Matrix", "Evaluator", "precision_map", "exchange_plan", "exact_sum", "MpError", "EvalReport"]
 
 _u8p = C.POINTER(C.c_uint8)
 _dp = C.POINTER(C.c_double)
@@ -65,6 +65,7 @@ class Handle:
             raise MpError(st, "mp_init failed")
         self.h = h
         self.device = device
+        self.rank, self.nranks, self.P, self.Q = rank, nranks, P, Q
 
     def check(self, st: int):
         if st != MP_OK:
@@ -97,7 +98,7 @@ class Handle:
 class Matrix:
     """mp_matrix_*: geometry + a caller-owned (torch) workspace."""
 
-    def __init__(self, handle: Handle, n: int, nb: int, storage_prec: np.ndarray | None = None):
+    def __init__(self, handle: Handle, n: int, nb: int, storage_prec: np.ndarray | None = None, group=None):
         import torch
 
         self.handle = handle
@@ -106,11 +107,27 @@ class Matrix:
         self.A = A
         self.n, self.nb = n, nb
         self.nt = lib.mp_matrix_nt(A)
+        if handle.nranks > 1:
+            self._connect(group)
         nbytes = C.c_size_t()
         handle.check(lib.mp_matrix_bytes(A, _u8(storage_prec), C.byref(nbytes)))
         self.nbytes = nbytes.value
         self.ws = torch.empty(self.nbytes, dtype=torch.uint8, device=f"cuda:{handle.device}")
         self.bind(storage_prec)
+
+    def _connect(self, group):
+        """Exchange the CUDA IPC handles of every rank's exchange area (torch.distributed all-gather)."""
+        import torch.distributed as dist
+
+        buf = (C.c_uint8 * 64)()
+        self.handle.check(lib.mp_matrix_comm_export(self.A, buf))
+        allh = [None] * self.handle.nranks
+        dist.all_gather_object(allh, bytes(buf), group=group)
+        joined = b"".join(allh)
+        self.handle.check(lib.mp_matrix_comm_connect(self.A, joined))
+
+    def owner(self, m: int, k: int) -> int:
+        return int(lib.mp_matrix_owner(self.A, m, k))
 
     def bind(self, storage_prec: np.ndarray | None):
         self.handle.check(lib.mp_matrix_bind(self.A, _u8(storage_prec), C.c_void_p(self.ws.data_ptr()), self.nbytes))
@@ -191,6 +208,22 @@ def precision_map(tile_sqnorm: np.ndarray | None, u_req: float = 1e-9, eps=None,
     return km, sm, cm
 
 
+def exchange_plan(nt: int, P: int, Q: int, rank: int, comm_prec: np.ndarray) -> list[tuple]:
+    """mp_exchange_plan: [(k, m, peer, prec, dir)] for `rank` (dir 0 = publish, 1 = pull)."""
+    from ._lib import Xfer
+
+    cm = np.ascontiguousarray(comm_prec, dtype=np.uint8)
+    cnt = C.c_int64(0)
+    st = lib.mp_exchange_plan(nt, P, Q, rank, _u8(cm), None, 0, C.byref(cnt))
+    if st != MP_OK:
+        raise MpError(st, "mp_exchange_plan failed")
+    arr = (Xfer * max(1, cnt.value))()
+    st = lib.mp_exchange_plan(nt, P, Q, rank, _u8(cm), arr, cnt.value, C.byref(cnt))
+    if st != MP_OK:
+        raise MpError(st, "mp_exchange_plan failed")
+    return [(x.k, x.m, x.peer, x.prec, x.dir) for x in arr[: cnt.value]]
+
+
 def exact_sum(v: np.ndarray) -> float:
     v = np.ascontiguousarray(v, dtype=np.float64)
     return float(lib.mpgeo_exact_sum(_d(v), v.size))
@@ -199,9 +232,9 @@ def exact_sum(v: np.ndarray) -> float:
 class Evaluator:
     """One log-likelihood evaluation per call (mp_eval) on a worst-case (all-FP64) workspace."""
 
-    def __init__(self, n: int, nb: int, device: int = 0, handle: Handle | None = None):
+    def __init__(self, n: int, nb: int, device: int = 0, handle: Handle | None = None, group=None):
         self.handle = handle or Handle(device)
-        self.M = Matrix(self.handle, n, nb, None)
+        self.M = Matrix(self.handle, n, nb, None, group=group)
         self.n, self.nb, self.nt = n, nb, self.M.nt
 
     def eval(self, x, y, z, theta, u_req: float = 1e-9, mode: int = MP_MAP_ADAPTIVE, policy: int = MP_COMM_AUTO,

@@ -12,8 +12,8 @@ import os
 _HERE = os.path.dirname(os.path.abspath(__file__))
 LIB_PATH = os.path.join(_HERE, "libmpgeo.so")
 
-MP_OK, MP_ERR_ARG, MP_ERR_NOT_SPD, MP_ERR_CUDA, MP_ERR_NCCL, MP_ERR_NOMEM, MP_ERR_UNSUPPORTED, MP_ERR_STATE = range(8)
-STATUS_NAMES = ["MP_OK", "MP_ERR_ARG", "MP_ERR_NOT_SPD", "MP_ERR_CUDA", "MP_ERR_NCCL", "MP_ERR_NOMEM",
+MP_OK, MP_ERR_ARG, MP_ERR_NOT_SPD, MP_ERR_CUDA, MP_ERR_COMM, MP_ERR_NOMEM, MP_ERR_UNSUPPORTED, MP_ERR_STATE = range(8)
+STATUS_NAMES = ["MP_OK", "MP_ERR_ARG", "MP_ERR_NOT_SPD", "MP_ERR_CUDA", "MP_ERR_COMM", "MP_ERR_NOMEM",
                 "MP_ERR_UNSUPPORTED", "MP_ERR_STATE"]
 MP_FP64, MP_FP32, MP_FP16 = 0, 1, 2
 MP_COMM_TTC, MP_COMM_AUTO = 0, 1
@@ -42,6 +42,10 @@ class Profile(C.Structure):
                 for i, name in enumerate(PROF_CLASSES)}
 
 
+class Xfer(C.Structure):
+    _fields_ = [("k", C.c_int32), ("m", C.c_int32), ("peer", C.c_int32), ("prec", C.c_int32), ("dir", C.c_int32)]
+
+
 class MpError(RuntimeError):
     def __init__(self, status: int, msg: str):
         super().__init__(f"{STATUS_NAMES[status] if 0 <= status < len(STATUS_NAMES) else status}: {msg}")
@@ -55,7 +59,6 @@ def _load() -> C.CDLL:
     lib = C.CDLL(LIB_PATH, mode=C.RTLD_GLOBAL)
     vp, i32, i64, dbl, u8p, dp = C.c_void_p, C.c_int, C.c_int64, C.c_double, C.POINTER(C.c_uint8), C.POINTER(C.c_double)
     sig = {
-        "mp_get_unique_id": (i32, [u8p]),
         "mp_init": (i32, [i32, i32, i32, i32, i32, u8p, vp, C.POINTER(vp)]),
         "mp_finalize": (i32, [vp]),
         "mp_last_error": (C.c_char_p, [vp]),
@@ -71,6 +74,9 @@ def _load() -> C.CDLL:
         "mp_matrix_maps": (i32, [vp, u8p, u8p, u8p]),
         "mp_matrix_get_tile": (i32, [vp, vp, i32, i32, dp]),
         "mp_matrix_set_tile": (i32, [vp, vp, i32, i32, dp]),
+        "mp_matrix_comm_export": (i32, [vp, vp]),
+        "mp_matrix_comm_connect": (i32, [vp, vp]),
+        "mp_exchange_plan": (i32, [i32, i32, i32, i32, u8p, C.POINTER(Xfer), i64, C.POINTER(i64)]),
         "mp_matrix_nt": (i32, [vp]),
         "mp_matrix_owner": (i32, [vp, i32, i32]),
         "mp_launch_count": (i64, [vp]),

@@ -13,7 +13,7 @@
 //      output tile: FP64 (DMMA), FP32 class and FP16 class.
 // Everything for one call is planned on the host first (job arrays for the batched kernels),
 // uploaded once into the control arena of the workspace, then enqueued.
-#include <dlfcn.h>
+#include <unistd.h>
 
 #include <algorithm>
 #include <climits>
@@ -27,28 +27,9 @@
 #include "../../include/mpgeo.h"
 #include "kernels.h"
 #include "tc_gemm.h"
+#include "dist.h"
 
 using namespace mpgeo;
-
-// ------------------------------------------------------------------ NCCL (loaded lazily)
-typedef struct { char internal[128]; } nccl_uid_t;
-typedef void* nccl_comm_t;
-struct NcclApi {
-    void* lib = nullptr;
-    int (*GetUniqueId)(nccl_uid_t*) = nullptr;
-    int (*CommInitRank)(nccl_comm_t*, int, nccl_uid_t, int) = nullptr;
-    int (*CommDestroy)(nccl_comm_t) = nullptr;
-    bool load() {
-        if (lib) return true;
-        lib = dlopen("libnccl.so.2", RTLD_NOW | RTLD_GLOBAL);
-        if (!lib) return false;
-        GetUniqueId = (int (*)(nccl_uid_t*))dlsym(lib, "ncclGetUniqueId");
-        CommInitRank = (int (*)(nccl_comm_t*, int, nccl_uid_t, int))dlsym(lib, "ncclCommInitRank");
-        CommDestroy = (int (*)(nccl_comm_t))dlsym(lib, "ncclCommDestroy");
-        return GetUniqueId && CommInitRank && CommDestroy;
-    }
-};
-static NcclApi g_nccl;
 
 // ------------------------------------------------------------------ objects
 struct ProfRec {
@@ -60,7 +41,6 @@ struct mp_handle {
     int device = 0, rank = 0, nranks = 1, P = 1, Q = 1;
     cudaStream_t stream = nullptr;
     bool own_stream = false;
-    nccl_comm_t nccl = nullptr;
     std::string err;
     int64_t launches = 0;
     int* d_info = nullptr;
@@ -85,8 +65,21 @@ struct Regions {
     std::vector<size_t> tile_off;  // per (m*nt+k), SIZE_MAX if not stored here
 };
 
+// Peer-memory exchange area of one matrix (multi-GPU only; cudaMalloc'ed by the library so it
+// can be exported with cudaIpcGetMemHandle).  Offsets are identical on every rank.
+struct Comm {
+    char* base = nullptr;
+    size_t bytes = 0;
+    std::vector<char*> peer;  // base of every rank's area (own = base)
+    bool connected = false;
+    uint64_t epoch = 0;       // incremented per collective call; stamps = epoch << 24 | step
+    size_t send = 0, pub = 0, done = 0, bar = 0, part = 0, yv = 0, pflag = 0, yflag = 0, norms = 0, nflag = 0,
+           scal = 0, sflag = 0, tmp = 0;
+};
+
 struct mp_matrix {
     mp_handle* h = nullptr;
+    Comm comm;
     int64_t n = 0;
     int nb = 0, nt = 0;
     char* ws = nullptr;
@@ -132,6 +125,7 @@ static size_t ctrl_bytes_for(int nt, int nb) {
     bytes += T * (T + 1) / 2 * sizeof(GenTile);
     bytes += T * T * sizeof(GemvTile);
     bytes += T * (sizeof(double*) + sizeof(int));
+    bytes += T * T * (sizeof(PackItem) + sizeof(PullItem) + 2 * sizeof(WaitItem)) + T * 8 * sizeof(WaitItem);
     bytes += 64 * 1024 + 32 * 256;  // alignment slack
     return bytes;
 }
@@ -256,15 +250,6 @@ extern "C" {
 
 const char* mp_version(void) { return "mpgeo 0.1 sm_100a (DMMA FP64, tcgen05 TF32x3/FP16)"; }
 
-mp_status mp_get_unique_id(uint8_t id[128]) {
-    if (!id) return MP_ERR_ARG;
-    if (!g_nccl.load()) return MP_ERR_NCCL;
-    nccl_uid_t u;
-    if (g_nccl.GetUniqueId(&u) != 0) return MP_ERR_NCCL;
-    memcpy(id, u.internal, 128);
-    return MP_OK;
-}
-
 mp_status mp_init(int device, int rank, int nranks, int P, int Q, const uint8_t* id, void* cuda_stream,
                   mp_handle** out) {
     if (!out || nranks < 1 || rank < 0 || rank >= nranks || P < 1 || Q < 1 || P * Q != nranks || P > Q)
@@ -298,12 +283,8 @@ mp_status mp_init(int device, int rank, int nranks, int P, int Q, const uint8_t*
     if (cudaMalloc(&h->d_info, sizeof(int)) != cudaSuccess) return fail(MP_ERR_CUDA);
     for (auto& e : h->ev)
         if (cudaEventCreate(&e) != cudaSuccess) return fail(MP_ERR_CUDA);
-    if (nranks > 1) {
-        if (!id || !g_nccl.load()) return fail(MP_ERR_NCCL);
-        nccl_uid_t u;
-        memcpy(u.internal, id, 128);
-        if (g_nccl.CommInitRank(&h->nccl, nranks, u, rank) != 0) return fail(MP_ERR_NCCL);
-    }
+    (void)id;  // reserved: the panel exchange is peer memory (mp_matrix_comm_export/connect)
+    if (nranks > MAX_PEERS) return fail(MP_ERR_UNSUPPORTED);
     *out = h;
     return MP_OK;
 }
@@ -312,7 +293,6 @@ mp_status mp_finalize(mp_handle* h) {
     if (!h) return MP_ERR_ARG;
     cudaSetDevice(h->device);
     if (h->stream) cudaStreamSynchronize(h->stream);
-    if (h->nccl) g_nccl.CommDestroy(h->nccl);
     for (auto& e : h->ev)
         if (e) cudaEventDestroy(e);
     for (auto& e : h->prof_pool)
@@ -371,7 +351,75 @@ mp_status mp_matrix_create(mp_handle* h, int64_t n, int nb, mp_matrix** A) {
 }
 
 mp_status mp_matrix_destroy(mp_matrix* A) {
+    if (!A) return MP_ERR_ARG;
+    for (size_t r = 0; r < A->comm.peer.size(); ++r)
+        if (A->comm.peer[r] && A->comm.peer[r] != A->comm.base) cudaIpcCloseMemHandle(A->comm.peer[r]);
+    if (A->comm.base) cudaFree(A->comm.base);
     delete A;
+    return MP_OK;
+}
+
+static size_t comm_layout(mp_matrix* A) {
+    Comm& c = A->comm;
+    const size_t nt = A->nt, nb = A->nb, nb2 = A->nb2();
+    size_t off = 0;
+    auto take = [&](size_t bytes) {
+        off = align_up(off, 256);
+        const size_t o = off;
+        off += bytes;
+        return o;
+    };
+    c.send = take(2 * nt * nb2 * 8);
+    c.pub = take(2 * nt * 8);
+    c.done = take(2 * 8);
+    c.bar = take(8);
+    c.part = take(nt * nb * 8);
+    c.yv = take(nt * nb * 8);
+    c.pflag = take(nt * 8);
+    c.yflag = take(nt * 8);
+    c.norms = take(nt * nt * 8);
+    c.nflag = take(8);
+    c.scal = take(4 * 8);
+    c.sflag = take(8);
+    c.tmp = take(nb * 8);
+    return align_up(off, 256);
+}
+
+mp_status mp_matrix_comm_export(mp_matrix* A, void* handle_out) {
+    if (!A || !handle_out) return MP_ERR_ARG;
+    mp_handle* h = A->h;
+    if (h->nranks < 2) FAIL(h, MP_ERR_STATE, "single-rank handle has no exchange area");
+    Comm& c = A->comm;
+    if (!c.base) {
+        c.bytes = comm_layout(A);
+        CK(h, cudaMalloc(&c.base, c.bytes));
+        CK(h, cudaMemset(c.base, 0, c.bytes));
+        CK(h, cudaDeviceSynchronize());
+    }
+    cudaIpcMemHandle_t ih;
+    CK(h, cudaIpcGetMemHandle(&ih, c.base));
+    memcpy(handle_out, &ih, sizeof ih);
+    return MP_OK;
+}
+
+mp_status mp_matrix_comm_connect(mp_matrix* A, const void* all_handles) {
+    if (!A || !all_handles) return MP_ERR_ARG;
+    mp_handle* h = A->h;
+    Comm& c = A->comm;
+    if (!c.base) FAIL(h, MP_ERR_STATE, "call mp_matrix_comm_export first");
+    c.peer.assign(h->nranks, nullptr);
+    for (int r = 0; r < h->nranks; ++r) {
+        if (r == h->rank) {
+            c.peer[r] = c.base;
+            continue;
+        }
+        cudaIpcMemHandle_t ih;
+        memcpy(&ih, (const char*)all_handles + (size_t)r * sizeof ih, sizeof ih);
+        void* p = nullptr;
+        CK(h, cudaIpcOpenMemHandle(&p, ih, cudaIpcMemLazyEnablePeerAccess));
+        c.peer[r] = (char*)p;
+    }
+    c.connected = true;
     return MP_OK;
 }
 
@@ -453,6 +501,29 @@ mp_status mp_matrix_set_tile(mp_handle* h, mp_matrix* A, int m, int k, const dou
     return MP_OK;
 }
 
+// ------------------------------------------------------------------ multi-rank host helpers
+// Host wait for a peer stamp (used by the host-synchronous collectives: norm gather, scalars).
+static mp_status host_wait_stamp(mp_handle* h, const uint64_t* dflag, uint64_t target) {
+    for (long it = 0;; ++it) {
+        uint64_t v = 0;
+        CK(h, cudaMemcpy(&v, dflag, 8, cudaMemcpyDeviceToHost));
+        if (v >= target) return MP_OK;
+        if (it > 20000000) FAIL(h, MP_ERR_COMM, "timeout waiting for a peer stamp");
+        if (it > 100) usleep(50);
+    }
+}
+
+// Barrier among all ranks through device flags (host-synchronous).
+static mp_status dist_barrier(mp_handle* h, mp_matrix* A, uint64_t stamp) {
+    Comm& X = A->comm;
+    CK(h, set_flag_launch((uint64_t*)(X.base + X.bar), stamp, h->stream));
+    CK(h, cudaStreamSynchronize(h->stream));
+    for (int r = 0; r < h->nranks; ++r)
+        if (r != h->rank)
+            if (mp_status st = host_wait_stamp(h, (const uint64_t*)(X.peer[r] + X.bar), stamp)) return st;
+    return MP_OK;
+}
+
 // ------------------------------------------------------------------ (1) generation
 static mp_status check_theta(mp_handle* h, const double* th) {
     if (!th || !(th[0] > 0) || !(th[1] > 0) || !(th[2] > 0) || !(th[2] <= 20.0) || !std::isfinite(th[0]) ||
@@ -480,7 +551,7 @@ mp_status mp_matern_gen(mp_handle* h, mp_matrix* A, const double* d_x, const dou
     if (!h || !A || !d_x || !d_y) return MP_ERR_ARG;
     if (h->broken) FAIL(h, MP_ERR_STATE, "handle unusable after an earlier CUDA failure");
     if (mp_status s = check_theta(h, theta)) return s;
-    if (h->nranks > 1) FAIL(h, MP_ERR_UNSUPPORTED, "multi-rank generation not in this build");
+    if (h->nranks > 1 && !A->comm.connected) FAIL(h, MP_ERR_COMM, "multi-rank matrix not connected");
     const int nt = A->nt;
     const MaternArgs a = matern_args(A, d_x, d_y, theta);
     if (!storage_prec) {
@@ -490,7 +561,8 @@ mp_status mp_matern_gen(mp_handle* h, mp_matrix* A, const double* d_x, const dou
         if (!tile_sqnorm) return MP_ERR_ARG;
         std::vector<GenTile> tl;
         for (int k = 0; k < nt; ++k)
-            for (int m = k; m < nt; ++m) tl.push_back(GenTile{m, k, 0, 0, nullptr});
+            for (int m = k; m < nt; ++m)
+                if (A->mine(m, k)) tl.push_back(GenTile{m, k, 0, 0, nullptr});
         Arena ar;
         ar.dev_base = A->ws + A->R.ctrl;
         GenTile* d_tl = ar.push(tl);
@@ -507,6 +579,23 @@ mp_status mp_matern_gen(mp_handle* h, mp_matrix* A, const double* d_x, const dou
         CK(h, cudaStreamSynchronize(h->stream));
         for (size_t i = 0; i < (size_t)nt * nt; ++i) tile_sqnorm[i] = 0.0;
         for (int i = 0; i < ntl; ++i) tile_sqnorm[(size_t)tl[i].m * nt + tl[i].k] = v[i];
+        if (h->nranks > 1) {
+            // all-gather over peer memory: every tile has exactly one owner, so the merge is exact
+            Comm& X = A->comm;
+            const uint64_t stamp = (++X.epoch << 24) + 1;
+            if (mp_status st = dist_barrier(h, A, stamp)) return st;
+            CK(h, cudaMemcpy(X.base + X.norms, tile_sqnorm, (size_t)nt * nt * 8, cudaMemcpyHostToDevice));
+            CK(h, set_flag_launch((uint64_t*)(X.base + X.nflag), stamp, h->stream));
+            CK(h, cudaStreamSynchronize(h->stream));
+            std::vector<double> tmp((size_t)nt * nt);
+            for (int r = 0; r < h->nranks; ++r) {
+                if (r == h->rank) continue;
+                if (mp_status st = host_wait_stamp(h, (const uint64_t*)(X.peer[r] + X.nflag), stamp)) return st;
+                CK(h, cudaMemcpy(tmp.data(), X.peer[r] + X.norms, tmp.size() * 8, cudaMemcpyDeviceToHost));
+                for (size_t i = 0; i < tmp.size(); ++i) tile_sqnorm[i] += tmp[i];
+            }
+            if (mp_status st = dist_barrier(h, A, stamp + 1)) return st;
+        }
         return MP_OK;
     }
     if (!A->bound) FAIL(h, MP_ERR_STATE, "matrix not bound");
@@ -536,7 +625,7 @@ struct FlopCount {
 };
 
 static mp_status plan_potrf(mp_handle* h, mp_matrix* A, const uint8_t* km, const uint8_t* cm, Arena& ar,
-                            std::vector<Op>& ops, FlopCount& fc) {
+                            std::vector<Op>& ops, FlopCount& fc, uint64_t epoch) {
     const int nt = A->nt, nb = A->nb, IB = POTRF_IB, OB = 4 * POTRF_IB;
     const size_t nb2 = A->nb2();
     double* const p64b = A->at<double>(A->R.p64);
@@ -551,11 +640,43 @@ static mp_status plan_potrf(mp_handle* h, mp_matrix* A, const uint8_t* km, const
     auto K = [&](int m, int k) { return km[(size_t)m * nt + k]; };
     auto C = [&](int m, int k) { return cm[(size_t)m * nt + k]; };
     const double fnb = (double)nb;
+    std::vector<Op>* cur = nullptr;
+    auto cur_push = [&](Op o) { cur->push_back(std::move(o)); };
+    // ---- multi-rank exchange helpers; unused on one rank
+    const bool dist = h->nranks > 1;
+    const bool la = h->lookahead && !dist;
+    const int R = h->nranks, me = h->rank;
+    Comm& X = A->comm;
+    auto ST = [&](int step) -> uint64_t { return (epoch << 24) + (uint64_t)(step + 2); };
+    auto sendslot = [&](int r, int s, int m) { return X.peer[r] + X.send + ((size_t)s * nt + m) * nb2 * 8; };
+    auto pubflag = [&](int r, int s, int m) { return (uint64_t*)(X.peer[r] + X.pub) + (size_t)s * nt + m; };
+    auto doneflag = [&](int r, int s) { return (uint64_t*)(X.peer[r] + X.done) + s; };
+    // the exchange records this rank executes (exchange.cpp, also checked by the CPU tests)
+    std::vector<std::vector<mp_xfer>> xpub(nt), xpull(nt);
+    if (dist) {
+        int64_t cnt = 0;
+        mp_exchange_plan(nt, h->P, h->Q, me, cm, nullptr, 0, &cnt);
+        std::vector<mp_xfer> xs((size_t)cnt);
+        if (mp_exchange_plan(nt, h->P, h->Q, me, cm, xs.data(), cnt, &cnt)) FAIL(h, MP_ERR_ARG, "exchange plan failed");
+        for (auto& x : xs) (x.dir == 0 ? xpub : xpull)[x.k].push_back(x);
+    }
+    auto local_formats = [&](int k, int m, bool& n16, bool& n32) {  // operand formats of MY successors of L_mk
+        n16 = n32 = false;
+        for (int n = k + 1; n < m; ++n)
+            if (A->mine(m, n)) n16 |= K(m, n) == MP_FP16, n32 |= K(m, n) == MP_FP32;
+        for (int n = m + 1; n < nt; ++n)
+            if (A->mine(n, m)) n16 |= K(n, m) == MP_FP16, n32 |= K(n, m) == MP_FP32;
+    };
+    auto push_wait = [&](std::vector<WaitItem>& w) {
+        if (w.empty()) return;
+        WaitItem* dw = ar.push(w);
+        const int n = (int)w.size();
+        cur_push(Op{[=](cudaStream_t s) { return wait_flags_launch(dw, n, s); }, C_CONV, 0});
+    };
 
     // per step: panel(k) = POTRF + TRSM + conversion; next(k) = the update of column k+1 (what
     // panel k+1 waits for); rest(k) = the rest of the trailing update
     std::vector<std::vector<Op>> pan(nt), nxt(nt), rst(nt);
-    std::vector<Op>* cur = nullptr;
     auto gemm = [&](std::vector<GemmJob>& jobs, int M, int N, int Kd, int lda, int ldb, int ldc, int lower,
                     double alpha, double beta, int round, bool cf32, int cls, double flops_per_job) {
         if (jobs.empty()) return;
@@ -576,7 +697,17 @@ static mp_status plan_potrf(mp_handle* h, mp_matrix* A, const uint8_t* km, const
     };
 
     for (int k = 0; k < nt; ++k) {
-        const size_t set = h->lookahead ? (size_t)(k & 1) : 0;
+        const size_t set = la ? (size_t)(k & 1) : 0;
+        const int sp = k & 1;  // send-slot parity (multi-rank)
+        bool send_free_waited = false;
+        auto wait_send_free = [&]() {  // every peer has pulled panel k-2 from slot set sp
+            if (send_free_waited || k < 2) return;
+            std::vector<WaitItem> w;
+            for (int r = 0; r < R; ++r)
+                if (r != me) w.push_back(WaitItem{doneflag(r, sp), ST(k - 2)});
+            push_wait(w);
+            send_free_waited = true;
+        };
         double* p64 = p64b + set * nt * nb2;
         __half* p16 = p16b + set * nt * nb2;
         float* phi = phib + set * nt * nb2;
@@ -585,6 +716,15 @@ static mp_status plan_potrf(mp_handle* h, mp_matrix* A, const uint8_t* km, const
         // ---- 1. DPOTRF(k,k), FP64: two-level blocking — 128-column blocks
         //      (diagonal block Cholesky + inverse, block column as GEMM with the inverse, update
         //      inside the 512-column outer block), then one K = 512 SYRK per outer block.
+        if (dist && k == 0) {  // device-side barrier: every rank finished the previous collective
+            uint64_t* bar = (uint64_t*)(X.base + X.bar);
+            const uint64_t bv = ST(-1);
+            cur_push(Op{[=](cudaStream_t s) { return set_flag_launch(bar, bv, s); }, C_CONV, 0});
+            std::vector<WaitItem> w;
+            for (int r = 0; r < R; ++r)
+                if (r != me) w.push_back(WaitItem{(uint64_t*)(X.peer[r] + X.bar), bv});
+            push_wait(w);
+        }
         if (A->mine(k, k)) {
             double* Akk = (double*)A->tile(k, k);
             for (int J0 = 0; J0 < nb; J0 += OB) {
@@ -617,12 +757,40 @@ static mp_status plan_potrf(mp_handle* h, mp_matrix* A, const uint8_t* km, const
             fc.potrf += fnb * fnb * fnb / 3.0;
         }
         if (k == nt - 1) break;
-        // ---- 2. L~_kk at comm(k,k) and its 128-block inverses (TRSM operand, Alg. 2 l.5-10)
+        // ---- 2. L~_kk at comm(k,k) and its 128-block inverses (TRSM operand, Alg. 2 l.5-10);
+        //      multi-rank: the owner publishes L~_kk in comm(k,k) precision, the TRSM owners of
+        //      column k pull it (fused transfer + up-conversion)
+        bool trsm_here = false;
+        for (int m = k + 1; m < nt; ++m) trsm_here |= A->mine(m, k);
         {
-            double* Akk = (double*)A->tile(k, k);
             const int pc = C(k, k);
-            cur->push_back({[=](cudaStream_t s) { return round_copy_launch(Akk, ltil, (int64_t)nb2, pc, s); }, C_TRSM, 0});
-            cur->push_back({[=](cudaStream_t s) { return trtri_blocks_launch(ltil, nb, wb2, s); }, C_TRSM, 0});
+            bool pub_kk = false;
+            int pull_kk = -1;
+            for (auto& x : xpub[k]) pub_kk |= x.m == k;
+            for (auto& x : xpull[k])
+                if (x.m == k) pull_kk = x.peer;
+            if (A->mine(k, k)) {
+                double* Akk = (double*)A->tile(k, k);
+                cur->push_back({[=](cudaStream_t s) { return round_copy_launch(Akk, ltil, (int64_t)nb2, pc, s); }, C_TRSM, 0});
+                if (pub_kk) {
+                    wait_send_free();
+                    std::vector<PackItem> pk{PackItem{ltil, sendslot(me, sp, k), pc, 0}};
+                    PackItem* dp = ar.push(pk);
+                    uint64_t* f = pubflag(me, sp, k);
+                    const uint64_t v = ST(k);
+                    cur_push(Op{[=](cudaStream_t s) { return pack_launch(dp, 1, (int64_t)nb2, s); }, C_CONV, 0});
+                    cur_push(Op{[=](cudaStream_t s) { return set_flag_launch(f, v, s); }, C_CONV, 0});
+                }
+            } else if (pull_kk >= 0) {
+                const int o = pull_kk;
+                std::vector<WaitItem> w{WaitItem{pubflag(o, sp, k), ST(k)}};
+                push_wait(w);
+                std::vector<PullItem> pl{PullItem{sendslot(o, sp, k), pubflag(o, sp, k), ST(k), ltil, nullptr, nullptr, nullptr, pc, 0}};
+                PullItem* dp = ar.push(pl);
+                cur_push(Op{[=](cudaStream_t s) { return pull_launch(dp, 1, (int64_t)nb2, s); }, C_CONV, 0});
+            }
+            if (trsm_here || !dist)
+                cur->push_back({[=](cudaStream_t s) { return trtri_blocks_launch(ltil, nb, wb2, s); }, C_TRSM, 0});
         }
         // ---- 3. panel in
         std::vector<PanelTile> pin, pout;
@@ -634,16 +802,9 @@ static mp_status plan_potrf(mp_handle* h, mp_matrix* A, const uint8_t* km, const
             t.store_prec = A->st(m, k);
             t.comm_prec = C(m, k);
             pin.push_back(t);
-            // which operand formats do the successors of L_mk need? (row m, column m)
+            // which operand formats do the successors of L_mk (row m, column m) on this GPU need?
             bool need16 = false, need32 = false;
-            for (int n = k + 1; n < m; ++n) {
-                need16 |= K(m, n) == MP_FP16;
-                need32 |= K(m, n) == MP_FP32;
-            }
-            for (int n = m + 1; n < nt; ++n) {
-                need16 |= K(n, m) == MP_FP16;
-                need32 |= K(n, m) == MP_FP32;
-            }
+            local_formats(k, m, need16, need32);
             if (use_tc) {
                 if (need16) t.p16 = p16 + (size_t)m * nb2;
                 if (need32) {
@@ -682,6 +843,56 @@ static mp_status plan_potrf(mp_handle* h, mp_matrix* A, const uint8_t* km, const
             fc.trsm += np * fnb * fnb * fnb;
             // ---- 5. panel out (K2)
             cur->push_back({[=](cudaStream_t s) { return panel_out_launch(d_out, np, (int64_t)nb2, s); }, C_CONV, 0});
+        }
+        if (dist) {
+            // ---- 5b. publish my L_mk (comm precision) for remote successors
+            std::vector<PackItem> packs;
+            std::vector<WaitItem> flags;  // (flag, value) pairs to set
+            for (auto& x : xpub[k]) {
+                const int m = x.m;
+                if (m == k) continue;
+                packs.push_back(PackItem{p64 + (size_t)m * nb2, sendslot(me, sp, m), C(m, k), 0});
+                flags.push_back(WaitItem{pubflag(me, sp, m), ST(k)});
+            }
+            if (!packs.empty()) {
+                wait_send_free();
+                PackItem* dp = ar.push(packs);
+                const int npk = (int)packs.size();
+                cur_push(Op{[=](cudaStream_t s) { return pack_launch(dp, npk, (int64_t)nb2, s); }, C_CONV, 0});
+                for (auto& f : flags) {
+                    uint64_t* fp = (uint64_t*)f.flag;
+                    const uint64_t v = f.target;
+                    cur_push(Op{[=](cudaStream_t s) { return set_flag_launch(fp, v, s); }, C_CONV, 0});
+                }
+            }
+            // ---- 5c. pull the remote L_mk my tiles need: peer payload -> FP64 panel slot + caches
+            std::vector<WaitItem> waits;
+            std::vector<PullItem> pulls;
+            for (auto& x : xpull[k]) {
+                const int m = x.m;
+                if (m == k) continue;
+                const int o = x.peer;
+                bool n16 = false, n32 = false;
+                local_formats(k, m, n16, n32);
+                PullItem it{sendslot(o, sp, m), pubflag(o, sp, m), ST(k), p64 + (size_t)m * nb2, nullptr, nullptr,
+                            nullptr, C(m, k), 0};
+                if (use_tc && n16) it.p16 = p16 + (size_t)m * nb2;
+                if (use_tc && n32) {
+                    it.hi = phi + (size_t)m * nb2;
+                    it.lo = plo + (size_t)m * nb2;
+                }
+                waits.push_back(WaitItem{it.flag, it.target});
+                pulls.push_back(it);
+            }
+            push_wait(waits);
+            if (!pulls.empty()) {
+                PullItem* dp = ar.push(pulls);
+                const int npl = (int)pulls.size();
+                cur_push(Op{[=](cudaStream_t s) { return pull_launch(dp, npl, (int64_t)nb2, s); }, C_CONV, 0});
+            }
+            uint64_t* df = doneflag(me, sp);
+            const uint64_t dv = ST(k);
+            cur_push(Op{[=](cudaStream_t s) { return set_flag_launch(df, dv, s); }, C_CONV, 0});
         }
         // ---- 6. trailing update: SYRK + GEMM grouped by kernel(m,n); the tiles of
         //      column k+1 (next) are emitted separately so panel k+1 can start as soon as they are done
@@ -728,7 +939,7 @@ static mp_status plan_potrf(mp_handle* h, mp_matrix* A, const uint8_t* km, const
         }  // part
     }
     // ---- assemble the schedule
-    if (!h->lookahead) {
+    if (!la) {
         for (int k = 0; k < nt; ++k)
             for (auto* v : {&pan[k], &nxt[k], &rst[k]})
                 for (auto& o : *v) ops.push_back(std::move(o));
@@ -763,7 +974,7 @@ static mp_status potrf_run(mp_handle* h, mp_matrix* A, const uint8_t* km, const 
     if (!h || !A || !km || !cm) return MP_ERR_ARG;
     if (h->broken) FAIL(h, MP_ERR_STATE, "handle unusable after an earlier CUDA failure");
     if (!A->bound || !A->generated) FAIL(h, MP_ERR_STATE, "matrix not generated");
-    if (h->nranks > 1) FAIL(h, MP_ERR_UNSUPPORTED, "multi-rank factorisation not in this build");
+    if (h->nranks > 1 && !A->comm.connected) FAIL(h, MP_ERR_COMM, "multi-rank matrix not connected");
     const int nt = A->nt;
     for (int k = 0; k < nt; ++k)
         for (int m = k; m < nt; ++m) {
@@ -780,7 +991,8 @@ static mp_status potrf_run(mp_handle* h, mp_matrix* A, const uint8_t* km, const 
     ar.dev_base = A->ws + A->R.ctrl;
     std::vector<Op> ops;
     FlopCount fc;
-    if (mp_status s = plan_potrf(h, A, km, cm, ar, ops, fc)) return s;
+    const uint64_t epoch = ++A->comm.epoch;
+    if (mp_status s = plan_potrf(h, A, km, cm, ar, ops, fc, epoch)) return s;
     if (mp_status s = run_plan(h, A, ar, ops)) return s;
     int hinfo = 0;
     CK(h, cudaMemcpyAsync(&hinfo, h->d_info, sizeof(int), cudaMemcpyDeviceToHost, h->stream));
@@ -804,13 +1016,143 @@ mp_status mp_tile_potrf(mp_handle* h, mp_matrix* A, const uint8_t* kernel_prec, 
 }
 
 // ------------------------------------------------------------------ (4) log-likelihood
+// Multi-rank forward solve (right-looking, 2D block-cyclic): rank (p, q) accumulates
+// racc_m = -sum_{own (m,j)} L_mj y_j; at step k the ranks of process row k mod P publish racc_k,
+// owner(k,k) forms r_k = z_k + sum_r racc_k^(r) (rank order), solves y_k = L_kk^{-1} r_k and
+// publishes y_k; the ranks of process column k mod Q read y_k straight from the owner's memory in
+// their GEMV.  log-determinant and y^T y partials are all-gathered and summed in rank order.
+static mp_status loglik_dist(mp_handle* h, mp_matrix* A, const double* d_z, double* loglik, double* logdet,
+                             double* quad) {
+    if (!A->comm.connected) FAIL(h, MP_ERR_COMM, "multi-rank matrix not connected");
+    Comm& X = A->comm;
+    const int nt = A->nt, nb = A->nb, P = h->P, Q = h->Q, me = h->rank;
+    const int myp = me / Q, myq = me % Q;
+    const int64_t n = A->n;
+    const uint64_t epoch = ++X.epoch;
+    auto ST = [&](int step) -> uint64_t { return (epoch << 24) + (uint64_t)(step + 2); };
+    if (mp_status st = dist_barrier(h, A, ST(-1))) return st;
+    double* racc = A->at<double>(A->R.vec_r);
+    double* zpad = A->at<double>(A->R.vec_y);
+    double* part = A->at<double>(A->R.partials);
+    CK(h, cudaMemsetAsync(racc, 0, (size_t)nt * nb * 8, h->stream));
+    CK(h, cudaMemsetAsync(zpad, 0, (size_t)nt * nb * 8, h->stream));
+    CK(h, cudaMemcpyAsync(zpad, d_z, (size_t)n * 8, cudaMemcpyDeviceToDevice, h->stream));
+    auto yslot = [&](int r, int k) { return (double*)(X.peer[r] + X.yv) + (size_t)k * nb; };
+    auto yflag = [&](int r, int k) { return (uint64_t*)(X.peer[r] + X.yflag) + k; };
+    auto pslot = [&](int r, int k) { return (double*)(X.peer[r] + X.part) + (size_t)k * nb; };
+    auto pflag = [&](int r, int k) { return (uint64_t*)(X.peer[r] + X.pflag) + k; };
+    Arena ar;
+    ar.dev_base = A->ws + A->R.ctrl;
+    std::vector<Op> ops;
+    std::vector<const double*> diag;
+    std::vector<int> nreal;
+    auto wait_op = [&](std::vector<WaitItem> w) {
+        if (w.empty()) return;
+        WaitItem* dw = ar.push(w);
+        const int nw = (int)w.size();
+        ops.push_back({[=](cudaStream_t s) { return wait_flags_launch(dw, nw, s); }, C_SOLVE, 0});
+    };
+    for (int k = 0; k < nt; ++k) {
+        if (myp == k % P) {  // publish my partial of row k
+            double* src = racc + (size_t)k * nb;
+            double* dst = pslot(me, k);
+            uint64_t* f = pflag(me, k);
+            const uint64_t v = ST(k);
+            ops.push_back({[=](cudaStream_t s) { return cudaMemcpyAsync(dst, src, (size_t)nb * 8, cudaMemcpyDeviceToDevice, s); },
+                           C_SOLVE, 0});
+            ops.push_back({[=](cudaStream_t s) { return set_flag_launch(f, v, s); }, C_SOLVE, 0});
+        }
+        const int o = A->owner(k, k);
+        if (o == me) {
+            std::vector<WaitItem> w;
+            GatherItem g{};
+            g.base = zpad + (size_t)k * nb;
+            g.n = 0;
+            for (int q = 0; q < Q; ++q) {
+                const int r = (k % P) * Q + q;
+                if (r != me) w.push_back(WaitItem{pflag(r, k), ST(k)});
+                g.src[g.n++] = pslot(r, k);
+            }
+            wait_op(w);
+            double* tmp = (double*)(X.base + X.tmp);
+            g.dst = tmp;
+            ops.push_back({[=](cudaStream_t s) { return gather_add_launch(g, nb, s); }, C_SOLVE, 0});
+            const double* Lkk = (const double*)A->tile(k, k);
+            double* yk = yslot(me, k);
+            ops.push_back({[=](cudaStream_t s) { return trsv_tile_launch(Lkk, nb, tmp, yk, s); }, C_SOLVE, 0});
+            uint64_t* f = yflag(me, k);
+            const uint64_t v = ST(k);
+            ops.push_back({[=](cudaStream_t s) { return set_flag_launch(f, v, s); }, C_SOLVE, 0});
+            diag.push_back(Lkk);
+            nreal.push_back((int)std::min<int64_t>(nb, n - (int64_t)k * nb));
+        }
+        if (myq == k % Q) {
+            std::vector<GemvTile> gv;
+            for (int m = k + 1; m < nt; ++m)
+                if (A->mine(m, k)) gv.push_back(GemvTile{A->tile(m, k), A->st(m, k), 0, racc + (size_t)m * nb});
+            if (!gv.empty()) {
+                if (o != me) wait_op({WaitItem{yflag(o, k), ST(k)}});
+                GemvTile* dg = ar.push(gv);
+                const int ng = (int)gv.size();
+                const double* yk = yslot(o, k);  // peer memory when o != me (NVLink / IPC load)
+                ops.push_back({[=](cudaStream_t s) { return gemv_sub_launch(dg, ng, yk, nb, s); }, C_SOLVE, 0});
+            }
+        }
+    }
+    // local partials: log diag of my diagonal tiles, y^T y of my y_k (slots of other k are unused)
+    const int nd = (int)diag.size();
+    std::vector<int> myk;
+    for (int k = 0; k < nt; ++k)
+        if (A->owner(k, k) == me) myk.push_back(k);
+    if (nd) {
+        const double* const* d_diag = ar.push(diag);
+        const int* d_nreal = ar.push(nreal);
+        ops.push_back({[=](cudaStream_t s) { return logdiag_launch(d_diag, d_nreal, nd, nb, part, s); }, C_SOLVE, 0});
+        double* ybase = yslot(me, 0);
+        const int ntt = nt;
+        ops.push_back({[=](cudaStream_t s) { return sumsq_chunks_launch(ybase, (int64_t)ntt * nb, nb, part + nd, s); },
+                       C_SOLVE, 0});
+    }
+    if (mp_status st = run_plan(h, A, ar, ops)) return st;
+    std::vector<double> hp(nd + nt, 0.0);
+    if (nd) CK(h, cudaMemcpyAsync(hp.data(), part, hp.size() * 8, cudaMemcpyDeviceToHost, h->stream));
+    CK(h, cudaStreamSynchronize(h->stream));
+    double sc[2] = {0.0, 0.0};
+    for (int i = 0; i < nd; ++i) sc[0] += hp[i];
+    for (int k : myk) sc[1] += hp[nd + k];
+    CK(h, cudaMemcpy(X.base + X.scal, sc, sizeof sc, cudaMemcpyHostToDevice));
+    CK(h, set_flag_launch((uint64_t*)(X.base + X.sflag), ST(nt), h->stream));
+    CK(h, cudaStreamSynchronize(h->stream));
+    double ld = 0.0, q = 0.0;
+    for (int r = 0; r < h->nranks; ++r) {
+        double v[2];
+        if (r != me) {
+            if (mp_status st = host_wait_stamp(h, (const uint64_t*)(X.peer[r] + X.sflag), ST(nt))) return st;
+            CK(h, cudaMemcpy(v, X.peer[r] + X.scal, sizeof v, cudaMemcpyDeviceToHost));
+        } else {
+            v[0] = sc[0];
+            v[1] = sc[1];
+        }
+        ld += v[0];
+        q += v[1];
+    }
+    ld *= 2.0;
+    // closing barrier: nobody reuses the exchange area while a peer still reads it
+    if (mp_status st = dist_barrier(h, A, ST(nt + 1))) return st;
+    const double ll = -0.5 * (double)n * std::log(2.0 * M_PI) - 0.5 * ld - 0.5 * q;
+    if (loglik) *loglik = ll;
+    if (logdet) *logdet = ld;
+    if (quad) *quad = q;
+    return MP_OK;
+}
+
 mp_status mp_loglik(mp_handle* h, const mp_matrix* Lc, const double* d_z, double* loglik, double* logdet,
                     double* quad) {
     mp_matrix* A = const_cast<mp_matrix*>(Lc);
     if (!h || !A || !d_z) return MP_ERR_ARG;
     if (h->broken) FAIL(h, MP_ERR_STATE, "handle unusable after an earlier CUDA failure");
     if (!A->factored) FAIL(h, MP_ERR_STATE, "matrix not factored");
-    if (h->nranks > 1) FAIL(h, MP_ERR_UNSUPPORTED, "multi-rank solve not in this build");
+    if (h->nranks > 1) return loglik_dist(h, A, d_z, loglik, logdet, quad);
     const int nt = A->nt, nb = A->nb;
     const int64_t n = A->n;
     double* r = A->at<double>(A->R.vec_r);
