@@ -14,9 +14,11 @@ larger than L2, so no explicit flush is needed between steps.
   python bench.py [--gpus N] [--steps K] [--warmup W] [--config c3] [--map adaptive]
   python bench.py --impl reference ...   # the CPU oracle on a bounded sample (the reference arm)
 
-N > 1 (torchrun): each rank evaluates its own replica (weak scaling, no collective on the data
-path; the Monte-Carlo MLE study of P:264 is embarrassingly parallel over replicas); time is the
-max over ranks and value is the flops of all ranks / that time.
+N > 1 (torchrun, one process per GPU): ONE evaluation distributed over a P x Q process grid (as
+square as possible, P <= Q; 2 -> 1x2, 4 -> 2x2, 8 -> 2x4), 2D block-cyclic tiles, panel
+tiles exchanged through peer memory in their communication precision; same
+workload as N = 1 (strong scaling); time is the max over ranks.  `--replicas` instead runs one
+independent evaluation per rank (weak scaling, no data-path exchange).
 """
 from __future__ import annotations
 
@@ -37,6 +39,7 @@ CONFIGS = {
     "c1": dict(n=1600, nb=400, theta=(1.0, 0.1, 0.5), map="fp64"),
     "c2": dict(n=40000, nb=2048, theta=(1.0, 0.03, 0.5), map="band"),
     "c3": dict(n=160000, nb=2048, theta=(1.0, 0.03, 0.5), map="adaptive"),
+    "c4": dict(n=360000, nb=2048, theta=(1.0, 0.03, 0.5), map="adaptive"),  # 8 GPUs (2x4)
     "c5": dict(n=250000, nb=2048, theta=(1.0, 0.03, 0.5), map="adaptive"),
 }
 METRIC = "Tflop/s & joules per MLE log-likelihood eval (n=360k) at 1/2/4/8 B200"
@@ -195,6 +198,7 @@ def main():
     ap.add_argument("--u-req", type=float, default=1e-9)
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--replicas", action="store_true", help="N>1: independent evaluations per rank")
     args = ap.parse_args()
     cfg = dict(CONFIGS[args.config])
     if args.map:
@@ -223,11 +227,22 @@ def main():
     mode = {"adaptive": mp.MP_MAP_ADAPTIVE, "fp64": mp.MP_MAP_FP64, "band": mp.MP_MAP_BAND,
             "extreme": mp.MP_MAP_EXTREME}[cfg["map"]]
     policy = mp.MP_COMM_AUTO if args.policy == "auto" else mp.MP_COMM_TTC
-    x, y = synth.locations(n, seed=rank)
-    z = synth.normal_vector(n, seed=1 + rank)
+    distributed = world > 1 and not args.replicas
+    seed = 0 if distributed or world == 1 else rank
+    x, y = synth.locations(n, seed=seed)
+    z = synth.normal_vector(n, seed=1 + seed)
     dx, dy, dz = (torch.from_numpy(a).cuda() for a in (x, y, z))
     hx, hy, hz = (torch.from_numpy(a).pin_memory() for a in (x, y, z))
-    ev = mp.Evaluator(n, nb, device=local)
+    if distributed:
+        P = int(math.isqrt(world))
+        while world % P:
+            P -= 1
+        Q = world // P
+        handle = mp.Handle(local, rank, world, P, Q)
+        ev = mp.Evaluator(n, nb, handle=handle)
+    else:
+        P = Q = 1
+        ev = mp.Evaluator(n, nb, device=local)
     h = ev.handle
     stream = h.stream
 
@@ -275,7 +290,8 @@ def main():
         dist.all_reduce(t)
         joules = float(t.item())
     flops_eval = n**3 / 3.0
-    value = world * args.steps * flops_eval / (t_ms / 1e3) / 1e12
+    evals_per_step = 1 if distributed else world
+    value = evals_per_step * args.steps * flops_eval / (t_ms / 1e3) / 1e12
 
     # ---- e2e: same metric through mp_eval with pinned HOST inputs (H2D inside the call) and the
     # results (norms, info, partial sums, scalars) read back to the host every step
@@ -297,7 +313,7 @@ def main():
         chunks = (n + 4095) // 4096
         d2h = (nt * (nt + 1) // 2) * 8 if mode in (mp.MP_MAP_ADAPTIVE, mp.MP_MAP_BAND) else 0
         d2h += 4 + (nt + chunks) * 8
-        e2e = {"value": world * args.steps * flops_eval / (te / 1e3) / 1e12, "unit": "Tflop/s",
+        e2e = {"value": evals_per_step * args.steps * flops_eval / (te / 1e3) / 1e12, "unit": "Tflop/s",
                "h2d_bytes_per_step": 3 * n * 8, "d2h_bytes_per_step": d2h, "ms_per_step": te / args.steps}
 
     if rank != 0:
@@ -321,12 +337,14 @@ def main():
     t_upd_s = (p["upd_fp64"]["ms"] + p["upd_fp32"]["ms"] + p["upd_fp16"]["ms"]) / 1e3 / args.steps
     out = {
         "metric": METRIC, "value": value, "unit": "Tflop/s", "n_gpus": world, "steps": args.steps,
-        "warmup": args.warmup, "ms_per_step": t_ms / args.steps, "higher_is_better": True, "scaling": "weak",
+        "warmup": args.warmup, "ms_per_step": t_ms / args.steps, "higher_is_better": True,
+        "scaling": "strong" if distributed else "weak",
         "vs_baseline": None, "dtype": "f64", "data": "synthetic",
         "config": {"workload": f"{args.config}: n={n} ({int(math.isqrt(n))}^2 jittered grid, Morton order), nb={nb}, "
                                f"theta={list(theta)}, {cfg['map']} map u_req={args.u_req}, comm={args.policy}",
                    "n": n, "nb": nb, "map": cfg["map"], "policy": args.policy,
-                   "parallelism": "replicas" if world > 1 else "1 GPU",
+                   "parallelism": (f"2D block-cyclic {P}x{Q}, peer-memory panel exchange" if distributed
+                                   else ("replicas" if world > 1 else "1 GPU")),
                    "l2": "matrix (~%.0f GB) >> 126 MB L2; no flush needed" % (n * n / 2 * 5 / 1e9)},
         "joules_per_eval": None if joules is None else joules / args.steps,
         "loglik": last.loglik, "tiles_fp64_fp32_fp16": list(last.tiles), "stc_tiles": last.stc_tiles,

@@ -88,6 +88,7 @@ def _load() -> C.CDLL:
         "mp_test_dgemm": (i32, [vp, vp, vp, i32, i32, i32, i32, i32, i32, i32, dbl, dbl, i32, i32]),
         "mp_test_tc_gemm": (i32, [i32, vp, vp, vp, i32, i32, i32, i32]),
         "mp_tc_available": (i32, []),
+        "mp_test_ozaki_gemm": (i32, [vp, vp, i32, i32, i32, i32, i32, i32]),
     }
     for name, (res, args) in sig.items():
         f = getattr(lib, name)

@@ -28,6 +28,7 @@
 #include "kernels.h"
 #include "tc_gemm.h"
 #include "dist.h"
+#include "ozaki.h"
 
 using namespace mpgeo;
 
@@ -48,6 +49,7 @@ struct mp_handle {
     bool broken = false;
     int tc_mode = 1;  // 1: tcgen05 kernels for FP32/FP16 classes when available, 0: DMMA emulation
     int lookahead = 1;  // 1: panel k+1 on the high-priority panel stream overlaps update k
+    int ozaki = 0;      // S in {7, 8}: FP64-class GEMM/SYRK emulated on INT8 tensor cores; 0: DMMA
     cudaStream_t pstream = nullptr;
     std::vector<cudaEvent_t> sync_ev;
     // profiling (mp_set_profiling): event pairs per launch, resolved in mp_get_profile
@@ -60,7 +62,7 @@ struct mp_handle {
 
 struct Regions {
     size_t total = 0;
-    size_t inputs = 0, p64 = 0, p16 = 0, phi = 0, plo = 0, ltilde = 0, wbuf = 0, wbuf2 = 0;
+    size_t inputs = 0, p64 = 0, p16 = 0, phi = 0, plo = 0, ltilde = 0, wbuf = 0, wbuf2 = 0, oz = 0, ozexp = 0;
     size_t vec_r = 0, vec_y = 0, partials = 0, norms = 0, ctrl = 0, ctrl_bytes = 0;
     std::vector<size_t> tile_off;  // per (m*nt+k), SIZE_MAX if not stored here
 };
@@ -126,6 +128,7 @@ static size_t ctrl_bytes_for(int nt, int nb) {
     bytes += T * T * sizeof(GemvTile);
     bytes += T * (sizeof(double*) + sizeof(int));
     bytes += T * T * (sizeof(PackItem) + sizeof(PullItem) + 2 * sizeof(WaitItem)) + T * 8 * sizeof(WaitItem);
+    bytes += T * T * sizeof(OzSplitItem) + T * (T + 1) * (T + 2) / 6 * sizeof(OzJob);
     bytes += 64 * 1024 + 32 * 256;  // alignment slack
     return bytes;
 }
@@ -160,6 +163,8 @@ static Regions layout(const mp_matrix* A, const uint8_t* storage) {
     R.p16 = take(2 * (size_t)nt * nb2 * 2);
     R.phi = take(2 * (size_t)nt * nb2 * 4);
     R.plo = take(2 * (size_t)nt * nb2 * 4);
+    R.oz = take(2 * (size_t)nt * nb2 * 8);         // Ozaki int8 slice planes (S <= 8), two sets
+    R.ozexp = take(2 * (size_t)nt * A->nb * 4);    // per-row exponents
     R.tile_off.assign((size_t)nt * nt, SIZE_MAX);
     for (int k = 0; k < nt; ++k)
         for (int m = k; m < nt; ++m)
@@ -262,6 +267,7 @@ mp_status mp_init(int device, int rank, int nranks, int P, int Q, const uint8_t*
     h->Q = Q;
     if (const char* e = getenv("MPGEO_TC")) h->tc_mode = atoi(e);
     if (const char* e = getenv("MPGEO_LOOKAHEAD")) h->lookahead = atoi(e);
+    if (const char* e = getenv("MPGEO_OZAKI")) h->ozaki = atoi(e);
     auto fail = [&](mp_status s) {
         if (h->own_stream && h->stream) cudaStreamDestroy(h->stream);
         delete h;
@@ -637,6 +643,9 @@ static mp_status plan_potrf(mp_handle* h, mp_matrix* A, const uint8_t* km, const
     double* wb2 = A->at<double>(A->R.wbuf2);
     int* d_info = h->d_info;
     const bool use_tc = h->tc_mode != 0 && tc_gemm_available() && nb % 256 == 0;
+    const int ozS = (h->ozaki == 7 || h->ozaki == 8) && ozaki_available() && nb % 128 == 0 ? h->ozaki : 0;
+    int8_t* const ozb = A->at<int8_t>(A->R.oz);
+    int* const ozeb = A->at<int>(A->R.ozexp);
     auto K = [&](int m, int k) { return km[(size_t)m * nt + k]; };
     auto C = [&](int m, int k) { return cm[(size_t)m * nt + k]; };
     const double fnb = (double)nb;
@@ -712,6 +721,9 @@ static mp_status plan_potrf(mp_handle* h, mp_matrix* A, const uint8_t* km, const
         __half* p16 = p16b + set * nt * nb2;
         float* phi = phib + set * nt * nb2;
         float* plo = plob + set * nt * nb2;
+        int8_t* ozs = ozb + set * nt * nb2 * 8;
+        int* oze = ozeb + set * (size_t)nt * nb;
+        const int64_t ozplane = (int64_t)nt * nb2;
         cur = &pan[k];
         // ---- 1. DPOTRF(k,k), FP64: two-level blocking — 128-column blocks
         //      (diagonal block Cholesky + inverse, block column as GEMM with the inverse, update
@@ -894,6 +906,22 @@ static mp_status plan_potrf(mp_handle* h, mp_matrix* A, const uint8_t* km, const
             const uint64_t dv = ST(k);
             cur_push(Op{[=](cudaStream_t s) { return set_flag_launch(df, dv, s); }, C_CONV, 0});
         }
+        // ---- 5d. Ozaki: split every panel tile this GPU's FP64-class successors read into int8 slices
+        if (ozS) {
+            std::vector<OzSplitItem> sp;
+            for (int m = k + 1; m < nt; ++m) {
+                bool need = A->mine(m, m);
+                for (int n = k + 1; n < m && !need; ++n) need |= A->mine(m, n) && K(m, n) == MP_FP64;
+                for (int n = m + 1; n < nt && !need; ++n) need |= A->mine(n, m) && K(n, m) == MP_FP64;
+                if (need)
+                    sp.push_back(OzSplitItem{p64 + (size_t)m * nb2, ozs + (size_t)m * nb2, oze + (size_t)m * nb, ozplane});
+            }
+            if (!sp.empty()) {
+                OzSplitItem* dsp = ar.push(sp);
+                const int nsp = (int)sp.size();
+                cur_push(Op{[=](cudaStream_t s) { return ozaki_split_launch(dsp, nsp, nb, ozS, s); }, C_CONV, 0});
+            }
+        }
         // ---- 6. trailing update: SYRK + GEMM grouped by kernel(m,n); the tiles of
         //      column k+1 (next) are emitted separately so panel k+1 can start as soon as they are done
         for (int part = 0; part < 2; ++part) {
@@ -919,6 +947,24 @@ static mp_status plan_potrf(mp_handle* h, mp_matrix* A, const uint8_t* km, const
             }
         }
         const double f3 = fnb * fnb * fnb;
+        if (ozS) {  // FP64 class on INT8 tensor cores
+            for (int lower = 1; lower >= 0; --lower) {
+                std::vector<OzJob> oj;
+                for (auto& g : (lower ? syrk : g64)) {
+                    const int mm = (int)(((const double*)g.A - p64) / (ptrdiff_t)nb2);
+                    const int nn = (int)(((const double*)g.B - p64) / (ptrdiff_t)nb2);
+                    oj.push_back(OzJob{mm, nn, (double*)g.C});
+                }
+                if (oj.empty()) continue;
+                OzJob* dj = ar.push(oj);
+                const int nj = (int)oj.size();
+                OzArgs oa{dj, ozs, oze, ozplane, nb, nt, ozS, lower};
+                cur_push(Op{[=](cudaStream_t s) { return ozaki_gemm_launch(oa, nj, s); }, C_UPD64,
+                            (lower ? f3 : 2 * f3) * nj});
+            }
+            syrk.clear();
+            g64.clear();
+        }
         gemm(syrk, nb, nb, nb, nb, nb, nb, 1, -1.0, 1.0, P64, false, C_UPD64, f3);
         gemm(g64, nb, nb, nb, nb, nb, nb, 0, -1.0, 1.0, P64, false, C_UPD64, 2 * f3);
         gemm(g32, nb, nb, nb, nb, nb, nb, 0, -1.0, 1.0, P32, true, C_UPD32, 2 * f3);

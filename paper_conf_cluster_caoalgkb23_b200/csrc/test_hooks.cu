@@ -1,7 +1,10 @@
 // Kernel-level test hooks (include/mpgeo_test.h).  Not on the hot path.
 #include "../../include/mpgeo_test.h"
+#include <vector>
+
 #include "kernels.h"
 #include "tc_gemm.h"
+#include "ozaki.h"
 
 using namespace mpgeo;
 
@@ -62,5 +65,32 @@ mp_status mp_test_tc_gemm(int kind, const void* d_panel, const void* d_panel_lo,
 }
 
 int mp_tc_available(void) { return tc_gemm_available() ? 1 : 0; }
+
+mp_status mp_test_ozaki_gemm(const double* d_panel, double* d_C, int nb, int nt, int m, int n, int S, int lower) {
+    if (!ozaki_available()) return MP_ERR_UNSUPPORTED;
+    const int64_t plane = (int64_t)nt * nb * nb;
+    int8_t* sl = nullptr;
+    int* ex = nullptr;
+    OzSplitItem* it = nullptr;
+    OzJob* dj = nullptr;
+    if (cudaMalloc(&sl, plane * S) || cudaMalloc(&ex, sizeof(int) * nt * nb) ||
+        cudaMalloc(&it, sizeof(OzSplitItem) * nt) || cudaMalloc(&dj, sizeof(OzJob)))
+        return MP_ERR_CUDA;
+    std::vector<OzSplitItem> h(nt);
+    for (int t = 0; t < nt; ++t)
+        h[t] = OzSplitItem{d_panel + (size_t)t * nb * nb, sl + (size_t)t * nb * nb, ex + (size_t)t * nb, plane};
+    cudaMemcpy(it, h.data(), sizeof(OzSplitItem) * nt, cudaMemcpyHostToDevice);
+    OzJob j{m, n, d_C};
+    cudaMemcpy(dj, &j, sizeof j, cudaMemcpyHostToDevice);
+    cudaError_t e = ozaki_split_launch(it, nt, nb, S, 0);
+    OzArgs a{dj, sl, ex, plane, nb, nt, S, lower};
+    if (e == cudaSuccess) e = ozaki_gemm_launch(a, 1, 0);
+    cudaError_t e2 = cudaDeviceSynchronize();
+    cudaFree(sl);
+    cudaFree(ex);
+    cudaFree(it);
+    cudaFree(dj);
+    return (e == cudaSuccess && e2 == cudaSuccess) ? MP_OK : MP_ERR_CUDA;
+}
 
 }  // extern "C"

@@ -123,3 +123,34 @@ def test_tc_gemm_tf32x3_matches_sgemm_accuracy(lib):
     err_1x = np.linalg.norm(single - exact) / np.linalg.norm(exact)
     assert err_tc <= 2 * err_sg + 1e-9, (err_tc, err_sg)
     assert err_tc < err_1x / 50  # far better than a single TF32 product
+
+
+@pytest.mark.parametrize("S", [7, 8])
+def test_ozaki_int8_fp64_gemm(lib, S):
+    """FP64 GEMM emulated with int8 slices on tcgen05 kind::i8 vs the exact FP64 product: for S = 8
+    the error stays within a few units of an FP64 GEMM's (|err| <= 8 K u max|a| max|b|)."""
+    nb, nt = 512, 3
+    rng = np.random.default_rng(S)
+    P = rng.standard_normal((nt * nb, nb)) * np.exp(rng.uniform(-3, 3, (nt * nb, 1)))  # row scales vary
+    Cm = rng.standard_normal((nb, nb))
+    dP, dC = dev(P), dev(Cm)
+    assert lib.mp_test_ozaki_gemm(C.c_void_p(dP.data_ptr()), C.c_void_p(dC.data_ptr()), nb, nt, 2, 0, S, 0) == 0
+    got = dC.cpu().numpy()
+    A, B = P[2 * nb:], P[:nb]
+    ref = Cm - A @ B.T
+    scale = np.abs(A).max(axis=1)[:, None] * np.abs(B).max(axis=1)[None, :]
+    err = np.max(np.abs(got - ref) / scale)
+    bound = {8: 8 * nb * 2.0**-53, 7: 8 * nb * 2.0**-46}[S]
+    assert err <= bound, (S, err, bound)
+    # lower-only (SYRK) variant leaves strictly-upper 128x64 blocks untouched
+    dC2 = dev(Cm)
+    assert lib.mp_test_ozaki_gemm(C.c_void_p(dP.data_ptr()), C.c_void_p(dC2.data_ptr()), nb, nt, 1, 1, S, 1) == 0
+    got2 = dC2.cpu().numpy()
+    ref2 = Cm - P[nb:2 * nb] @ P[nb:2 * nb].T
+    for bi in range(nb // 128):
+        for bj in range(nb // 64):
+            blk = (slice(bi * 128, (bi + 1) * 128), slice(bj * 64, (bj + 1) * 64))
+            if bj * 64 > bi * 128 + 127:
+                assert np.array_equal(got2[blk], Cm[blk])
+            else:
+                assert np.max(np.abs(got2[blk] - ref2[blk])) <= 1e-9
