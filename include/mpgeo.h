@@ -79,6 +79,12 @@ typedef enum {
     MP_MAP_USER = 4       /* kernel_prec supplied by the caller */
 } mp_map_mode;
 
+/* Covariance family of the generated matrix (§III-A). */
+typedef enum {
+    MP_COV_MATERN = 0,  /* sigma^2 2^(1-nu)/Gamma(nu) (h/beta)^nu K_nu(h/beta), theta = {sigma^2, beta, nu} */
+    MP_COV_SQEXP = 1    /* sigma^2 exp(-h^2/beta), theta = {sigma^2, beta, unused} */
+} mp_covariance;
+
 typedef struct mp_handle mp_handle;
 typedef struct mp_matrix mp_matrix;
 
@@ -221,6 +227,9 @@ mp_status mp_eval(mp_handle* h, mp_matrix* A, const double* x, const double* y, 
 /* Maps used by the last mp_eval on A (host NT*NT arrays; any may be NULL). */
 mp_status mp_matrix_maps(const mp_matrix* A, uint8_t* kernel_prec, uint8_t* storage_prec,
                          uint8_t* comm_prec);
+
+/* Select the covariance family mp_matern_gen / mp_eval generate for A (default MP_COV_MATERN). */
+mp_status mp_matrix_set_covariance(mp_matrix* A, mp_covariance kind);
 
 /* Copy owned tile (m, k) of A to host as FP64 nb x nb row-major (padding
  * included), for tests.  Returns MP_ERR_ARG if (m, k) is not owned here. */

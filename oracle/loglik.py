@@ -50,13 +50,13 @@ def loglik_from_factor(factor: dict, z: np.ndarray, nt: int, nb: int) -> tuple[f
     return ll, ld, q
 
 
-def loglik(x, y, z, theta, nb: int, maps=None) -> dict:
+def loglik(x, y, z, theta, nb: int, maps=None, kernel: str = "matern") -> dict:
     """One full evaluation: generate tiles, factor (Alg. 1), Eq. (1).
 
     maps=None -> the FP64 definition; maps=(kernel, storage, comm) -> MP emulation."""
     n = x.shape[0]
     nt = num_tiles(n, nb)
-    tiles = gen_lower_tiles(x, y, theta, nb)
+    tiles = gen_lower_tiles(x, y, theta, nb, kernel)
     if maps is None:
         fac = tile_cholesky(tiles, nt, nb)
     else:

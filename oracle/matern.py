@@ -37,6 +37,21 @@ def matern(h, sigma2: float, beta: float, nu: float):
     return out
 
 
+def sqexp(h, sigma2: float, beta: float):
+    """2D/3D squared exponential, P:81 (§III-A item 1): C(h; theta) = sigma^2 exp(-h^2 / beta)."""
+    h = np.asarray(h, dtype=np.float64)
+    return sigma2 * np.exp(-(h * h) / beta)
+
+
+def covariance(h, theta, kernel: str = "matern"):
+    """C(h; theta) for the two covariance families of the paper."""
+    if kernel == "matern":
+        return matern(h, theta[0], theta[1], theta[2])
+    if kernel == "sqexp":
+        return sqexp(h, theta[0], theta[1])
+    raise ValueError(kernel)
+
+
 def matern_closed_form(h, sigma2: float, beta: float, nu: float):
     """Elementary forms of P:82 for half-integer nu:
     nu=1/2: e^-r;  nu=3/2: (1+r) e^-r;  nu=5/2: (1 + r + r^2/3) e^-r,  r = h/beta."""

@@ -19,7 +19,7 @@ import math
 
 import numpy as np
 
-from .matern import distance, matern
+from .matern import covariance, distance, matern
 
 
 def num_tiles(n: int, nb: int) -> int:
@@ -30,20 +30,19 @@ def tile_range(i: int, n: int, nb: int) -> tuple[int, int]:
     return i * nb, min(n, (i + 1) * nb)
 
 
-def gen_tile(x, y, theta, m: int, k: int, nb: int) -> np.ndarray:
-    """Sigma_ij = C(||s_i - s_j||; theta) for i in tile row m, j in tile column k (P:75, P:82)."""
+def gen_tile(x, y, theta, m: int, k: int, nb: int, kernel: str = "matern") -> np.ndarray:
+    """Sigma_ij = C(||s_i - s_j||; theta) for i in tile row m, j in tile column k (P:75, P:81-82)."""
     n = x.shape[0]
     r0, r1 = tile_range(m, n, nb)
     c0, c1 = tile_range(k, n, nb)
     h = distance(x[r0:r1, None], y[r0:r1, None], x[None, c0:c1], y[None, c0:c1])
-    sigma2, beta, nu = theta
-    return matern(h, sigma2, beta, nu)
+    return covariance(h, theta, kernel)
 
 
-def gen_lower_tiles(x, y, theta, nb: int) -> dict:
+def gen_lower_tiles(x, y, theta, nb: int, kernel: str = "matern") -> dict:
     """All lower tiles {(m, k): ndarray} of Sigma(theta)."""
     nt = num_tiles(x.shape[0], nb)
-    return {(m, k): gen_tile(x, y, theta, m, k, nb) for k in range(nt) for m in range(k, nt)}
+    return {(m, k): gen_tile(x, y, theta, m, k, nb, kernel) for k in range(nt) for m in range(k, nt)}
 
 
 def dense_covariance(x, y, theta) -> np.ndarray:

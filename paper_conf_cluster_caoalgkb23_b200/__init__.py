@@ -17,7 +17,7 @@ import numpy as np
 
 from ._lib import (EvalReport, MpError, Profile, PROF_CLASSES, lib, MP_OK, MP_ERR_NOT_SPD, MP_FP64, MP_FP32, MP_FP16,  # noqa: F401
                    MP_COMM_TTC, MP_COMM_AUTO, MP_MAP_ADAPTIVE, MP_MAP_FP64, MP_MAP_BAND, MP_MAP_EXTREME,
-                   MP_MAP_USER)
+                   MP_MAP_USER, MP_COV_MATERN, MP_COV_SQEXP)
 
 __all__ = ["Handle", "Matrix", "Evaluator", "precision_map", "exchange_plan", "exact_sum", "MpError", "EvalReport"]
 
@@ -137,6 +137,10 @@ class Matrix:
         self.handle.check(lib.mp_matrix_get_tile(self.handle.h, self.A, m, k, _d(out)))
         return out
 
+    def set_covariance(self, kind: int):
+        """MP_COV_MATERN (P:82, default) or MP_COV_SQEXP (P:81)."""
+        self.handle.check(lib.mp_matrix_set_covariance(self.A, kind))
+
     def set_tile(self, m: int, k: int, t: np.ndarray):
         t = np.ascontiguousarray(t, dtype=np.float64)
         assert t.shape == (self.nb, self.nb)
@@ -232,9 +236,12 @@ def exact_sum(v: np.ndarray) -> float:
 class Evaluator:
     """One log-likelihood evaluation per call (mp_eval) on a worst-case (all-FP64) workspace."""
 
-    def __init__(self, n: int, nb: int, device: int = 0, handle: Handle | None = None, group=None):
+    def __init__(self, n: int, nb: int, device: int = 0, handle: Handle | None = None, group=None,
+                 covariance: int = MP_COV_MATERN):
         self.handle = handle or Handle(device)
         self.M = Matrix(self.handle, n, nb, None, group=group)
+        if covariance != MP_COV_MATERN:
+            self.M.set_covariance(covariance)
         self.n, self.nb, self.nt = n, nb, self.M.nt
 
     def eval(self, x, y, z, theta, u_req: float = 1e-9, mode: int = MP_MAP_ADAPTIVE, policy: int = MP_COMM_AUTO,

@@ -18,6 +18,7 @@ STATUS_NAMES = ["MP_OK", "MP_ERR_ARG", "MP_ERR_NOT_SPD", "MP_ERR_CUDA", "MP_ERR_
 MP_FP64, MP_FP32, MP_FP16 = 0, 1, 2
 MP_COMM_TTC, MP_COMM_AUTO = 0, 1
 MP_MAP_ADAPTIVE, MP_MAP_FP64, MP_MAP_BAND, MP_MAP_EXTREME, MP_MAP_USER = range(5)
+MP_COV_MATERN, MP_COV_SQEXP = 0, 1
 
 
 class EvalReport(C.Structure):
@@ -74,6 +75,7 @@ def _load() -> C.CDLL:
         "mp_matrix_maps": (i32, [vp, u8p, u8p, u8p]),
         "mp_matrix_get_tile": (i32, [vp, vp, i32, i32, dp]),
         "mp_matrix_set_tile": (i32, [vp, vp, i32, i32, dp]),
+        "mp_matrix_set_covariance": (i32, [vp, i32]),
         "mp_matrix_comm_export": (i32, [vp, vp]),
         "mp_matrix_comm_connect": (i32, [vp, vp]),
         "mp_exchange_plan": (i32, [i32, i32, i32, i32, u8p, C.POINTER(Xfer), i64, C.POINTER(i64)]),

@@ -87,6 +87,7 @@ struct mp_matrix {
     char* ws = nullptr;
     size_t ws_bytes = 0;
     bool bound = false, generated = false, factored = false;
+    int cov = MP_COV_MATERN;
     std::vector<uint8_t> storage, kmap, cmap;
     Regions R;
     int owner(int m, int k) const { return (m % h->P) * h->Q + (k % h->Q); }
@@ -531,10 +532,18 @@ static mp_status dist_barrier(mp_handle* h, mp_matrix* A, uint64_t stamp) {
 }
 
 // ------------------------------------------------------------------ (1) generation
-static mp_status check_theta(mp_handle* h, const double* th) {
-    if (!th || !(th[0] > 0) || !(th[1] > 0) || !(th[2] > 0) || !(th[2] <= 20.0) || !std::isfinite(th[0]) ||
-        !std::isfinite(th[1]))
-        FAIL(h, MP_ERR_ARG, "invalid theta (sigma2, beta > 0, 0 < nu <= 20)");
+static mp_status check_theta(mp_handle* h, const double* th, int cov = MP_COV_MATERN) {
+    if (!th || !(th[0] > 0) || !(th[1] > 0) || !std::isfinite(th[0]) || !std::isfinite(th[1]))
+        FAIL(h, MP_ERR_ARG, "invalid theta (sigma2, beta > 0)");
+    if (cov == MP_COV_MATERN && (!(th[2] > 0) || !(th[2] <= 20.0)))
+        FAIL(h, MP_ERR_ARG, "invalid theta (Matern: 0 < nu <= 20)");
+    return MP_OK;
+}
+
+mp_status mp_matrix_set_covariance(mp_matrix* A, mp_covariance kind) {
+    if (!A || (kind != MP_COV_MATERN && kind != MP_COV_SQEXP)) return MP_ERR_ARG;
+    A->cov = kind;
+    A->generated = A->factored = false;
     return MP_OK;
 }
 
@@ -547,8 +556,14 @@ static MaternArgs matern_args(const mp_matrix* A, const double* x, const double*
     a.sigma2 = th[0];
     a.beta = th[1];
     a.nu = th[2];
-    a.kind = th[2] == 0.5 ? 0 : th[2] == 1.5 ? 1 : th[2] == 2.5 ? 2 : 3;
-    a.coef = std::pow(2.0, 1.0 - th[2]) / std::tgamma(th[2]);
+    if (A->cov == MP_COV_SQEXP) {
+        a.kind = 4;
+        a.nu = 0.0;
+        a.coef = 0.0;
+    } else {
+        a.kind = th[2] == 0.5 ? 0 : th[2] == 1.5 ? 1 : th[2] == 2.5 ? 2 : 3;
+        a.coef = std::pow(2.0, 1.0 - th[2]) / std::tgamma(th[2]);
+    }
     return a;
 }
 
@@ -556,7 +571,7 @@ mp_status mp_matern_gen(mp_handle* h, mp_matrix* A, const double* d_x, const dou
                         const uint8_t* storage_prec, double* tile_sqnorm) {
     if (!h || !A || !d_x || !d_y) return MP_ERR_ARG;
     if (h->broken) FAIL(h, MP_ERR_STATE, "handle unusable after an earlier CUDA failure");
-    if (mp_status s = check_theta(h, theta)) return s;
+    if (mp_status s = check_theta(h, theta, A->cov)) return s;
     if (h->nranks > 1 && !A->comm.connected) FAIL(h, MP_ERR_COMM, "multi-rank matrix not connected");
     const int nt = A->nt;
     const MaternArgs a = matern_args(A, d_x, d_y, theta);
@@ -1267,7 +1282,7 @@ mp_status mp_eval(mp_handle* h, mp_matrix* A, const double* x, const double* y, 
                   const uint8_t* user_kernel_prec, mp_eval_report* rep) {
     if (!h || !A || !x || !y || !z || !rep) return MP_ERR_ARG;
     if (!A->bound) FAIL(h, MP_ERR_STATE, "bind a worst-case workspace (mp_matrix_bytes with NULL) first");
-    if (mp_status s = check_theta(h, theta)) return s;
+    if (mp_status s = check_theta(h, theta, A->cov)) return s;
     memset(rep, 0, sizeof *rep);
     const int nt = A->nt;
     const int64_t n = A->n;

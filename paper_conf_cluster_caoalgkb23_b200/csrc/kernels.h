@@ -41,7 +41,7 @@ struct MaternArgs {
     int64_t n;
     int nb;
     double sigma2, beta, nu;
-    int kind;     // 0: nu = 1/2, 1: nu = 3/2, 2: nu = 5/2, 3: general nu
+    int kind;     // 0: nu = 1/2, 1: nu = 3/2, 2: nu = 5/2, 3: general nu, 4: squared exponential
     double coef;  // 2^(1-nu) / Gamma(nu) for the general formula
 };
 constexpr int GEN_ROWS = 16;  // rows per CTA in the generation kernels

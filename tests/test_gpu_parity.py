@@ -233,3 +233,17 @@ def test_user_matrix_factor_matches_lapack(mp, handle):
     assert M.potrf(km, cm) == 0
     L = gpu_factor_dense(M, n)
     assert np.max(np.abs(L - np.linalg.cholesky(A))) <= 1e-12
+
+
+def test_sqexp_covariance_path(mp, handle):
+    """The paper's 2D squared exponential through the same path: tiles and l vs the oracle."""
+    n, nb, theta = 2500, 512, (1.0, 0.01, 0.0)
+    x, y = synth.locations(n, 3)
+    z = synth.normal_vector(n, 4)
+    ref = oracle_loglik(x, y, z, theta, nb, kernel="sqexp")
+    ev = mp.Evaluator(n, nb, handle=handle, covariance=mp.MP_COV_SQEXP)
+    r = ev.eval(x, y, z, theta, mode=mp.MP_MAP_FP64)
+    assert abs(r.loglik - ref["loglik"]) <= 1e-10 * abs(ref["loglik"])
+    g = ev.M.tile(2, 1)
+    t = ref["tiles"][2, 1]
+    assert np.max(np.abs(g[: t.shape[0], : t.shape[1]] - t)) <= 1e-15

@@ -60,3 +60,13 @@ def test_monotone_decreasing_in_distance():
 
 def test_distance_is_euclidean():
     assert distance(0.0, 0.0, 3.0, 4.0) == 5.0
+
+
+def test_sqexp_closed_form_and_limits():
+    """C(h) = sigma^2 exp(-h^2/beta); pinned against mpmath and its limits."""
+    from oracle.matern import sqexp
+    for h in [0.0, 1e-4, 0.01, 0.2, 0.9]:
+        ref = float(mpmath.mpf(1.7) * mpmath.exp(-(mpmath.mpf(h) ** 2) / mpmath.mpf(0.05)))
+        got = float(sqexp(np.array([h]), 1.7, 0.05)[0])
+        assert abs(got - ref) <= 4e-16 * (1 + h * h / 0.05) * ref
+    assert sqexp(np.array([0.0]), 2.0, 0.3)[0] == 2.0
