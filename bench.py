@@ -43,7 +43,8 @@ CONFIGS = {
     "c5": dict(n=250000, nb=2048, theta=(1.0, 0.03, 0.5), map="adaptive"),
 }
 METRIC = "Tflop/s & joules per MLE log-likelihood eval (n=360k) at 1/2/4/8 B200"
-FP64_NOMINAL, BF16_NOMINAL = 40.0, 2250.0  # TFLOP/s dense, B200 datasheet (ratio used for the FP64 peak)
+FP64_NOMINAL, BF16_NOMINAL, INT8_NOMINAL = 40.0, 2250.0, 4500.0  # dense TFLOP/s (TOP/s), B200 nominal
+OZ_PRODUCTS = 36  # int8 GEMMs per FP64 GEMM in the Ozaki split with S = 8 slices (S (S+1) / 2)
 
 
 def measured_peaks():
@@ -323,15 +324,18 @@ def main():
     peaks, peak_src = measured_peaks()
     p = prof.as_dict()
     dom = p["upd_fp64"]
+    engine = h.config()
     fp64_peak = peaks["bf16_tflops_sustained"] * FP64_NOMINAL / BF16_NOMINAL
-    achieved = dom["flops"] / (dom["ms"] / 1e3) / 1e12 if dom["ms"] > 0 else 0.0
+    int8_peak = peaks["bf16_tflops_sustained"] * INT8_NOMINAL / BF16_NOMINAL
+    fp64_eq = dom["flops"] / (dom["ms"] / 1e3) / 1e12 if dom["ms"] > 0 else 0.0
     try:
         cub = cublas_dgemm_tflops()
     except Exception:
         cub = None
     last = reps[-1]
     upd = list(last.flops_update)
-    roof_time_s = (upd[0] / (fp64_peak * 1e12)
+    fp64_class_peak = (int8_peak / OZ_PRODUCTS) if engine["ozaki"] else fp64_peak
+    roof_time_s = (upd[0] / (fp64_class_peak * 1e12)
                    + upd[1] / (peaks["bf16_tflops_sustained"] * 0.5 / 3 * 1e12)
                    + upd[2] / (peaks["bf16_tflops_sustained"] * 1e12))
     t_upd_s = (p["upd_fp64"]["ms"] + p["upd_fp32"]["ms"] + p["upd_fp16"]["ms"]) / 1e3 / args.steps
@@ -343,6 +347,8 @@ def main():
         "config": {"workload": f"{args.config}: n={n} ({int(math.isqrt(n))}^2 jittered grid, Morton order), nb={nb}, "
                                f"theta={list(theta)}, {cfg['map']} map u_req={args.u_req}, comm={args.policy}",
                    "n": n, "nb": nb, "map": cfg["map"], "policy": args.policy,
+                   "fp64_engine": "ozaki-int8 (S=8)" if engine["ozaki"] else "dmma",
+                   "fp32_fp16_engine": "tcgen05" if engine["tc"] else "dmma-rounded", "lookahead": engine["lookahead"],
                    "parallelism": (f"2D block-cyclic {P}x{Q}, peer-memory panel exchange" if distributed
                                    else ("replicas" if world > 1 else "1 GPU")),
                    "l2": "matrix (~%.0f GB) >> 126 MB L2; no flush needed" % (n * n / 2 * 5 / 1e9)},
@@ -354,11 +360,20 @@ def main():
                         "tflops": (v["flops"] / (v["ms"] / 1e3) / 1e12) if v["ms"] > 0 and v["flops"] else None}
                     for k, v in p.items()},
         "update_roofline_fraction": roof_time_s / t_upd_s if t_upd_s > 0 else None,
-        "roofline": {"bound": "tensor", "kernel": "dgemm_nt_kernel (FP64 DMMA trailing update)",
-                     "achieved": achieved, "peak": fp64_peak, "unit": "TFLOP/s",
-                     "frac": achieved / fp64_peak if fp64_peak else None, "traffic": None,
-                     "peak_source": f"{peak_src} bf16_tflops_sustained x {FP64_NOMINAL}/{BF16_NOMINAL} (FP64 DMMA nominal / bf16 nominal)",
-                     "cublas_dgemm_tflops_live": cub, "frac_vs_cublas_dgemm": (achieved / cub) if cub else None},
+        "roofline": (
+            {"bound": "tensor", "kernel": "ozaki_gemm_kernel<8> (FP64-class update as 36 INT8 tcgen05 GEMMs)",
+             "achieved": OZ_PRODUCTS * fp64_eq, "peak": int8_peak, "unit": "TFLOP/s",
+             "frac": OZ_PRODUCTS * fp64_eq / int8_peak, "traffic": None,
+             "peak_source": f"{peak_src} bf16_tflops_sustained x {INT8_NOMINAL}/{BF16_NOMINAL} (INT8 nominal / bf16 nominal); "
+                            "achieved = executed int8 multiply-add ops x 2 per second",
+             "fp64_equivalent_tflops": fp64_eq, "cublas_dgemm_tflops_live": cub,
+             "fp64_equivalent_vs_cublas_dgemm": (fp64_eq / cub) if cub else None}
+            if engine["ozaki"] else
+            {"bound": "tensor", "kernel": "dgemm_nt_kernel (FP64 DMMA trailing update)",
+             "achieved": fp64_eq, "peak": fp64_peak, "unit": "TFLOP/s",
+             "frac": fp64_eq / fp64_peak if fp64_peak else None, "traffic": None,
+             "peak_source": f"{peak_src} bf16_tflops_sustained x {FP64_NOMINAL}/{BF16_NOMINAL} (FP64 DMMA nominal / bf16 nominal)",
+             "cublas_dgemm_tflops_live": cub, "frac_vs_cublas_dgemm": (fp64_eq / cub) if cub else None}),
         "gpu_launches": launches,
         "clocks": ck,
         "e2e": e2e,

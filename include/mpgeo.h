@@ -257,6 +257,11 @@ typedef struct {
 mp_status mp_set_profiling(mp_handle* h, int enable);  /* enable also resets the counters */
 mp_status mp_get_profile(mp_handle* h, mp_profile* out);  /* synchronises the stream */
 
+/* Engine configuration of a handle (read from MPGEO_* at mp_init): tcgen05 kernels for the FP32
+ * and FP16 classes (1) or DMMA on rounded operands (0); panel lookahead (1/0); FP64-class
+ * engine: 8 = Ozaki split with 8 int8 slices on tcgen05 kind::i8, 0 = DMMA FP64. */
+mp_status mp_handle_config(const mp_handle* h, int* tc, int* lookahead, int* ozaki);
+
 /* Total kernels launched on this handle since mp_init (for bench accounting). */
 int64_t mp_launch_count(const mp_handle* h);
 

@@ -79,6 +79,11 @@ class Handle:
         self.check(lib.mp_get_profile(self.h, C.byref(p)))
         return p
 
+    def config(self) -> dict:
+        tc, la, oz = C.c_int(), C.c_int(), C.c_int()
+        self.check(lib.mp_handle_config(self.h, C.byref(tc), C.byref(la), C.byref(oz)))
+        return {"tc": tc.value, "lookahead": la.value, "ozaki": oz.value}
+
     @property
     def launches(self) -> int:
         return int(lib.mp_launch_count(self.h))

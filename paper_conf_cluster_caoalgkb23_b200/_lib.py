@@ -82,6 +82,7 @@ def _load() -> C.CDLL:
         "mp_matrix_nt": (i32, [vp]),
         "mp_matrix_owner": (i32, [vp, i32, i32]),
         "mp_launch_count": (i64, [vp]),
+        "mp_handle_config": (i32, [vp, C.POINTER(i32), C.POINTER(i32), C.POINTER(i32)]),
         "mp_set_profiling": (i32, [vp, i32]),
         "mp_get_profile": (i32, [vp, C.POINTER(Profile)]),
         "mp_version": (C.c_char_p, []),

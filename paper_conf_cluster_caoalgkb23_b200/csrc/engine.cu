@@ -49,7 +49,7 @@ struct mp_handle {
     bool broken = false;
     int tc_mode = 1;  // 1: tcgen05 kernels for FP32/FP16 classes when available, 0: DMMA emulation
     int lookahead = 1;  // 1: panel k+1 on the high-priority panel stream overlaps update k
-    int ozaki = 0;      // S in {7, 8}: FP64-class GEMM/SYRK emulated on INT8 tensor cores; 0: DMMA
+    int ozaki = 8;      // 8: FP64-class GEMM/SYRK emulated on INT8 tensor cores (S = 8 slices); 0: DMMA
     cudaStream_t pstream = nullptr;
     std::vector<cudaEvent_t> sync_ev;
     // profiling (mp_set_profiling): event pairs per launch, resolved in mp_get_profile
@@ -341,6 +341,14 @@ mp_status mp_get_profile(mp_handle* h, mp_profile* out) {
     return MP_OK;
 }
 int64_t mp_launch_count(const mp_handle* h) { return h ? h->launches : 0; }
+
+mp_status mp_handle_config(const mp_handle* h, int* tc, int* lookahead, int* ozaki) {
+    if (!h) return MP_ERR_ARG;
+    if (tc) *tc = (h->tc_mode != 0 && tc_gemm_available()) ? 1 : 0;
+    if (lookahead) *lookahead = h->lookahead;
+    if (ozaki) *ozaki = (h->ozaki == 8 && ozaki_available()) ? 8 : 0;
+    return MP_OK;
+}
 
 // ------------------------------------------------------------------ matrices
 mp_status mp_matrix_create(mp_handle* h, int64_t n, int nb, mp_matrix** A) {
@@ -658,7 +666,7 @@ static mp_status plan_potrf(mp_handle* h, mp_matrix* A, const uint8_t* km, const
     double* wb2 = A->at<double>(A->R.wbuf2);
     int* d_info = h->d_info;
     const bool use_tc = h->tc_mode != 0 && tc_gemm_available() && nb % 256 == 0;
-    const int ozS = (h->ozaki == 7 || h->ozaki == 8) && ozaki_available() && nb % 128 == 0 ? h->ozaki : 0;
+    const int ozS = h->ozaki == 8 && ozaki_available() && nb % 128 == 0 ? 8 : 0;
     int8_t* const ozb = A->at<int8_t>(A->R.oz);
     int* const ozeb = A->at<int>(A->R.ozexp);
     auto K = [&](int m, int k) { return km[(size_t)m * nt + k]; };

@@ -314,9 +314,8 @@ static cudaError_t oz_launch_s(const OzArgs& a, int njobs, cudaStream_t s) {
 cudaError_t ozaki_gemm_launch(const OzArgs& a, int njobs, cudaStream_t s) {
     if (njobs <= 0) return cudaSuccess;
     if (a.nb % OZ_BM || a.nb > 2048 * 4) return cudaErrorInvalidValue;
-    if (a.S == 7) return oz_launch_s<7>(a, njobs, s);
     if (a.S == 8) return oz_launch_s<8>(a, njobs, s);
-    return cudaErrorInvalidValue;
+    return cudaErrorInvalidValue;  // S = 8 is the only validated split (FP64-level accuracy)
 }
 
 bool ozaki_available() { return oz_encode() != nullptr; }

@@ -66,13 +66,12 @@ __device__ void smem_trtri_gj(double* S, double* wd, double* rowp, int n) {
             if (c < p) S[c * PLD + p] = rowp[c];
             else wd[p] = rowp[p];
         }
-        // rows i > p: W[i][c] -= L_ip * W[p][c], c <= p   (i fastest: conflict-free S[c][i])
-        const int rows = n - p - 1;
-        const int work = rows * (p + 1);
-        for (int w = tid; w < work; w += PT) {
-            const int c = w / rows, i = p + 1 + (w - c * rows);
+        // rows i > p: W[i][c] -= L_ip * W[p][c], c <= p; lanes run over i (conflict-free S[c][i]),
+        // warps over c, L_ip kept in a register
+        const int lane = tid & 31, wq = tid >> 5;
+        for (int i = p + 1 + lane; i < n; i += 32) {
             const double l = S[i * PLD + p];
-            if (c < i) S[c * PLD + i] = fma(-l, rowp[c], S[c * PLD + i]);
+            for (int c = wq; c <= p; c += PT / 32) S[c * PLD + i] = fma(-l, rowp[c], S[c * PLD + i]);
         }
         __syncthreads();
     }

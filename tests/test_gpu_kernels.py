@@ -125,7 +125,7 @@ def test_tc_gemm_tf32x3_matches_sgemm_accuracy(lib):
     assert err_tc < err_1x / 50  # far better than a single TF32 product
 
 
-@pytest.mark.parametrize("S", [7, 8])
+@pytest.mark.parametrize("S", [8])
 def test_ozaki_int8_fp64_gemm(lib, S):
     """FP64 GEMM emulated with int8 slices on tcgen05 kind::i8 vs the exact FP64 product: for S = 8
     the error stays within a few units of an FP64 GEMM's (|err| <= 8 K u max|a| max|b|)."""
@@ -140,7 +140,7 @@ def test_ozaki_int8_fp64_gemm(lib, S):
     ref = Cm - A @ B.T
     scale = np.abs(A).max(axis=1)[:, None] * np.abs(B).max(axis=1)[None, :]
     err = np.max(np.abs(got - ref) / scale)
-    bound = {8: 8 * nb * 2.0**-53, 7: 8 * nb * 2.0**-46}[S]
+    bound = 8 * nb * 2.0**-53
     assert err <= bound, (S, err, bound)
     # lower-only (SYRK) variant leaves strictly-upper 128x64 blocks untouched
     dC2 = dev(Cm)

@@ -1,5 +1,5 @@
-"""The whole path with the FP64 class on INT8 tensor cores (Ozaki split, S = 8)
-must still meet the all-FP64 tolerances: residual <= 1e-13 and l relative error <= 1e-10."""
+"""Both FP64-class engines — Ozaki split on INT8 tensor cores (default) and DMMA FP64
+(MPGEO_OZAKI=0) — must meet the all-FP64 tolerances: residual <= 1e-13, l relative error <= 1e-10."""
 import os
 
 import numpy as np
@@ -8,32 +8,33 @@ import pytest
 import synth
 from oracle.cholesky import residual
 from oracle.loglik import loglik as oracle_loglik
-from oracle.precision import all_fp64_maps, precision_maps
-from oracle.tiles import num_tiles, tile_sqnorms
+from oracle.precision import all_fp64_maps
+from oracle.tiles import num_tiles
 from tests.gpu_helpers import to_dev
 
 pytestmark = pytest.mark.gpu
 
 
-@pytest.fixture(scope="module")
-def oz_handle():
+@pytest.fixture(scope="module", params=["8", "0"], ids=["ozaki", "dmma"])
+def engine_handle(request):
     import paper_conf_cluster_caoalgkb23_b200 as mp
-    os.environ["MPGEO_OZAKI"] = "8"
+    os.environ["MPGEO_OZAKI"] = request.param
     try:
         h = mp.Handle(0)
     finally:
         del os.environ["MPGEO_OZAKI"]
+    assert h.config()["ozaki"] == int(request.param)
     return h
 
 
 @pytest.mark.parametrize("n,nb,theta", [(4900, 512, (1.0, 0.1, 0.5)), (8192, 1024, (1.0, 0.3, 0.5)),
                                          (3600, 512, (1.2, 0.05, 1.5))])
-def test_ozaki_fp64_path(oz_handle, n, nb, theta):
+def test_fp64_path_engines(engine_handle, n, nb, theta):
     import paper_conf_cluster_caoalgkb23_b200 as mp
     x, y = synth.locations(n, 0) if int(np.sqrt(n)) ** 2 == n else synth.uniform_locations(n, 0)
     z = synth.normal_vector(n, 1)
     nt = num_tiles(n, nb)
-    M = mp.Matrix(oz_handle, n, nb, None)
+    M = mp.Matrix(engine_handle, n, nb, None)
     dx, dy, dz = to_dev(x), to_dev(y), to_dev(z)
     km, sm, cm = all_fp64_maps(nt)
     M.matern_gen(dx, dy, theta, sm)
@@ -46,12 +47,12 @@ def test_ozaki_fp64_path(oz_handle, n, nb, theta):
     assert abs(ll - ref["loglik"]) <= 1e-10 * abs(ref["loglik"])
 
 
-def test_ozaki_mixed_precision_path(oz_handle):
+def test_mixed_precision_path_engines(engine_handle):
     import paper_conf_cluster_caoalgkb23_b200 as mp
     n, nb, theta = 10000, 512, (1.0, 0.03, 0.5)
     x, y = synth.locations(n, 0)
     z = synth.normal_vector(n, 1)
     ref = oracle_loglik(x, y, z, theta, nb)
-    ev = mp.Evaluator(n, nb, handle=oz_handle)
+    ev = mp.Evaluator(n, nb, handle=engine_handle)
     r = ev.eval(x, y, z, theta, u_req=1e-9)
     assert abs(r.loglik - ref["loglik"]) <= 1e-8 * abs(ref["loglik"])

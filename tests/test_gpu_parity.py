@@ -237,7 +237,7 @@ def test_user_matrix_factor_matches_lapack(mp, handle):
 
 def test_sqexp_covariance_path(mp, handle):
     """The paper's 2D squared exponential through the same path: tiles and l vs the oracle."""
-    n, nb, theta = 2500, 512, (1.0, 0.01, 0.0)
+    n, nb, theta = 1600, 512, (1.0, 0.0003, 0.0)
     x, y = synth.locations(n, 3)
     z = synth.normal_vector(n, 4)
     ref = oracle_loglik(x, y, z, theta, nb, kernel="sqexp")
