@@ -15,11 +15,14 @@
 // Epilogue: G_g -> FP64 (exact), scaled by 2^{-7g} (exact), summed smallest first, multiplied by
 // 2^{e_i + f_j} (exact), C -= result in FP64.
 //
-// CTA tile 128 x 64: 8 TMEM accumulators x 64 columns = all 512 TMEM columns.  K-major int8
+// CTA tile 128 x 64: 8 TMEM accumulators x 64 columns = all 512 TMEM columns; per k-step 12 MMAs of
+// N = 64..256 (A slice s against the concatenated B slices 1..S+1-s) instead of 36 of N = 64, which
+// cuts the shared-memory operand reads per MMA cycle by ~45%.  K-major int8
 // operands, 64-byte rows with the 64-byte TMA/UMMA swizzle; one 3D TMA box brings all S slices of
 // a 128 x 64 (A) or 64 x 64 (B) block; 2 stages of 96 KB.
 #include <cudaTypedefs.h>
 #include <stdint.h>
+#include <stdlib.h>
 #include <string.h>
 
 #include "common.cuh"
@@ -76,7 +79,7 @@ cudaError_t ozaki_split_launch(const OzSplitItem* items, int n, int nb, int S, c
 constexpr int OZ_BM = 128, OZ_BN = 64, OZ_BK = 64, OZ_THREADS = 256, OZ_STAGES = 2;
 
 struct __align__(64) OzParams {
-    CUtensorMap a, b;  // 3D [S][rows][nb] int8, boxes {64, 128, S} and {64, 64, S}
+    CUtensorMap a, b;  // 3D [S][rows][nb] int8, boxes {64, 128, S / CL} and {64, 64, S}
     const OzJob* jobs;
     const int* exps;   // row exponents of the slice cache rows [nt*nb]
     int nb, S, tiles_n, tiles_per_job, lower;
@@ -104,6 +107,26 @@ __device__ __forceinline__ void oz_tma3d(uint32_t dst, const CUtensorMap* map, u
         "l"((uint64_t)map), "r"(bar), "r"(c0), "r"(c1), "r"(c2)
         : "memory");
 }
+__device__ __forceinline__ void oz_tma3d_mc(uint32_t dst, const CUtensorMap* map, uint32_t bar, int c0, int c1, int c2,
+                                            uint16_t mask) {
+    asm volatile(
+        "cp.async.bulk.tensor.3d.shared::cluster.global.mbarrier::complete_tx::bytes.multicast::cluster [%0], [%1, {%3, %4, %5}], [%2], %6;" ::"r"(dst),
+        "l"((uint64_t)map), "r"(bar), "r"(c0), "r"(c1), "r"(c2), "h"(mask)
+        : "memory");
+}
+__device__ __forceinline__ void oz_commit_mc(uint32_t bar, uint16_t mask) {
+    asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.multicast::cluster.b64 [%0], %1;" ::"r"(bar),
+                 "h"(mask)
+                 : "memory");
+}
+__device__ __forceinline__ void oz_cluster_sync() {
+    asm volatile("barrier.cluster.arrive.release.aligned;\n\tbarrier.cluster.wait.acquire.aligned;" ::: "memory");
+}
+__device__ __forceinline__ uint32_t oz_cluster_rank() {
+    uint32_t r;
+    asm volatile("mov.u32 %0, %%cluster_ctarank;" : "=r"(r));
+    return r;
+}
 __device__ __forceinline__ void oz_fence_before() { asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory"); }
 __device__ __forceinline__ void oz_fence_after() { asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory"); }
 __device__ __forceinline__ void oz_commit(uint32_t bar) {
@@ -118,14 +141,15 @@ __device__ __forceinline__ uint64_t oz_desc(uint32_t saddr) {
     d |= (uint64_t)4 << 61;
     return d;
 }
-// instruction descriptor: D = S32 (2), A = B = signed int8 (1), K-major, N = 64, M = 128
-constexpr uint32_t OZ_IDESC = (2u << 4) | (1u << 7) | (1u << 10) | ((uint32_t)(OZ_BN >> 3) << 17) |
-                              ((uint32_t)(OZ_BM >> 4) << 24);
-__device__ __forceinline__ void oz_mma(uint32_t tmem, uint64_t a, uint64_t b, uint32_t accum) {
+// instruction descriptor: D = S32 (2), A = B = signed int8 (1), K-major, M = 128, N = n (16..256)
+__device__ __forceinline__ uint32_t oz_idesc(int n) {
+    return (2u << 4) | (1u << 7) | (1u << 10) | ((uint32_t)(n >> 3) << 17) | ((uint32_t)(OZ_BM >> 4) << 24);
+}
+__device__ __forceinline__ void oz_mma(uint32_t tmem, uint64_t a, uint64_t b, uint32_t idesc, uint32_t accum) {
     asm volatile(
         "{\n\t.reg .pred p;\n\tsetp.ne.b32 p, %4, 0;\n\t"
         "tcgen05.mma.cta_group::1.kind::i8 [%0], %1, %2, %3, p;\n\t}" ::"r"(tmem),
-        "l"(a), "l"(b), "r"(OZ_IDESC), "r"(accum));
+        "l"(a), "l"(b), "r"(idesc), "r"(accum));
 }
 __device__ __forceinline__ void oz_ld32(uint32_t taddr, uint32_t (&r)[32]) {
     asm volatile(
@@ -139,7 +163,10 @@ __device__ __forceinline__ void oz_ld32(uint32_t taddr, uint32_t (&r)[32]) {
     asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
 }
 
-template <int S>
+// CL = CTAs per cluster along N (1 or 2).  With CL = 2 the two CTAs compute neighbouring 64-column
+// blocks of the same 128 rows: each loads half of the A slice planes and multicasts them to both,
+// and every MMA commit releases the stage in both CTAs (a stage is refilled only when both consumed it).
+template <int S, int CL>
 __global__ void __launch_bounds__(OZ_THREADS, 1) ozaki_gemm_kernel(const __grid_constant__ OzParams p) {
     constexpr int A_SL = OZ_BM * OZ_BK;     // bytes of one A slice block (8 KB)
     constexpr int B_SL = OZ_BN * OZ_BK;     // 4 KB
@@ -155,7 +182,9 @@ __global__ void __launch_bounds__(OZ_THREADS, 1) ozaki_gemm_kernel(const __grid_
     const int job = blockIdx.x / p.tiles_per_job;
     const int t = blockIdx.x - job * p.tiles_per_job;
     const int bi = t / p.tiles_n, bj = t - bi * p.tiles_n;
-    if (p.lower && bj * OZ_BN > bi * OZ_BM + OZ_BM - 1) return;  // strictly upper block of a SYRK
+    // strictly upper block of a SYRK (with CL = 2 both CTAs of a cluster exit together: BM = 2 BN)
+    if (p.lower && (bj / CL) * CL * OZ_BN > bi * OZ_BM + OZ_BM - 1) return;
+    const uint32_t crank = CL > 1 ? oz_cluster_rank() : 0;
     const OzJob jb = p.jobs[job];
     const int rowA = jb.m * p.nb + bi * OZ_BM;
     const int rowB = jb.n * p.nb + bj * OZ_BN;
@@ -164,7 +193,7 @@ __global__ void __launch_bounds__(OZ_THREADS, 1) ozaki_gemm_kernel(const __grid_
     if (threadIdx.x == 0) {
         for (int s = 0; s < OZ_STAGES; ++s) {
             oz_mbar_init(oz_smem_u32(&full_bar[s]), 1);
-            oz_mbar_init(oz_smem_u32(&empty_bar[s]), 1);
+            oz_mbar_init(oz_smem_u32(&empty_bar[s]), CL);  // one MMA commit from every CTA of the cluster
         }
         oz_mbar_init(oz_smem_u32(&done_bar), 1);
         asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
@@ -181,6 +210,7 @@ __global__ void __launch_bounds__(OZ_THREADS, 1) ozaki_gemm_kernel(const __grid_
     }
     oz_fence_before();
     __syncthreads();
+    if (CL > 1) oz_cluster_sync();  // peers' barriers are initialised before any multicast arrives
     oz_fence_after();
     const uint32_t tmem = tmem_slot;
 
@@ -192,7 +222,12 @@ __global__ void __launch_bounds__(OZ_THREADS, 1) ozaki_gemm_kernel(const __grid_
             const uint32_t st = oz_smem_u32(smem + s * STAGE);
             const uint32_t fb = oz_smem_u32(&full_bar[s]);
             oz_expect_tx(fb, STAGE);
-            oz_tma3d(st, &p.a, fb, kb * OZ_BK, rowA, 0);
+            if (CL > 1) {
+                constexpr int PL = S / CL;  // A planes loaded (and multicast) by this CTA
+                oz_tma3d_mc(st + crank * PL * A_SL, &p.a, fb, kb * OZ_BK, rowA, (int)crank * PL, (uint16_t)((1u << CL) - 1));
+            } else {
+                oz_tma3d(st, &p.a, fb, kb * OZ_BK, rowA, 0);
+            }
             oz_tma3d(st + S * A_SL, &p.b, fb, kb * OZ_BK, rowB, 0);
         }
     } else if (warp == 1 && lane == 0) {
@@ -205,20 +240,26 @@ __global__ void __launch_bounds__(OZ_THREADS, 1) ozaki_gemm_kernel(const __grid_
 #pragma unroll
             for (int k = 0; k < OZ_BK / 32; ++k) {
                 const uint32_t koff = k * 32;
+                // For A slice s, the B slices t = 1 .. S+1-s are contiguous in shared memory: ONE MMA
+                // with N = 64 (S+1-s) (split at N = 256) writes product (s, t) into TMEM columns
+                // (s-1+t-1)*64 = (g-2)*64, exactly group g = s+t's accumulator.  The s = 1 MMAs
+                // cover all 8 groups and initialise them (accumulate = 0) on the first k-step.
 #pragma unroll
-                for (int g = 2; g <= S + 1; ++g) {
+                for (int sa = 1; sa <= S; ++sa) {
+                    const int nt_total = S + 1 - sa;  // number of B slices paired with sa
+                    const uint64_t da = oz_desc(base + (sa - 1) * A_SL + koff);
 #pragma unroll
-                    for (int sa = 1; sa < g; ++sa) {
-                        const int sb = g - sa;
-                        if (sa > S || sb > S) continue;
-                        const uint64_t da = oz_desc(base + (sa - 1) * A_SL + koff);
-                        const uint64_t db = oz_desc(base + S * A_SL + (sb - 1) * B_SL + koff);
-                        const uint32_t acc = (kb | k) != 0 || sa != (g - 1 > S ? g - S : 1);
-                        oz_mma(tmem + (uint32_t)(g - 2) * OZ_BN, da, db, acc);
+                    for (int t0 = 0; t0 < nt_total; t0 += 4) {  // <= 4 slices x 64 = 256 columns per MMA
+                        const int cnt = nt_total - t0 < 4 ? nt_total - t0 : 4;
+                        const uint64_t db = oz_desc(base + S * A_SL + t0 * B_SL + koff);
+                        const uint32_t col = (uint32_t)(sa - 1 + t0) * OZ_BN;
+                        const uint32_t acc = (kb | k) != 0 || sa != 1;
+                        oz_mma(tmem + col, da, db, oz_idesc(cnt * OZ_BN), acc);
                     }
                 }
             }
-            oz_commit(oz_smem_u32(&empty_bar[s]));
+            if (CL > 1) oz_commit_mc(oz_smem_u32(&empty_bar[s]), (uint16_t)((1u << CL) - 1));
+            else oz_commit(oz_smem_u32(&empty_bar[s]));
         }
         oz_commit(oz_smem_u32(&done_bar));
     } else if (warp >= 4) {
@@ -253,6 +294,7 @@ __global__ void __launch_bounds__(OZ_THREADS, 1) ozaki_gemm_kernel(const __grid_
     }
     oz_fence_before();
     __syncthreads();
+    if (CL > 1) oz_cluster_sync();  // no CTA leaves while its peer may still signal or fill it
     if (warp == 2) {
         oz_fence_after();
         asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem), "r"(512) : "memory");
@@ -284,19 +326,19 @@ static bool oz_map(CUtensorMap* m, const int8_t* base, uint64_t planes, uint64_t
               CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
 }
 
-template <int S>
+template <int S, int CL>
 static cudaError_t oz_launch_s(const OzArgs& a, int njobs, cudaStream_t s) {
     constexpr int SMEM = OZ_STAGES * S * (OZ_BM + OZ_BN) * OZ_BK + 1024;
     static bool attr = false;
     if (!attr) {
-        cudaError_t e = cudaFuncSetAttribute(ozaki_gemm_kernel<S>, cudaFuncAttributeMaxDynamicSharedMemorySize, SMEM);
+        cudaError_t e = cudaFuncSetAttribute(ozaki_gemm_kernel<S, CL>, cudaFuncAttributeMaxDynamicSharedMemorySize, SMEM);
         if (e != cudaSuccess) return e;
         attr = true;
     }
     OzParams p;
     memset(&p, 0, sizeof p);
     const uint64_t rows = (uint64_t)a.nt * a.nb;
-    if (!oz_map(&p.a, a.slices, S, rows, a.nb, a.plane_stride, OZ_BM, S) ||
+    if (!oz_map(&p.a, a.slices, S, rows, a.nb, a.plane_stride, OZ_BM, S / CL) ||
         !oz_map(&p.b, a.slices, S, rows, a.nb, a.plane_stride, OZ_BN, S))
         return cudaErrorInvalidValue;
     p.jobs = a.jobs;
@@ -307,14 +349,29 @@ static cudaError_t oz_launch_s(const OzArgs& a, int njobs, cudaStream_t s) {
     p.tiles_per_job = (a.nb / OZ_BM) * p.tiles_n;
     p.lower = a.lower;
     const long long grid = (long long)njobs * p.tiles_per_job;
-    ozaki_gemm_kernel<S><<<(unsigned)grid, OZ_THREADS, SMEM, s>>>(p);
-    return cudaGetLastError();
+    cudaLaunchConfig_t cfg = {};
+    cfg.gridDim = dim3((unsigned)grid);
+    cfg.blockDim = dim3(OZ_THREADS);
+    cfg.dynamicSmemBytes = SMEM;
+    cfg.stream = s;
+    cudaLaunchAttribute at[1];
+    at[0].id = cudaLaunchAttributeClusterDimension;
+    at[0].val.clusterDim.x = CL;
+    at[0].val.clusterDim.y = 1;
+    at[0].val.clusterDim.z = 1;
+    cfg.attrs = at;
+    cfg.numAttrs = 1;
+    return cudaLaunchKernelEx(&cfg, ozaki_gemm_kernel<S, CL>, p);
 }
 
 cudaError_t ozaki_gemm_launch(const OzArgs& a, int njobs, cudaStream_t s) {
     if (njobs <= 0) return cudaSuccess;
     if (a.nb % OZ_BM || a.nb > 2048 * 4) return cudaErrorInvalidValue;
-    if (a.S == 8) return oz_launch_s<8>(a, njobs, s);
+    static const int cl = [] {
+        const char* e = getenv("MPGEO_OZAKI_CLUSTER");
+        return e ? atoi(e) : 2;
+    }();
+    if (a.S == 8) return cl == 2 ? oz_launch_s<8, 2>(a, njobs, s) : oz_launch_s<8, 1>(a, njobs, s);
     return cudaErrorInvalidValue;  // S = 8 is the only validated split (FP64-level accuracy)
 }
 

@@ -40,6 +40,12 @@ def main(which):
         for _ in range(3):
             assert lib.mp_test_tc_gemm(2, p(P16), None, p(Cf), nb, nt, 1, 0) == 0
             assert lib.mp_test_tc_gemm(1, p(hi), p(lo), p(Cf), nb, nt, 1, 0) == 0
+    if which in ("ozaki", "all"):
+        nb, nt = 2048, 4
+        P = torch.randn(nt * nb, nb, dtype=torch.float64, device="cuda")
+        Cm = torch.zeros(nb, nb, dtype=torch.float64, device="cuda")
+        for _ in range(3):
+            assert lib.mp_test_ozaki_gemm(p(P), p(Cm), nb, nt, 2, 1, 8, 0) == 0
     if which in ("tf32err", "all"):
         from tests.test_gpu_kernels import tf32_rna
         for K in (64, 256, 1024, 2048):
