@@ -241,9 +241,13 @@ def test_sqexp_covariance_path(mp, handle):
     x, y = synth.locations(n, 3)
     z = synth.normal_vector(n, 4)
     ref = oracle_loglik(x, y, z, theta, nb, kernel="sqexp")
+    M = mp.Matrix(handle, n, nb, None)
+    M.set_covariance(mp.MP_COV_SQEXP)
+    M.matern_gen(to_dev(x), to_dev(y), theta, np.zeros((M.nt, M.nt), np.uint8))
+    for key in [(2, 1), (3, 3), (3, 0)]:
+        g = M.tile(*key)
+        t = ref["tiles"][key]
+        assert np.max(np.abs(g[: t.shape[0], : t.shape[1]] - t)) <= 1e-15
     ev = mp.Evaluator(n, nb, handle=handle, covariance=mp.MP_COV_SQEXP)
     r = ev.eval(x, y, z, theta, mode=mp.MP_MAP_FP64)
     assert abs(r.loglik - ref["loglik"]) <= 1e-10 * abs(ref["loglik"])
-    g = ev.M.tile(2, 1)
-    t = ref["tiles"][2, 1]
-    assert np.max(np.abs(g[: t.shape[0], : t.shape[1]] - t)) <= 1e-15
