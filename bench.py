@@ -334,9 +334,10 @@ def main():
         cub = None
     last = reps[-1]
     upd = list(last.flops_update)
-    fp64_class_peak = (int8_peak / OZ_PRODUCTS) if engine["ozaki"] else fp64_peak
+    fp64_class_peak = (int8_peak / OZ_PRODUCTS) if engine["ozaki"] % 100 == 8 else fp64_peak
+    fp32_class_peak = (int8_peak / 10) if engine["ozaki"] >= 100 else peaks["bf16_tflops_sustained"] * 0.5 / 3
     roof_time_s = (upd[0] / (fp64_class_peak * 1e12)
-                   + upd[1] / (peaks["bf16_tflops_sustained"] * 0.5 / 3 * 1e12)
+                   + upd[1] / (fp32_class_peak * 1e12)
                    + upd[2] / (peaks["bf16_tflops_sustained"] * 1e12))
     t_upd_s = (p["upd_fp64"]["ms"] + p["upd_fp32"]["ms"] + p["upd_fp16"]["ms"]) / 1e3 / args.steps
     out = {
@@ -347,8 +348,10 @@ def main():
         "config": {"workload": f"{args.config}: n={n} ({int(math.isqrt(n))}^2 jittered grid, Morton order), nb={nb}, "
                                f"theta={list(theta)}, {cfg['map']} map u_req={args.u_req}, comm={args.policy}",
                    "n": n, "nb": nb, "map": cfg["map"], "policy": args.policy,
-                   "fp64_engine": "ozaki-int8 (S=8)" if engine["ozaki"] else "dmma",
-                   "fp32_fp16_engine": "tcgen05" if engine["tc"] else "dmma-rounded", "lookahead": engine["lookahead"],
+                   "fp64_engine": "ozaki-int8 (S=8)" if engine["ozaki"] % 100 == 8 else "dmma",
+                   "fp32_engine": ("ozaki-int8 (S=4)" if engine["ozaki"] >= 100 else
+                                   ("tcgen05 3xTF32" if engine["tc"] else "dmma-rounded")),
+                   "fp16_engine": "tcgen05 f16" if engine["tc"] else "dmma-rounded", "lookahead": engine["lookahead"],
                    "parallelism": (f"2D block-cyclic {P}x{Q}, peer-memory panel exchange" if distributed
                                    else ("replicas" if world > 1 else "1 GPU")),
                    "l2": "matrix (~%.0f GB) >> 126 MB L2; no flush needed" % (n * n / 2 * 5 / 1e9)},
@@ -368,7 +371,7 @@ def main():
                             "achieved = executed int8 multiply-add ops x 2 per second",
              "fp64_equivalent_tflops": fp64_eq, "cublas_dgemm_tflops_live": cub,
              "fp64_equivalent_vs_cublas_dgemm": (fp64_eq / cub) if cub else None}
-            if engine["ozaki"] else
+            if engine["ozaki"] % 100 == 8 else
             {"bound": "tensor", "kernel": "dgemm_nt_kernel (FP64 DMMA trailing update)",
              "achieved": fp64_eq, "peak": fp64_peak, "unit": "TFLOP/s",
              "frac": fp64_eq / fp64_peak if fp64_peak else None, "traffic": None,

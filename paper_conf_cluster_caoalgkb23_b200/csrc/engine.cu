@@ -50,6 +50,7 @@ struct mp_handle {
     int tc_mode = 1;  // 1: tcgen05 kernels for FP32/FP16 classes when available, 0: DMMA emulation
     int lookahead = 1;  // 1: panel k+1 on the high-priority panel stream overlaps update k
     int ozaki = 8;      // 8: FP64-class GEMM/SYRK emulated on INT8 tensor cores (S = 8 slices); 0: DMMA
+    int ozaki32 = 1;    // 1: FP32-class GEMM on INT8 tensor cores (first 4 slices); 0: 3xTF32 tcgen05
     cudaStream_t pstream = nullptr;
     std::vector<cudaEvent_t> sync_ev;
     // profiling (mp_set_profiling): event pairs per launch, resolved in mp_get_profile
@@ -62,7 +63,8 @@ struct mp_handle {
 
 struct Regions {
     size_t total = 0;
-    size_t inputs = 0, p64 = 0, p16 = 0, phi = 0, plo = 0, ltilde = 0, wbuf = 0, wbuf2 = 0, oz = 0, ozexp = 0;
+    size_t inputs = 0, p64 = 0, p16 = 0, phi = 0, plo = 0, ltilde = 0, wbuf = 0, wbuf2 = 0, oz = 0, ozexp = 0,
+           wdiag = 0;
     size_t vec_r = 0, vec_y = 0, partials = 0, norms = 0, ctrl = 0, ctrl_bytes = 0;
     std::vector<size_t> tile_off;  // per (m*nt+k), SIZE_MAX if not stored here
 };
@@ -159,6 +161,7 @@ static Regions layout(const mp_matrix* A, const uint8_t* storage) {
     R.ltilde = take(nb2 * 8);
     R.wbuf = take((size_t)POTRF_IB * POTRF_IB * 8);
     R.wbuf2 = take((size_t)ceil_div(A->nb, POTRF_IB) * POTRF_IB * POTRF_IB * 8);
+    R.wdiag = take((size_t)nt * ceil_div(A->nb, POTRF_IB) * POTRF_IB * POTRF_IB * 8);  // solve: block inverses
     // two sets of panel buffers (panel parity) so panel k+1 can be produced while update k reads panel k
     R.p64 = take(2 * (size_t)nt * nb2 * 8);
     R.p16 = take(2 * (size_t)nt * nb2 * 2);
@@ -201,6 +204,7 @@ struct Op {
     int stream = 0;  // 0: the handle's stream, 1: the high-priority panel stream (lookahead)
     int kind = 0;    // 0: launch, 1: record event `ev` on `stream`, 2: make `stream` wait for `ev`
     int ev = -1;
+    int nlaunch = 1;  // kernels this op launches (for the launch count)
 };
 static Op op_record(int stream, int ev) { Op o{nullptr, 0, 0}; o.stream = stream; o.kind = 1; o.ev = ev; return o; }
 static Op op_wait(int stream, int ev) { Op o{nullptr, 0, 0}; o.stream = stream; o.kind = 2; o.ev = ev; return o; }
@@ -246,7 +250,7 @@ static mp_status run_plan(mp_handle* h, mp_matrix* A, Arena& ar, std::vector<Op>
         } else {
             CK(h, op.fn(st));
         }
-        h->launches++;
+        h->launches += op.nlaunch;
     }
     return MP_OK;
 }
@@ -269,6 +273,7 @@ mp_status mp_init(int device, int rank, int nranks, int P, int Q, const uint8_t*
     if (const char* e = getenv("MPGEO_TC")) h->tc_mode = atoi(e);
     if (const char* e = getenv("MPGEO_LOOKAHEAD")) h->lookahead = atoi(e);
     if (const char* e = getenv("MPGEO_OZAKI")) h->ozaki = atoi(e);
+    if (const char* e = getenv("MPGEO_OZAKI32")) h->ozaki32 = atoi(e);
     auto fail = [&](mp_status s) {
         if (h->own_stream && h->stream) cudaStreamDestroy(h->stream);
         delete h;
@@ -344,9 +349,10 @@ int64_t mp_launch_count(const mp_handle* h) { return h ? h->launches : 0; }
 
 mp_status mp_handle_config(const mp_handle* h, int* tc, int* lookahead, int* ozaki) {
     if (!h) return MP_ERR_ARG;
+    // ozaki: 0 = DMMA FP64 class; 8 = INT8 FP64 class; +100 if the FP32 class also runs on INT8
     if (tc) *tc = (h->tc_mode != 0 && tc_gemm_available()) ? 1 : 0;
     if (lookahead) *lookahead = h->lookahead;
-    if (ozaki) *ozaki = (h->ozaki == 8 && ozaki_available()) ? 8 : 0;
+    if (ozaki) *ozaki = (h->ozaki == 8 && ozaki_available()) ? (8 + (h->ozaki32 ? 100 : 0)) : 0;
     return MP_OK;
 }
 
@@ -667,6 +673,7 @@ static mp_status plan_potrf(mp_handle* h, mp_matrix* A, const uint8_t* km, const
     int* d_info = h->d_info;
     const bool use_tc = h->tc_mode != 0 && tc_gemm_available() && nb % 256 == 0;
     const int ozS = h->ozaki == 8 && ozaki_available() && nb % 128 == 0 ? 8 : 0;
+    const bool oz32 = ozS && h->ozaki32 && nb % 256 == 0;
     int8_t* const ozb = A->at<int8_t>(A->R.oz);
     int* const ozeb = A->at<int>(A->R.ozexp);
     auto K = [&](int m, int k) { return km[(size_t)m * nt + k]; };
@@ -842,7 +849,7 @@ static mp_status plan_potrf(mp_handle* h, mp_matrix* A, const uint8_t* km, const
             local_formats(k, m, need16, need32);
             if (use_tc) {
                 if (need16) t.p16 = p16 + (size_t)m * nb2;
-                if (need32) {
+                if (need32 && !oz32) {
                     t.hi = phi + (size_t)m * nb2;
                     t.lo = plo + (size_t)m * nb2;
                 }
@@ -912,7 +919,7 @@ static mp_status plan_potrf(mp_handle* h, mp_matrix* A, const uint8_t* km, const
                 PullItem it{sendslot(o, sp, m), pubflag(o, sp, m), ST(k), p64 + (size_t)m * nb2, nullptr, nullptr,
                             nullptr, C(m, k), 0};
                 if (use_tc && n16) it.p16 = p16 + (size_t)m * nb2;
-                if (use_tc && n32) {
+                if (use_tc && n32 && !oz32) {
                     it.hi = phi + (size_t)m * nb2;
                     it.lo = plo + (size_t)m * nb2;
                 }
@@ -934,8 +941,9 @@ static mp_status plan_potrf(mp_handle* h, mp_matrix* A, const uint8_t* km, const
             std::vector<OzSplitItem> sp;
             for (int m = k + 1; m < nt; ++m) {
                 bool need = A->mine(m, m);
-                for (int n = k + 1; n < m && !need; ++n) need |= A->mine(m, n) && K(m, n) == MP_FP64;
-                for (int n = m + 1; n < nt && !need; ++n) need |= A->mine(n, m) && K(n, m) == MP_FP64;
+                auto int8_class = [&](int p) { return p == MP_FP64 || (oz32 && p == MP_FP32); };
+                for (int n = k + 1; n < m && !need; ++n) need |= A->mine(m, n) && int8_class(K(m, n));
+                for (int n = m + 1; n < nt && !need; ++n) need |= A->mine(n, m) && int8_class(K(n, m));
                 if (need)
                     sp.push_back(OzSplitItem{p64 + (size_t)m * nb2, ozs + (size_t)m * nb2, oze + (size_t)m * nb, ozplane});
             }
@@ -951,6 +959,7 @@ static mp_status plan_potrf(mp_handle* h, mp_matrix* A, const uint8_t* km, const
         cur = part == 0 ? &nxt[k] : &rst[k];
         std::vector<GemmJob> syrk, g64, g32, g16;
         std::vector<TcJob> t32, t16;
+        std::vector<OzJob> o32;
         for (int m = k + 1; m < nt; ++m) {
             if (A->mine(m, m) && ((m == k + 1) == (part == 0))) {
                 syrk.push_back(GemmJob{p64 + (size_t)m * nb2, p64 + (size_t)m * nb2, A->tile(m, m)});
@@ -962,6 +971,8 @@ static mp_status plan_potrf(mp_handle* h, mp_matrix* A, const uint8_t* km, const
                 fc.upd[p] += 2.0 * fnb * fnb * fnb;
                 if (p == MP_FP64) {
                     g64.push_back(GemmJob{p64 + (size_t)m * nb2, p64 + (size_t)n * nb2, A->tile(m, n)});
+                } else if (oz32 && p == MP_FP32) {
+                    o32.push_back(OzJob{m, n, A->tile(m, n)});
                 } else if (use_tc) {
                     (p == MP_FP32 ? t32 : t16).push_back(TcJob{m, n, (float*)A->tile(m, n)});
                 } else {
@@ -981,7 +992,7 @@ static mp_status plan_potrf(mp_handle* h, mp_matrix* A, const uint8_t* km, const
                 if (oj.empty()) continue;
                 OzJob* dj = ar.push(oj);
                 const int nj = (int)oj.size();
-                OzArgs oa{dj, ozs, oze, ozplane, nb, nt, ozS, lower};
+                OzArgs oa{dj, ozs, oze, ozplane, nb, nt, ozS, lower, 0};
                 cur_push(Op{[=](cudaStream_t s) { return ozaki_gemm_launch(oa, nj, s); }, C_UPD64,
                             (lower ? f3 : 2 * f3) * nj});
             }
@@ -992,6 +1003,12 @@ static mp_status plan_potrf(mp_handle* h, mp_matrix* A, const uint8_t* km, const
         gemm(g64, nb, nb, nb, nb, nb, nb, 0, -1.0, 1.0, P64, false, C_UPD64, 2 * f3);
         gemm(g32, nb, nb, nb, nb, nb, nb, 0, -1.0, 1.0, P32, true, C_UPD32, 2 * f3);
         gemm(g16, nb, nb, nb, nb, nb, nb, 0, -1.0, 1.0, P16, true, C_UPD16, 2 * f3);
+        if (!o32.empty()) {  // FP32 class on INT8 tensor cores: 4 slices, FP32 C tiles
+            OzJob* dj = ar.push(o32);
+            const int nj = (int)o32.size();
+            OzArgs oa{dj, ozs, oze, ozplane, nb, nt, 4, 0, 1};
+            cur_push(Op{[=](cudaStream_t s) { return ozaki_gemm_launch(oa, nj, s); }, C_UPD32, 2 * f3 * nj});
+        }
         if (!t32.empty()) {
             TcJob* dj = ar.push(t32);
             const int nj = (int)t32.size();
@@ -1236,13 +1253,23 @@ mp_status mp_loglik(mp_handle* h, const mp_matrix* Lc, const double* d_z, double
     std::vector<Op> ops;
     std::vector<const double*> diag;
     std::vector<int> nreal;
+    for (int k = 0; k < nt; ++k) diag.push_back((const double*)A->tile(k, k));
+    // 128-block inverses of every diagonal tile in one launch, then a blocked TRSV per tile
+    double* wdiag = A->at<double>(A->R.wdiag);
+    const size_t wstride = (size_t)ceil_div(nb, POTRF_IB) * POTRF_IB * POTRF_IB;
+    {
+        const double* const* d_all = ar.push(diag);
+        ops.push_back({[=](cudaStream_t s) { return trtri_batch_launch(d_all, nt, nb, wdiag, s); }, C_SOLVE, 0});
+    }
     for (int k = 0; k < nt; ++k) {
-        const double* Lkk = (const double*)A->tile(k, k);
-        diag.push_back(Lkk);
+        const double* Lkk = diag[k];
         nreal.push_back((int)std::min<int64_t>(nb, n - (int64_t)k * nb));
         double* rk = r + (size_t)k * nb;
         double* yk = y + (size_t)k * nb;
-        ops.push_back({[=](cudaStream_t s) { return trsv_tile_launch(Lkk, nb, rk, yk, s); }, C_SOLVE, 0});
+        const double* Wk = wdiag + (size_t)k * wstride;
+        Op op{[=](cudaStream_t s) { return trsv_blocked_launch(Lkk, nb, Wk, rk, yk, s); }, C_SOLVE, 0};
+        op.nlaunch = 2 * ceil_div(nb, POTRF_IB) - 1;
+        ops.push_back(std::move(op));
         std::vector<GemvTile> gv;
         for (int m = k + 1; m < nt; ++m) gv.push_back(GemvTile{A->tile(m, k), A->st(m, k), 0, r + (size_t)m * nb});
         if (!gv.empty()) {

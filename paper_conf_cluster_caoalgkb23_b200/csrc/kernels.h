@@ -27,6 +27,8 @@ cudaError_t potrf_diag_block_launch(double* A, int lda, int jb, double* W, int c
                                     cudaStream_t s);
 // For each diagonal block b of the nb x nb lower matrix L (ld nb): W_b = inv(L_bb).
 cudaError_t trtri_blocks_launch(const double* L, int nb, double* W, cudaStream_t s);
+// Batched over tiles: W[t][b] = inv(L_t,bb) for every 128-block b of every tile t
+cudaError_t trtri_batch_launch(const double* const* Ls, int ntiles, int nb, double* W, cudaStream_t s);
 
 // ---- K1: Matérn generation (matern.cu)
 struct GenTile {
@@ -78,6 +80,9 @@ cudaError_t zero_upper_launch(double* A, int nb, cudaStream_t s);
 // ---- K8: solve and reductions (solve.cu)
 // y[0..nb) = L^{-1} r[0..nb) for one FP64 lower tile (ld nb), rows >= nreal are identity pads
 cudaError_t trsv_tile_launch(const double* L, int nb, const double* r, double* y, cudaStream_t s);
+// Blocked TRSV of one FP64 lower tile with its block inverses Wk ([block][128][128]): y = L^{-1} r
+// (r is overwritten with intermediate values)
+cudaError_t trsv_blocked_launch(const double* L, int nb, const double* Wk, double* r, double* y, cudaStream_t s);
 struct GemvTile {
     const void* L;    // tile (m, k), storage precision, nb x nb
     int prec;

@@ -76,13 +76,21 @@ cudaError_t ozaki_split_launch(const OzSplitItem* items, int n, int nb, int S, c
 }
 
 // ------------------------------------------------------------------ GEMM
-constexpr int OZ_BM = 128, OZ_BN = 64, OZ_BK = 64, OZ_THREADS = 256, OZ_STAGES = 2;
+constexpr int OZ_BM = 128, OZ_BK = 64, OZ_THREADS = 256, OZ_STAGES = 2;
 
 struct __align__(64) OzParams {
     CUtensorMap a, b;  // 3D [S][rows][nb] int8, boxes {64, 128, S / CL} and {64, 64, S}
     const OzJob* jobs;
     const int* exps;   // row exponents of the slice cache rows [nt*nb]
     int nb, S, tiles_n, tiles_per_job, lower;
+};
+
+// S slices -> S TMEM accumulators of BN columns (S * BN = 512): S = 8 (FP64 class) uses 128 x 64
+// tiles, S = 4 (FP32 class: the first 4 planes of the same split, 28 bits) uses 128 x 128 tiles.
+template <int S>
+struct OzCfg {
+    static constexpr int BN = 512 / S;
+    static constexpr int PER_MMA = 256 / BN;  // B slices concatenated per MMA (N <= 256)
 };
 
 __device__ __forceinline__ uint32_t oz_smem_u32(const void* p) { return (uint32_t)__cvta_generic_to_shared(p); }
@@ -166,17 +174,18 @@ __device__ __forceinline__ void oz_ld32(uint32_t taddr, uint32_t (&r)[32]) {
 // CL = CTAs per cluster along N (1 or 2).  With CL = 2 the two CTAs compute neighbouring 64-column
 // blocks of the same 128 rows: each loads half of the A slice planes and multicasts them to both,
 // and every MMA commit releases the stage in both CTAs (a stage is refilled only when both consumed it).
-template <int S, int CL>
+template <int S, int CL, bool CF32>
 __global__ void __launch_bounds__(OZ_THREADS, 1) ozaki_gemm_kernel(const __grid_constant__ OzParams p) {
+    constexpr int OZ_BN = OzCfg<S>::BN;
     constexpr int A_SL = OZ_BM * OZ_BK;     // bytes of one A slice block (8 KB)
-    constexpr int B_SL = OZ_BN * OZ_BK;     // 4 KB
+    constexpr int B_SL = OZ_BN * OZ_BK;     // 4 KB (BN = 64) or 8 KB (BN = 128)
     constexpr int STAGE = S * (A_SL + B_SL);
     constexpr int NG = S;                   // groups g = 2 .. S+1
     extern __shared__ uint8_t oz_smem_raw[];
     uint8_t* smem = (uint8_t*)(((uintptr_t)oz_smem_raw + 1023) & ~(uintptr_t)1023);
     __shared__ __align__(8) uint64_t full_bar[OZ_STAGES], empty_bar[OZ_STAGES], done_bar;
     __shared__ uint32_t tmem_slot;
-    __shared__ double colscale[OZ_BN];
+    __shared__ double colscale[128];
 
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     const int job = blockIdx.x / p.tiles_per_job;
@@ -249,8 +258,8 @@ __global__ void __launch_bounds__(OZ_THREADS, 1) ozaki_gemm_kernel(const __grid_
                     const int nt_total = S + 1 - sa;  // number of B slices paired with sa
                     const uint64_t da = oz_desc(base + (sa - 1) * A_SL + koff);
 #pragma unroll
-                    for (int t0 = 0; t0 < nt_total; t0 += 4) {  // <= 4 slices x 64 = 256 columns per MMA
-                        const int cnt = nt_total - t0 < 4 ? nt_total - t0 : 4;
+                    for (int t0 = 0; t0 < nt_total; t0 += OzCfg<S>::PER_MMA) {  // N <= 256 per MMA
+                        const int cnt = nt_total - t0 < OzCfg<S>::PER_MMA ? nt_total - t0 : OzCfg<S>::PER_MMA;
                         const uint64_t db = oz_desc(base + S * A_SL + t0 * B_SL + koff);
                         const uint32_t col = (uint32_t)(sa - 1 + t0) * OZ_BN;
                         const uint32_t acc = (kb | k) != 0 || sa != 1;
@@ -268,28 +277,41 @@ __global__ void __launch_bounds__(OZ_THREADS, 1) ozaki_gemm_kernel(const __grid_
         const int q = warp - 4;
         const int row = bi * OZ_BM + q * 32 + lane;
         const uint32_t tl = (uint32_t)(q * 32) << 16;
-        double acc[OZ_BN];
-#pragma unroll
-        for (int j = 0; j < OZ_BN; ++j) acc[j] = 0.0;
+        const double rs = ldexp(1.0, p.exps[rowA + q * 32 + lane]);
 #pragma unroll 1
-        for (int g = S + 1; g >= 2; --g) {  // smallest terms first
-            const double sc = ldexp(1.0, -7 * g);
+        for (int c0 = 0; c0 < OZ_BN; c0 += 32) {  // 32-column chunks: all groups, then C update
+            double acc[32];
 #pragma unroll
-            for (int c0 = 0; c0 < OZ_BN; c0 += 32) {
+            for (int j = 0; j < 32; ++j) acc[j] = 0.0;
+#pragma unroll 1
+            for (int g = S + 1; g >= 2; --g) {  // smallest terms first
+                const double sc = ldexp(1.0, -7 * g);
                 uint32_t r[32];
                 oz_ld32(tmem + tl + (uint32_t)((g - 2) * OZ_BN + c0), r);
 #pragma unroll
-                for (int v = 0; v < 32; ++v) acc[c0 + v] = fma((double)(int)r[v], sc, acc[c0 + v]);
+                for (int v = 0; v < 32; ++v) acc[v] = fma((double)(int)r[v], sc, acc[v]);
             }
-        }
-        const double rs = ldexp(1.0, p.exps[rowA + q * 32 + lane]);
-        double* crow = (double*)jb.C + (size_t)row * p.nb + bj * OZ_BN;
+            if (CF32) {
+                float* crow = (float*)jb.C + (size_t)row * p.nb + bj * OZ_BN + c0;
 #pragma unroll
-        for (int j = 0; j < OZ_BN; j += 2) {
-            double2 c = *(double2*)(crow + j);
-            c.x -= acc[j] * rs * colscale[j];
-            c.y -= acc[j + 1] * rs * colscale[j + 1];
-            *(double2*)(crow + j) = c;
+                for (int j = 0; j < 32; j += 4) {
+                    float4 c = *(float4*)(crow + j);
+                    c.x = (float)((double)c.x - acc[j] * rs * colscale[c0 + j]);
+                    c.y = (float)((double)c.y - acc[j + 1] * rs * colscale[c0 + j + 1]);
+                    c.z = (float)((double)c.z - acc[j + 2] * rs * colscale[c0 + j + 2]);
+                    c.w = (float)((double)c.w - acc[j + 3] * rs * colscale[c0 + j + 3]);
+                    *(float4*)(crow + j) = c;
+                }
+            } else {
+                double* crow = (double*)jb.C + (size_t)row * p.nb + bj * OZ_BN + c0;
+#pragma unroll
+                for (int j = 0; j < 32; j += 2) {
+                    double2 c = *(double2*)(crow + j);
+                    c.x -= acc[j] * rs * colscale[c0 + j];
+                    c.y -= acc[j + 1] * rs * colscale[c0 + j + 1];
+                    *(double2*)(crow + j) = c;
+                }
+            }
         }
     }
     oz_fence_before();
@@ -326,20 +348,22 @@ static bool oz_map(CUtensorMap* m, const int8_t* base, uint64_t planes, uint64_t
               CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
 }
 
-template <int S, int CL>
+template <int S, int CL, bool CF32>
 static cudaError_t oz_launch_s(const OzArgs& a, int njobs, cudaStream_t s) {
+    constexpr int OZ_BN = OzCfg<S>::BN;
     constexpr int SMEM = OZ_STAGES * S * (OZ_BM + OZ_BN) * OZ_BK + 1024;
     static bool attr = false;
     if (!attr) {
-        cudaError_t e = cudaFuncSetAttribute(ozaki_gemm_kernel<S, CL>, cudaFuncAttributeMaxDynamicSharedMemorySize, SMEM);
+        cudaError_t e = cudaFuncSetAttribute(ozaki_gemm_kernel<S, CL, CF32>, cudaFuncAttributeMaxDynamicSharedMemorySize, SMEM);
         if (e != cudaSuccess) return e;
         attr = true;
     }
     OzParams p;
     memset(&p, 0, sizeof p);
     const uint64_t rows = (uint64_t)a.nt * a.nb;
-    if (!oz_map(&p.a, a.slices, S, rows, a.nb, a.plane_stride, OZ_BM, S / CL) ||
-        !oz_map(&p.b, a.slices, S, rows, a.nb, a.plane_stride, OZ_BN, S))
+    // the slice cache always holds 8 planes; an S-slice GEMM reads the first S (prefix-consistent split)
+    if (!oz_map(&p.a, a.slices, 8, rows, a.nb, a.plane_stride, OZ_BM, S / CL) ||
+        !oz_map(&p.b, a.slices, 8, rows, a.nb, a.plane_stride, OZ_BN, S))
         return cudaErrorInvalidValue;
     p.jobs = a.jobs;
     p.exps = a.exps;
@@ -361,7 +385,7 @@ static cudaError_t oz_launch_s(const OzArgs& a, int njobs, cudaStream_t s) {
     at[0].val.clusterDim.z = 1;
     cfg.attrs = at;
     cfg.numAttrs = 1;
-    return cudaLaunchKernelEx(&cfg, ozaki_gemm_kernel<S, CL>, p);
+    return cudaLaunchKernelEx(&cfg, ozaki_gemm_kernel<S, CL, CF32>, p);
 }
 
 cudaError_t ozaki_gemm_launch(const OzArgs& a, int njobs, cudaStream_t s) {
@@ -371,7 +395,8 @@ cudaError_t ozaki_gemm_launch(const OzArgs& a, int njobs, cudaStream_t s) {
         const char* e = getenv("MPGEO_OZAKI_CLUSTER");
         return e ? atoi(e) : 2;
     }();
-    if (a.S == 8) return cl == 2 ? oz_launch_s<8, 2>(a, njobs, s) : oz_launch_s<8, 1>(a, njobs, s);
+    if (a.S == 8 && !a.c_f32) return cl == 2 ? oz_launch_s<8, 2, false>(a, njobs, s) : oz_launch_s<8, 1, false>(a, njobs, s);
+    if (a.S == 4 && a.c_f32) return cl == 2 ? oz_launch_s<4, 2, true>(a, njobs, s) : oz_launch_s<4, 1, true>(a, njobs, s);
     return cudaErrorInvalidValue;  // S = 8 is the only validated split (FP64-level accuracy)
 }
 

@@ -12,7 +12,7 @@ struct OzSplitItem {
 };
 struct OzJob {
     int m, n;   // panel rows of the operands (slice-cache rows m*nb.., n*nb..)
-    double* C;  // FP64 nb x nb output tile
+    void* C;    // nb x nb output tile (FP64, or FP32 when c_f32)
 };
 struct OzArgs {
     const OzJob* jobs;
@@ -20,6 +20,7 @@ struct OzArgs {
     const int* exps;       // [nt*nb] row exponents
     int64_t plane_stride;  // = nt*nb*nb
     int nb, nt, S, lower;
+    int c_f32;             // C tiles are FP32 (FP32 class, S = 4) instead of FP64 (S = 8)
 };
 bool ozaki_available();
 cudaError_t ozaki_split_launch(const OzSplitItem* items, int n, int nb, int S, cudaStream_t s);

@@ -121,6 +121,26 @@ __global__ void __launch_bounds__(PT, 1) trtri_blocks_kernel(const double* L, in
     write_block(S, wd, jb, nullptr, 0, W + (size_t)b * PB * PB);
 }
 
+// Batched: blockIdx.y selects the diagonal tile; W layout [tile][block][128][128].
+__global__ void __launch_bounds__(PT, 1) trtri_batch_kernel(const double* const* Ls, int nb, double* W) {
+    extern __shared__ double S[];
+    double* wd = S + PB * PLD + PB;
+    double* rowp = wd + PB;
+    const int b = blockIdx.x, t = blockIdx.y;
+    const int nblk = (nb + PB - 1) / PB;
+    const int j0 = b * PB;
+    const int jb = min(PB, nb - j0);
+    const double* Lb = Ls[t] + (size_t)j0 * nb + j0;
+    const int tid = threadIdx.x;
+    for (int idx = tid; idx < jb * jb; idx += PT) {
+        const int r = idx / jb, c = idx - r * jb;
+        if (c <= r) S[r * PLD + c] = Lb[(size_t)r * nb + c];
+    }
+    __syncthreads();
+    smem_trtri_gj(S, wd, rowp, jb);
+    write_block(S, wd, jb, nullptr, 0, W + ((size_t)t * nblk + b) * PB * PB);
+}
+
 static cudaError_t set_smem(const void* f, int bytes) {
     return cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, bytes);
 }
@@ -134,6 +154,18 @@ cudaError_t potrf_diag_block_launch(double* A, int lda, int jb, double* W, int c
         init = true;
     }
     potrf_diag_block_kernel<<<1, PT, P_SMEM, s>>>(A, lda, jb, W, col0, info);
+    return cudaGetLastError();
+}
+
+cudaError_t trtri_batch_launch(const double* const* Ls, int ntiles, int nb, double* W, cudaStream_t s) {
+    static bool init = false;
+    if (!init) {
+        cudaError_t e = set_smem((const void*)trtri_batch_kernel, P_SMEM);
+        if (e != cudaSuccess) return e;
+        init = true;
+    }
+    if (ntiles <= 0) return cudaSuccess;
+    trtri_batch_kernel<<<dim3((nb + PB - 1) / PB, ntiles), PT, P_SMEM, s>>>(Ls, nb, W);
     return cudaGetLastError();
 }
 

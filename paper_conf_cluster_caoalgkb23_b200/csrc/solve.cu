@@ -117,6 +117,47 @@ __global__ void sumsq_chunks_kernel(const double* v, int64_t n, int chunk, doubl
     }
 }
 
+// ---- blocked TRSV on one diagonal tile with the 128-block inverses W_j = L_jj^{-1}:
+//   y_j = W_j r_j  (one CTA),  then  r_i -= L_ij y_j  for the rows below (many CTAs)
+constexpr int TB = 128;
+
+__global__ void __launch_bounds__(128) blk_matvec_kernel(const double* W, const double* r, double* y, int jb) {
+    // warp per row, lanes over columns: y[i] = sum_c W[i][c] r[c]
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    for (int i = warp; i < jb; i += 4) {
+        double s = 0.0;
+        for (int c = lane; c < jb; c += 32) s = fma(W[i * TB + c], r[c], s);
+        s = warp_sum(s);
+        if (lane == 0) y[i] = s;
+    }
+}
+
+__global__ void __launch_bounds__(256) blk_update_kernel(const double* L, int nb, int j0, int jb, const double* y,
+                                                         double* r, int row0) {
+    // rows i = row0 + blockIdx.x*8 + warp: r[i] -= sum_c L[i][j0 + c] y[c]
+    __shared__ double ys[TB];
+    for (int c = threadIdx.x; c < jb; c += 256) ys[c] = y[c];
+    __syncthreads();
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    const int i = row0 + blockIdx.x * 8 + warp;
+    if (i >= nb) return;
+    const double* row = L + (size_t)i * nb + j0;
+    double s = 0.0;
+    for (int c = lane; c < jb; c += 32) s = fma(row[c], ys[c], s);
+    s = warp_sum(s);
+    if (lane == 0) r[i] -= s;
+}
+
+cudaError_t trsv_blocked_launch(const double* L, int nb, const double* Wk, double* r, double* y, cudaStream_t s) {
+    for (int j0 = 0; j0 < nb; j0 += TB) {
+        const int jb = nb - j0 < TB ? nb - j0 : TB;
+        blk_matvec_kernel<<<1, 128, 0, s>>>(Wk + (size_t)(j0 / TB) * TB * TB, r + j0, y + j0, jb);
+        const int rows = nb - (j0 + jb);
+        if (rows > 0) blk_update_kernel<<<(rows + 7) / 8, 256, 0, s>>>(L, nb, j0, jb, y + j0, r, j0 + jb);
+    }
+    return cudaGetLastError();
+}
+
 cudaError_t trsv_tile_launch(const double* L, int nb, const double* r, double* y, cudaStream_t s) {
     const int smem = nb * 8;
     if (smem > 48 * 1024) {

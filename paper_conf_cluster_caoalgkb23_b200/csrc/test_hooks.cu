@@ -73,7 +73,7 @@ mp_status mp_test_ozaki_gemm(const double* d_panel, double* d_C, int nb, int nt,
     int* ex = nullptr;
     OzSplitItem* it = nullptr;
     OzJob* dj = nullptr;
-    if (cudaMalloc(&sl, plane * S) || cudaMalloc(&ex, sizeof(int) * nt * nb) ||
+    if (cudaMalloc(&sl, plane * 8) || cudaMalloc(&ex, sizeof(int) * nt * nb) ||
         cudaMalloc(&it, sizeof(OzSplitItem) * nt) || cudaMalloc(&dj, sizeof(OzJob)))
         return MP_ERR_CUDA;
     std::vector<OzSplitItem> h(nt);
@@ -82,8 +82,8 @@ mp_status mp_test_ozaki_gemm(const double* d_panel, double* d_C, int nb, int nt,
     cudaMemcpy(it, h.data(), sizeof(OzSplitItem) * nt, cudaMemcpyHostToDevice);
     OzJob j{m, n, d_C};
     cudaMemcpy(dj, &j, sizeof j, cudaMemcpyHostToDevice);
-    cudaError_t e = ozaki_split_launch(it, nt, nb, S, 0);
-    OzArgs a{dj, sl, ex, plane, nb, nt, S, lower};
+    cudaError_t e = ozaki_split_launch(it, nt, nb, 8, 0);  // the cache always holds 8 planes
+    OzArgs a{dj, sl, ex, plane, nb, nt, S, lower, S == 4 ? 1 : 0};  // S = 4: FP32 class, C is float
     if (e == cudaSuccess) e = ozaki_gemm_launch(a, 1, 0);
     cudaError_t e2 = cudaDeviceSynchronize();
     cudaFree(sl);

@@ -154,3 +154,21 @@ def test_ozaki_int8_fp64_gemm(lib, S):
                 assert np.array_equal(got2[blk], Cm[blk])
             else:
                 assert np.max(np.abs(got2[blk] - ref2[blk])) <= 1e-9
+
+
+def test_ozaki_int8_fp32_class_gemm(lib):
+    """FP32 class on INT8 tensor cores (first 4 slices = 28 bits, reading C13b): error vs the exact
+    product of the FP32 operands within 2x an SGEMM's on the same inputs (the C13 pin)."""
+    nb, nt = 512, 2
+    rng = np.random.default_rng(11)
+    A32 = (rng.standard_normal((nt * nb, nb)) * np.exp(rng.uniform(-2, 2, (nt * nb, 1)))).astype(np.float32)
+    Cm = np.zeros((nb, nb), np.float32)
+    dP, dC = dev(A32.astype(np.float64)), dev(Cm)
+    assert lib.mp_test_ozaki_gemm(C.c_void_p(dP.data_ptr()), C.c_void_p(dC.data_ptr()), nb, nt, 1, 0, 4, 0) == 0
+    got = -dC.cpu().numpy().astype(np.float64)
+    Ad = A32.astype(np.float64)
+    exact = Ad[nb:] @ Ad[:nb].T
+    sgemm = (A32[nb:] @ A32[:nb].T).astype(np.float64)
+    err = np.linalg.norm(got - exact) / np.linalg.norm(exact)
+    err_sg = np.linalg.norm(sgemm - exact) / np.linalg.norm(exact)
+    assert err <= 2 * err_sg, (err, err_sg)
