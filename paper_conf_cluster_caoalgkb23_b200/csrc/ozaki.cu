@@ -76,7 +76,7 @@ cudaError_t ozaki_split_launch(const OzSplitItem* items, int n, int nb, int S, c
 }
 
 // ------------------------------------------------------------------ GEMM
-constexpr int OZ_BM = 128, OZ_BK = 64, OZ_THREADS = 256, OZ_STAGES = 2;
+constexpr int OZ_BM = 128, OZ_BK = 64, OZ_THREADS = 256;
 
 struct __align__(64) OzParams {
     CUtensorMap a, b;  // 3D [S][rows][nb] int8, boxes {64, 128, S / CL} and {64, 64, S}
@@ -91,6 +91,7 @@ template <int S>
 struct OzCfg {
     static constexpr int BN = 512 / S;
     static constexpr int PER_MMA = 256 / BN;  // B slices concatenated per MMA (N <= 256)
+    static constexpr int STAGES = S == 8 ? 2 : 3;  // 96 KB / 64 KB per stage
 };
 
 __device__ __forceinline__ uint32_t oz_smem_u32(const void* p) { return (uint32_t)__cvta_generic_to_shared(p); }
@@ -180,7 +181,7 @@ __global__ void __launch_bounds__(OZ_THREADS, 1) ozaki_gemm_kernel(const __grid_
     constexpr int A_SL = OZ_BM * OZ_BK;     // bytes of one A slice block (8 KB)
     constexpr int B_SL = OZ_BN * OZ_BK;     // 4 KB (BN = 64) or 8 KB (BN = 128)
     constexpr int STAGE = S * (A_SL + B_SL);
-    constexpr int NG = S;                   // groups g = 2 .. S+1
+    constexpr int OZ_STAGES = OzCfg<S>::STAGES;
     extern __shared__ uint8_t oz_smem_raw[];
     uint8_t* smem = (uint8_t*)(((uintptr_t)oz_smem_raw + 1023) & ~(uintptr_t)1023);
     __shared__ __align__(8) uint64_t full_bar[OZ_STAGES], empty_bar[OZ_STAGES], done_bar;
@@ -351,7 +352,7 @@ static bool oz_map(CUtensorMap* m, const int8_t* base, uint64_t planes, uint64_t
 template <int S, int CL, bool CF32>
 static cudaError_t oz_launch_s(const OzArgs& a, int njobs, cudaStream_t s) {
     constexpr int OZ_BN = OzCfg<S>::BN;
-    constexpr int SMEM = OZ_STAGES * S * (OZ_BM + OZ_BN) * OZ_BK + 1024;
+    constexpr int SMEM = OzCfg<S>::STAGES * S * (OZ_BM + OZ_BN) * OZ_BK + 1024;
     static bool attr = false;
     if (!attr) {
         cudaError_t e = cudaFuncSetAttribute(ozaki_gemm_kernel<S, CL, CF32>, cudaFuncAttributeMaxDynamicSharedMemorySize, SMEM);
