@@ -683,7 +683,7 @@ static mp_status plan_potrf(mp_handle* h, mp_matrix* A, const uint8_t* km, const
     auto cur_push = [&](Op o) { cur->push_back(std::move(o)); };
     // ---- multi-rank exchange helpers; unused on one rank
     const bool dist = h->nranks > 1;
-    const bool la = h->lookahead && !dist;
+    const bool la = h->lookahead != 0;  // also multi-rank: exchange waits run on the panel stream
     const int R = h->nranks, me = h->rank;
     Comm& X = A->comm;
     auto ST = [&](int step) -> uint64_t { return (epoch << 24) + (uint64_t)(step + 2); };
