@@ -50,7 +50,7 @@ struct mp_handle {
     int tc_mode = 1;  // 1: tcgen05 kernels for FP32/FP16 classes when available, 0: DMMA emulation
     int lookahead = 1;  // 1: panel k+1 on the high-priority panel stream overlaps update k
     int ozaki = 8;      // 8: FP64-class GEMM/SYRK emulated on INT8 tensor cores (S = 8 slices); 0: DMMA
-    int ozaki32 = 1;    // 1: FP32-class GEMM on INT8 tensor cores (first 4 slices); 0: 3xTF32 tcgen05
+    int ozaki32 = 0;    // 1: FP32-class GEMM on INT8 tensor cores (first 4 slices); 0: 3xTF32 tcgen05 (default)
     cudaStream_t pstream = nullptr;
     std::vector<cudaEvent_t> sync_ev;
     // profiling (mp_set_profiling): event pairs per launch, resolved in mp_get_profile

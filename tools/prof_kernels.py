@@ -44,8 +44,18 @@ def main(which):
         nb, nt = 2048, 4
         P = torch.randn(nt * nb, nb, dtype=torch.float64, device="cuda")
         Cm = torch.zeros(nb, nb, dtype=torch.float64, device="cuda")
+        C32 = torch.zeros(nb, nb, dtype=torch.float32, device="cuda")
         for _ in range(3):
             assert lib.mp_test_ozaki_gemm(p(P), p(Cm), nb, nt, 2, 1, 8, 0) == 0
+            assert lib.mp_test_ozaki_gemm(p(P), p(C32), nb, nt, 2, 1, 4, 0) == 0
+        for S, Cx in ((8, Cm), (4, C32)):
+            s, e = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            s.record()
+            for _ in range(5):
+                lib.mp_test_ozaki_gemm(p(P), p(Cx), nb, nt, 2, 1, S, 0)
+            e.record()
+            torch.cuda.synchronize()
+            print(f"ozaki S={S}: {s.elapsed_time(e) / 5:.3f} ms per call (incl. split of {nt} tiles + malloc)")
     if which in ("tf32err", "all"):
         from tests.test_gpu_kernels import tf32_rna
         for K in (64, 256, 1024, 2048):
