@@ -47,6 +47,13 @@ FP64_NOMINAL, BF16_NOMINAL, INT8_NOMINAL = 40.0, 2250.0, 4500.0  # dense TFLOP/s
 OZ_PRODUCTS = 36  # int8 GEMMs per FP64 GEMM in the Ozaki split with S = 8 slices (S (S+1) / 2)
 
 
+def ncu_traffic():
+    """dram bytes per FP64-equivalent flop of the dominant kernel, from one `ncu --set full` capture of a
+    launch inside a bench run (profiles/r01/ncu_traffic.json, written by tools/ncu_traffic.py)."""
+    p = os.path.join(ROOT, "profiles", "r01", "ncu_traffic.json")
+    return json.load(open(p)) if os.path.exists(p) else None
+
+
 def measured_peaks():
     p = os.path.join(ROOT, "MEASURED_PEAKS.json")
     if os.path.exists(p):
@@ -328,6 +335,12 @@ def main():
     fp64_peak = peaks["bf16_tflops_sustained"] * FP64_NOMINAL / BF16_NOMINAL
     int8_peak = peaks["bf16_tflops_sustained"] * INT8_NOMINAL / BF16_NOMINAL
     fp64_eq = dom["flops"] / (dom["ms"] / 1e3) / 1e12 if dom["ms"] > 0 else 0.0
+    flops_per_launch = dom["flops"] / max(1, dom["launches"])
+    tr = ncu_traffic()
+    traffic = (tr["dram_bytes_per_flop"] * flops_per_launch) if tr and engine["ozaki"] % 100 == 8 else None
+    # algorithmic bytes of an FP64-class tile-GEMM on the INT8 path: 8 int8 planes of A and B (8 B/entry each)
+    # + row exponents + the FP64 C tile read and written (16 B/entry)
+    alg_bytes_per_launch = flops_per_launch / (2.0 * nb**3) * (8 + 8 + 16) * nb * nb
     try:
         cub = cublas_dgemm_tflops()
     except Exception:
@@ -366,7 +379,9 @@ def main():
         "roofline": (
             {"bound": "tensor", "kernel": "ozaki_gemm_kernel<8> (FP64-class update as 36 INT8 tcgen05 GEMMs)",
              "achieved": OZ_PRODUCTS * fp64_eq, "peak": int8_peak, "unit": "TFLOP/s",
-             "frac": OZ_PRODUCTS * fp64_eq / int8_peak, "traffic": None,
+             "frac": OZ_PRODUCTS * fp64_eq / int8_peak, "traffic": traffic,
+             "algorithmic_bytes_per_launch": alg_bytes_per_launch,
+             "traffic_source": tr.get("source") if tr else None,
              "peak_source": f"{peak_src} bf16_tflops_sustained x {INT8_NOMINAL}/{BF16_NOMINAL} (INT8 nominal / bf16 nominal); "
                             "achieved = executed int8 multiply-add ops x 2 per second",
              "fp64_equivalent_tflops": fp64_eq, "cublas_dgemm_tflops_live": cub,
