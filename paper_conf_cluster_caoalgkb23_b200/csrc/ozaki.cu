@@ -397,7 +397,8 @@ cudaError_t ozaki_gemm_launch(const OzArgs& a, int njobs, cudaStream_t s) {
         return e ? atoi(e) : 2;
     }();
     if (a.S == 8 && !a.c_f32) return cl == 2 ? oz_launch_s<8, 2, false>(a, njobs, s) : oz_launch_s<8, 1, false>(a, njobs, s);
-    if (a.S == 4 && a.c_f32) return cl == 2 ? oz_launch_s<4, 2, true>(a, njobs, s) : oz_launch_s<4, 1, true>(a, njobs, s);
+    // S = 4: the 2-CTA multicast variant measured 2.6x slower than single-CTA (profiles/r01): no cluster
+    if (a.S == 4 && a.c_f32) return oz_launch_s<4, 1, true>(a, njobs, s);
     return cudaErrorInvalidValue;  // S = 8 is the only validated split (FP64-level accuracy)
 }
 
