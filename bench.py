@@ -49,7 +49,7 @@ OZ_PRODUCTS = 36  # int8 GEMMs per FP64 GEMM in the Ozaki split with S = 8 slice
 
 def ncu_traffic():
     """dram bytes per FP64-equivalent flop of the dominant kernel, from one `ncu --set full` capture of a
-    launch inside a bench run (profiles/r01/ncu_traffic.json, written by tools/ncu_traffic.py)."""
+    launch inside a bench run (profiles/r01/ncu_traffic.json records the capture and its command)."""
     p = os.path.join(ROOT, "profiles", "r01", "ncu_traffic.json")
     return json.load(open(p)) if os.path.exists(p) else None
 
@@ -204,6 +204,7 @@ def main():
     ap.add_argument("--map", default=None, choices=["adaptive", "fp64", "band", "extreme"])
     ap.add_argument("--policy", default="auto", choices=["auto", "ttc"])
     ap.add_argument("--u-req", type=float, default=1e-9)
+    ap.add_argument("--theta", default=None, help="sigma2,beta,nu override (e.g. 1,0.03,0.8 for the Bessel path)")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--replicas", action="store_true", help="N>1: independent evaluations per rank")
@@ -211,6 +212,8 @@ def main():
     cfg = dict(CONFIGS[args.config])
     if args.map:
         cfg["map"] = args.map
+    if args.theta:
+        cfg["theta"] = tuple(float(v) for v in args.theta.split(","))
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
     local = int(os.environ.get("LOCAL_RANK", "0"))
