@@ -50,6 +50,7 @@ struct mp_handle {
     int tc_mode = 1;  // 1: tcgen05 kernels for FP32/FP16 classes when available, 0: DMMA emulation
     int lookahead = 1;  // 1: panel k+1 on the high-priority panel stream overlaps update k
     int ozaki = 8;      // 8: FP64-class GEMM/SYRK emulated on INT8 tensor cores (S = 8 slices); 0: DMMA
+    int matern_table = 1;  // general nu: tabulated correlation (1) or direct K_nu per entry (0)
     int ozaki32 = 0;    // 1: FP32-class GEMM on INT8 tensor cores (first 4 slices); 0: 3xTF32 tcgen05 (default)
     cudaStream_t pstream = nullptr;
     std::vector<cudaEvent_t> sync_ev;
@@ -64,7 +65,7 @@ struct mp_handle {
 struct Regions {
     size_t total = 0;
     size_t inputs = 0, p64 = 0, p16 = 0, phi = 0, plo = 0, ltilde = 0, wbuf = 0, wbuf2 = 0, oz = 0, ozexp = 0,
-           wdiag = 0;
+           wdiag = 0, mtab = 0;
     size_t vec_r = 0, vec_y = 0, partials = 0, norms = 0, ctrl = 0, ctrl_bytes = 0;
     std::vector<size_t> tile_off;  // per (m*nt+k), SIZE_MAX if not stored here
 };
@@ -118,6 +119,7 @@ struct mp_matrix {
     } while (0)
 
 static size_t align_up(size_t v, size_t a) { return (v + a - 1) / a * a; }
+constexpr int MT_PIECES_MAX = 512;
 static int ceil_div(int a, int b) { return (a + b - 1) / b; }
 
 // Upper bound of control-arena bytes for one call on an nt x nt tile matrix.
@@ -162,6 +164,7 @@ static Regions layout(const mp_matrix* A, const uint8_t* storage) {
     R.wbuf = take((size_t)POTRF_IB * POTRF_IB * 8);
     R.wbuf2 = take((size_t)ceil_div(A->nb, POTRF_IB) * POTRF_IB * POTRF_IB * 8);
     R.wdiag = take((size_t)nt * ceil_div(A->nb, POTRF_IB) * POTRF_IB * POTRF_IB * 8);  // solve: block inverses
+    R.mtab = take((size_t)MT_PIECES_MAX * (MT_DEG + 1) * 8);  // general-nu Matern table
     // two sets of panel buffers (panel parity) so panel k+1 can be produced while update k reads panel k
     R.p64 = take(2 * (size_t)nt * nb2 * 8);
     R.p16 = take(2 * (size_t)nt * nb2 * 2);
@@ -274,6 +277,7 @@ mp_status mp_init(int device, int rank, int nranks, int P, int Q, const uint8_t*
     if (const char* e = getenv("MPGEO_LOOKAHEAD")) h->lookahead = atoi(e);
     if (const char* e = getenv("MPGEO_OZAKI")) h->ozaki = atoi(e);
     if (const char* e = getenv("MPGEO_OZAKI32")) h->ozaki32 = atoi(e);
+    if (const char* e = getenv("MPGEO_MATERN_TABLE")) h->matern_table = atoi(e);
     auto fail = [&](mp_status s) {
         if (h->own_stream && h->stream) cudaStreamDestroy(h->stream);
         delete h;
@@ -562,7 +566,7 @@ mp_status mp_matrix_set_covariance(mp_matrix* A, mp_covariance kind) {
 }
 
 static MaternArgs matern_args(const mp_matrix* A, const double* x, const double* y, const double* th) {
-    MaternArgs a;
+    MaternArgs a{};
     a.x = x;
     a.y = y;
     a.n = A->n;
@@ -588,7 +592,27 @@ mp_status mp_matern_gen(mp_handle* h, mp_matrix* A, const double* d_x, const dou
     if (mp_status s = check_theta(h, theta, A->cov)) return s;
     if (h->nranks > 1 && !A->comm.connected) FAIL(h, MP_ERR_COMM, "multi-rank matrix not connected");
     const int nt = A->nt;
-    const MaternArgs a = matern_args(A, d_x, d_y, theta);
+    MaternArgs a = matern_args(A, d_x, d_y, theta);
+    if (a.kind == 3 && A->bound && h->matern_table) {
+        // pieces of width w = 1/8 in u = log r on [log 2 - w*split, log r_max]; r_max bounds every
+        // distance of points in the unit square (sqrt 2) — outside points fall back to direct K_nu
+        const double w = 0.125;
+        const double rmax = 1.5 / a.beta;
+        const int split = 96;  // 12 units of u below log 2: r down to 2 e^-12 ~ 1.2e-5
+        const int above = std::max(1, (int)std::ceil((std::log(rmax) - std::log(2.0)) / w));
+        if (split + above <= MT_PIECES_MAX) {
+            a.u0 = std::log(2.0) - w * split;
+            a.w = w;
+            a.inv_w = 1.0 / w;
+            a.split = split;
+            a.npieces = split + above;
+            double* tab = A->at<double>(A->R.mtab);
+            a.tab = nullptr;  // the table kernel samples the direct formula
+            CK(h, matern_table_launch(a, tab, h->stream));
+            h->launches++;
+            a.tab = tab;
+        }
+    }
     if (!storage_prec) {
         // pass 1: norms.  Needs scratch for partials: use the bound workspace if present,
         // otherwise the caller must bind first (norm scratch lives in the workspace).

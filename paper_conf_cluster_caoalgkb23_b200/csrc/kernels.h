@@ -45,7 +45,14 @@ struct MaternArgs {
     double sigma2, beta, nu;
     int kind;     // 0: nu = 1/2, 1: nu = 3/2, 2: nu = 5/2, 3: general nu, 4: squared exponential
     double coef;  // 2^(1-nu) / Gamma(nu) for the general formula
+    // general nu: piecewise Chebyshev table of the normalised correlation in u = log(r) (see matern.cu)
+    const double* tab;  // [npieces][MT_DEG + 1] coefficients, null = evaluate K_nu directly
+    double u0, inv_w, w;
+    int npieces, split;  // pieces p >= split carry rho(r) e^r (r > 2), pieces below carry rho(r)
 };
+constexpr int MT_DEG = 11;  // Chebyshev degree per piece
+// Build the table for kind 3 (one CTA per piece); pieces of width w in u = log r from u0.
+cudaError_t matern_table_launch(const MaternArgs& a, double* tab, cudaStream_t s);
 constexpr int GEN_ROWS = 16;  // rows per CTA in the generation kernels
 // Pass 1: partial sums of squares, partials[t * (nb/GEN_ROWS) + chunk]
 cudaError_t matern_norm_launch(const MaternArgs& a, const GenTile* tiles, int ntiles, double* partials,
