@@ -251,3 +251,29 @@ def test_sqexp_covariance_path(mp, handle):
     ev = mp.Evaluator(n, nb, handle=handle, covariance=mp.MP_COV_SQEXP)
     r = ev.eval(x, y, z, theta, mode=mp.MP_MAP_FP64)
     assert abs(r.loglik - ref["loglik"]) <= 1e-10 * abs(ref["loglik"])
+
+
+@pytest.mark.parametrize("nu", [0.3, 0.8, 1.7, 3.2])
+def test_general_nu_tabulated_generation_vs_mpmath(mp, handle, nu):
+    """General nu is generated from a per-evaluation piecewise Chebyshev table of the correlation
+    (matern.cu): sampled entries against 30-digit mpmath, relative error <= (3 + r) * 2^-52."""
+    import mpmath
+    mpmath.mp.dps = 30
+    n, nb, theta = 4096, 512, (1.4, 0.04, nu)
+    x, y = synth.locations(n, 6)
+    M = mp.Matrix(handle, n, nb, None)
+    M.matern_gen(to_dev(x), to_dev(y), theta, np.zeros((M.nt, M.nt), np.uint8))
+    rng = np.random.default_rng(int(nu * 10))
+    for (m, k) in [(0, 0), (3, 2), (7, 0), (5, 5)]:
+        t = M.tile(m, k)
+        for _ in range(12):
+            i, j = int(rng.integers(0, nb)), int(rng.integers(0, nb))
+            gi, gj = m * nb + i, k * nb + j
+            if gi == gj:
+                continue
+            dx, dy = x[gi] - x[gj], y[gi] - y[gj]
+            h = float(np.sqrt(dx * dx + dy * dy))
+            r = mpmath.mpf(h) / mpmath.mpf(theta[1])
+            ref = float(mpmath.mpf(theta[0]) * 2 ** (1 - mpmath.mpf(nu)) / mpmath.gamma(nu) * r**nu
+                        * mpmath.besselk(nu, r))
+            assert abs(t[i, j] - ref) <= (3 + float(r)) * 2.0**-52 * abs(ref) + 1e-300, (nu, m, k, i, j)
