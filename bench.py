@@ -229,11 +229,16 @@ def main():
     import paper_conf_cluster_caoalgkb23_b200 as mp
     import synth
 
+    # one process per GPU; on a box with fewer GPUs than ranks the ranks share devices (the peer-memory
+    # exchange then runs over same-device IPC) — used to validate the N > 1 path on one GPU
+    local = local % torch.cuda.device_count()
     torch.cuda.set_device(local)
     dist = None
     if world > 1:
         import torch.distributed as dist
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        # the process group only carries timings and the 64-byte IPC handles (the data path is the
+        # library's own peer-memory exchange), so gloo is enough
+        dist.init_process_group("gloo")
     n, nb, theta = cfg["n"], cfg["nb"], cfg["theta"]
     mode = {"adaptive": mp.MP_MAP_ADAPTIVE, "fp64": mp.MP_MAP_FP64, "band": mp.MP_MAP_BAND,
             "extreme": mp.MP_MAP_EXTREME}[cfg["map"]]
@@ -267,9 +272,9 @@ def main():
     torch.cuda.synchronize()
 
     def barrier():
+        torch.cuda.synchronize()
         if dist:
             dist.barrier()
-        torch.cuda.synchronize()
 
     # ---- timed region: K evaluations, inputs resident in HBM
     clocks = ClockSampler(local)
@@ -292,12 +297,14 @@ def main():
     h.set_profiling(False)
     t_ms = ev_s.elapsed_time(ev_e)
     if dist:
-        t = torch.tensor([t_ms], device="cuda")
+        t = torch.tensor([t_ms], dtype=torch.float64)
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
         t_ms = float(t.item())
     joules = None if e0_mj is None or e1_mj is None else (e1_mj - e0_mj) / 1e3
+    if joules is not None and rank >= torch.cuda.device_count():
+        joules = 0.0  # ranks sharing a device (single-GPU validation): count each GPU once
     if dist and joules is not None:
-        t = torch.tensor([joules], device="cuda", dtype=torch.float64)
+        t = torch.tensor([joules], dtype=torch.float64)
         dist.all_reduce(t)
         joules = float(t.item())
     flops_eval = n**3 / 3.0
@@ -317,7 +324,7 @@ def main():
         barrier()
         te = es.elapsed_time(ee)
         if dist:
-            t = torch.tensor([te], device="cuda")
+            t = torch.tensor([te], dtype=torch.float64)
             dist.all_reduce(t, op=dist.ReduceOp.MAX)
             te = float(t.item())
         nt = ev.nt
