@@ -594,7 +594,7 @@ mp_status mp_matern_gen(mp_handle* h, mp_matrix* A, const double* d_x, const dou
     const int nt = A->nt;
     MaternArgs a = matern_args(A, d_x, d_y, theta);
     if (a.kind == 3 && A->bound && h->matern_table) {
-        // pieces of width w = 1/8 in u = log r on [log 2 - w*split, log r_max]; r_max bounds every
+        // pieces of width w = 1/8 in u = log(r/2) on [-w*split, log(r_max/2)]; r_max bounds every
         // distance of points in the unit square (sqrt 2) — outside points fall back to direct K_nu
         const double w = 0.125;
         const double rmax = 1.5 / a.beta;

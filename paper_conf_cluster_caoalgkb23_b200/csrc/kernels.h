@@ -50,7 +50,7 @@ struct MaternArgs {
     double u0, inv_w, w;
     int npieces, split;  // pieces p >= split carry rho(r) e^r (r > 2), pieces below carry rho(r)
 };
-constexpr int MT_DEG = 11;  // Chebyshev degree per piece
+constexpr int MT_DEG = 15;  // Chebyshev degree per piece
 // Build the table for kind 3 (one CTA per piece); pieces of width w in u = log r from u0.
 cudaError_t matern_table_launch(const MaternArgs& a, double* tab, cudaStream_t s);
 constexpr int GEN_ROWS = 16;  // rows per CTA in the generation kernels
