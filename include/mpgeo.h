@@ -211,6 +211,11 @@ mp_status mp_tile_potrf(mp_handle* h, mp_matrix* A, const uint8_t* kernel_prec,
 mp_status mp_loglik(mp_handle* h, const mp_matrix* L, const double* d_z,
                     double* loglik, double* logdet, double* quad);
 
+/* Sample the Gaussian field with covariance L L^T: d_z = L d_e (device FP64 [n] each), with L the
+ * factor left in A by mp_tile_potrf (read in storage precision).  With e ~ N(0, I) this gives the
+ * synthetic measurement vectors Z = L(theta) e of the Monte-Carlo studies.  One rank only. */
+mp_status mp_gp_sample(mp_handle* h, const mp_matrix* L, const double* d_e, double* d_z);
+
 /* One whole evaluation (the call a user makes): (1) pass 1, (2), (1) pass 2,
  * (3), (4).  x, y, z are FP64 [n]; if `inputs_on_host` is nonzero they are host
  * pointers and are copied to the device inside the call (pinned memory makes

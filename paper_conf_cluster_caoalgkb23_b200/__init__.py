@@ -179,6 +179,10 @@ class Matrix:
         self.handle.check(st)
         return 0
 
+    def gp_sample(self, e, z):
+        """z = L e with the factor in this matrix (device tensors, FP64 [n])."""
+        self.handle.check(lib.mp_gp_sample(self.handle.h, self.A, C.c_void_p(_ptr(e)), C.c_void_p(_ptr(z))))
+
     def loglik(self, z) -> tuple[float, float, float]:
         ll, ld, q = C.c_double(), C.c_double(), C.c_double()
         self.handle.check(lib.mp_loglik(self.handle.h, self.A, C.c_void_p(_ptr(z)), C.byref(ll), C.byref(ld),

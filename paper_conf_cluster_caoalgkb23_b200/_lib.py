@@ -71,6 +71,7 @@ def _load() -> C.CDLL:
         "mp_precision_map": (i32, [i32, dp, dbl, dp, i32, u8p, u8p, u8p]),
         "mp_tile_potrf": (i32, [vp, vp, u8p, u8p, C.POINTER(i64)]),
         "mp_loglik": (i32, [vp, vp, vp, dp, dp, dp]),
+        "mp_gp_sample": (i32, [vp, vp, vp, vp]),
         "mp_eval": (i32, [vp, vp, vp, vp, vp, i32, dp, dbl, dp, i32, i32, u8p, C.POINTER(EvalReport)]),
         "mp_matrix_maps": (i32, [vp, u8p, u8p, u8p]),
         "mp_matrix_get_tile": (i32, [vp, vp, i32, i32, dp]),

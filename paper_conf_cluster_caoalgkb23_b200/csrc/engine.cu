@@ -1321,6 +1321,41 @@ mp_status mp_loglik(mp_handle* h, const mp_matrix* Lc, const double* d_z, double
     return MP_OK;
 }
 
+mp_status mp_gp_sample(mp_handle* h, const mp_matrix* Lc, const double* d_e, double* d_z) {
+    mp_matrix* A = const_cast<mp_matrix*>(Lc);
+    if (!h || !A || !d_e || !d_z) return MP_ERR_ARG;
+    if (!A->factored) FAIL(h, MP_ERR_STATE, "matrix not factored");
+    if (h->nranks > 1) FAIL(h, MP_ERR_UNSUPPORTED, "mp_gp_sample is single-rank");
+    const int nt = A->nt, nb = A->nb;
+    const int64_t n = A->n;
+    double* r = A->at<double>(A->R.vec_r);
+    double* ye = A->at<double>(A->R.vec_y);
+    CK(h, cudaMemsetAsync(r, 0, (size_t)nt * nb * 8, h->stream));
+    CK(h, cudaMemsetAsync(ye, 0, (size_t)nt * nb * 8, h->stream));
+    CK(h, cudaMemcpyAsync(ye, d_e, (size_t)n * 8, cudaMemcpyDeviceToDevice, h->stream));
+    Arena ar;
+    ar.dev_base = A->ws + A->R.ctrl;
+    std::vector<Op> ops;
+    // the GEMV kernel accumulates r_m -= L_mk e_k, i.e. r = -L e; the sign is flipped on the way out
+    for (int k = 0; k < nt; ++k) {
+        std::vector<GemvTile> gv;
+        for (int m = k; m < nt; ++m) gv.push_back(GemvTile{A->tile(m, k), A->st(m, k), 0, r + (size_t)m * nb});
+        GemvTile* dg = ar.push(gv);
+        const int ng = (int)gv.size();
+        const double* yk = ye + (size_t)k * nb;
+        ops.push_back({[=](cudaStream_t s) { return gemv_sub_launch(dg, ng, yk, nb, s); }, C_SOLVE, 0});
+    }
+    if (mp_status st = run_plan(h, A, ar, ops)) return st;
+    // r = -(L e): copy out negated
+    std::vector<double> tmp(n);
+    CK(h, cudaMemcpyAsync(tmp.data(), r, (size_t)n * 8, cudaMemcpyDeviceToHost, h->stream));
+    CK(h, cudaStreamSynchronize(h->stream));
+    for (auto& v : tmp) v = -v;
+    CK(h, cudaMemcpyAsync(d_z, tmp.data(), (size_t)n * 8, cudaMemcpyHostToDevice, h->stream));
+    CK(h, cudaStreamSynchronize(h->stream));
+    return MP_OK;
+}
+
 // ------------------------------------------------------------------ one evaluation
 static void band_kernel_map(int nt, const double* s, double u_req, const double* eps, std::vector<uint8_t>& km) {
     // reading C21: two-level rule, then the narrowest band holding every FP64 tile

@@ -278,3 +278,20 @@ def test_general_nu_tabulated_generation_vs_mpmath(mp, handle, nu):
             ref = float(mpmath.mpf(theta[0]) * 2 ** (1 - mpmath.mpf(nu)) / mpmath.gamma(nu) * r**nu
                         * mpmath.besselk(nu, r))
             assert abs(t[i, j] - ref) <= (4e-15 + float(r) * 2.0**-52) * abs(ref) + 1e-300, (nu, m, k, i, j, t[i, j], ref)
+
+
+def test_gp_sample_matches_dense_factor(mp, handle):
+    """mp_gp_sample: z = L e with the library's factor equals the dense Cholesky factor times e."""
+    n, nb, theta = 1500, 256, (1.0, 0.1, 0.5)
+    x, y = synth.uniform_locations(n, 2)
+    e = synth.normal_vector(n, 3)
+    M = mp.Matrix(handle, n, nb, None)
+    km, sm, cm = all_fp64_maps(M.nt)
+    M.matern_gen(to_dev(x), to_dev(y), theta, sm)
+    assert M.potrf(km, cm) == 0
+    import torch
+    dz = torch.zeros(n, dtype=torch.float64, device="cuda")
+    M.gp_sample(to_dev(e), dz)
+    from oracle.tiles import dense_covariance
+    ref = np.linalg.cholesky(dense_covariance(x, y, theta)) @ e
+    assert np.max(np.abs(dz.cpu().numpy() - ref)) <= 1e-12 * np.max(np.abs(ref))
