@@ -11,8 +11,8 @@
 //   warps 4-7        epilogue: tcgen05.ld 32x32b (warp w reads TMEM lanes 32(w%4)..+31 = its rows),
 //                    C -= acc with 16-byte loads/stores of the row.
 // KIND 0 (FP16 class, "FP16_32"): kind::f16, BN = 256, BK = 64, 4 stages (48 KB each).
-// KIND 1 (FP32 class, 3xTF32, reading C13): kind::tf32, BN = 128, BK = 32, 3 stages of
-//   {A_hi, A_lo, B_hi, B_lo} (64 KB); per k-step three MMAs lo.hi + hi.lo + hi.hi; K is split in
+// KIND 1 (FP32 class, 3xTF32, reading C13): kind::tf32, BN = 256, BK = 32, 2 stages of
+//   {A_hi, A_lo, B_hi, B_lo} (96 KB), 8 epilogue warps; per k-step three MMAs lo.hi + hi.lo + hi.hi; K is split in
 //   chunks of 64 accumulated in two ping-pong TMEM accumulators and summed by the epilogue in FP32.
 #include <cudaTypedefs.h>
 #include <stdint.h>
@@ -23,7 +23,11 @@
 namespace mpgeo {
 
 constexpr int TC_BM = 128;
-constexpr int TC_THREADS = 256;
+template <int KIND>
+struct TcThreads {
+    static constexpr int EPI_WARPS = KIND == 0 ? 4 : 8;  // 3xTF32: two warpgroups, one per 128-column half
+    static constexpr int N = (4 + EPI_WARPS) * 32;
+};
 
 struct __align__(64) TcParams {
     CUtensorMap a, b, a_lo, b_lo;
@@ -33,14 +37,14 @@ struct __align__(64) TcParams {
 
 template <int KIND>
 struct TcCfg {
-    static constexpr int BN = KIND == 0 ? 256 : 128;
+    static constexpr int BN = 256;
     static constexpr int ESZ = KIND == 0 ? 2 : 4;
     static constexpr int BK = 128 / ESZ;          // elements per 128-byte row
     static constexpr int UK = KIND == 0 ? 16 : 8;  // K per tcgen05.mma (32 bytes)
     static constexpr int A_BYTES = TC_BM * 128;
     static constexpr int B_BYTES = BN * 128;
     static constexpr int STAGE_BYTES = KIND == 0 ? A_BYTES + B_BYTES : 2 * (A_BYTES + B_BYTES);
-    static constexpr int STAGES = KIND == 0 ? 4 : 3;
+    static constexpr int STAGES = KIND == 0 ? 4 : 2;
     static constexpr int SMEM = STAGES * STAGE_BYTES + 1024;
     // KIND 1: accumulate CHUNK_KB k-blocks (64 of K) per TMEM accumulator, two accumulators
     // ping-pong; the epilogue sums the chunks in FP32 registers (round-to-nearest), which keeps
@@ -121,7 +125,7 @@ __device__ __forceinline__ void tmem_ld32(uint32_t taddr, uint32_t (&r)[32]) {
 }
 
 template <int KIND>
-__global__ void __launch_bounds__(TC_THREADS, 1) tc_gemm_kernel(const __grid_constant__ TcParams p) {
+__global__ void __launch_bounds__(TcThreads<KIND>::N, 1) tc_gemm_kernel(const __grid_constant__ TcParams p) {
     using Cfg = TcCfg<KIND>;
     extern __shared__ uint8_t smem_raw[];
     uint8_t* smem = (uint8_t*)(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
@@ -146,7 +150,7 @@ __global__ void __launch_bounds__(TC_THREADS, 1) tc_gemm_kernel(const __grid_con
         mbar_init(smem_u32(&done_bar), 1);
         for (int i = 0; i < 2; ++i) {
             mbar_init(smem_u32(&acc_full[i]), 1);
-            mbar_init(smem_u32(&acc_empty[i]), 4);  // one arrive per epilogue warp
+            mbar_init(smem_u32(&acc_empty[i]), TcThreads<KIND>::EPI_WARPS);  // one arrive per epilogue warp
         }
         asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
         asm volatile("prefetch.tensormap [%0];" ::"l"((uint64_t)&p.a) : "memory");
@@ -219,16 +223,19 @@ __global__ void __launch_bounds__(TC_THREADS, 1) tc_gemm_kernel(const __grid_con
         }
         if (KIND == 0) tc_commit(smem_u32(&done_bar));
     } else if (warp >= 4) {
-        // ---------------- epilogue: C -= acc
-        const int q = warp - 4;
+        // ---------------- epilogue: C -= acc.  Warp w reads TMEM lanes 32 (w % 4) .. +31 (its rows);
+        // with 8 epilogue warps the two warpgroups split the columns in halves.
+        constexpr int COLS = Cfg::BN / (TcThreads<KIND>::EPI_WARPS / 4);
+        const int q = (warp - 4) & 3;
+        const int half = (warp - 4) >> 2;
         const int row = bi * TC_BM + q * 32 + lane;
-        float* crow = jb.C + (size_t)row * p.nb + bj * Cfg::BN;
-        const uint32_t tl = (uint32_t)(q * 32) << 16;
+        float* crow = jb.C + (size_t)row * p.nb + bj * Cfg::BN + half * COLS;
+        const uint32_t tl = ((uint32_t)(q * 32) << 16) + (uint32_t)(half * COLS);
         if (KIND == 0) {
             mbar_wait(smem_u32(&done_bar), 0);
             tc_fence_after();
 #pragma unroll 1
-            for (int c0 = 0; c0 < Cfg::BN; c0 += 32) {
+            for (int c0 = 0; c0 < COLS; c0 += 32) {
                 uint32_t r[32];
                 tmem_ld32(tmem + tl + (uint32_t)c0, r);
                 float4* cp = (float4*)(crow + c0);
@@ -243,9 +250,9 @@ __global__ void __launch_bounds__(TC_THREADS, 1) tc_gemm_kernel(const __grid_con
                 }
             }
         } else {
-            float sum[Cfg::BN];
+            float sum[COLS];
 #pragma unroll
-            for (int i = 0; i < Cfg::BN; ++i) sum[i] = 0.f;
+            for (int i = 0; i < COLS; ++i) sum[i] = 0.f;
             const int nchunks = (KB + Cfg::CHUNK_KB - 1) / Cfg::CHUNK_KB;
 #pragma unroll 1
             for (int c = 0; c < nchunks; ++c) {
@@ -253,7 +260,7 @@ __global__ void __launch_bounds__(TC_THREADS, 1) tc_gemm_kernel(const __grid_con
                 mbar_wait(smem_u32(&acc_full[abuf]), (uint32_t)(c >> 1) & 1u);
                 tc_fence_after();
 #pragma unroll
-                for (int c0 = 0; c0 < Cfg::BN; c0 += 32) {
+                for (int c0 = 0; c0 < COLS; c0 += 32) {
                     uint32_t r[32];
                     tmem_ld32(tmem + tl + abuf * Cfg::BN + (uint32_t)c0, r);
 #pragma unroll
@@ -264,7 +271,7 @@ __global__ void __launch_bounds__(TC_THREADS, 1) tc_gemm_kernel(const __grid_con
                 if (lane == 0) asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(&acc_empty[abuf])) : "memory");
             }
 #pragma unroll
-            for (int c0 = 0; c0 < Cfg::BN; c0 += 4) {
+            for (int c0 = 0; c0 < COLS; c0 += 4) {
                 float4* cp = (float4*)(crow + c0);
                 float4 cv = *cp;
                 cv.x -= sum[c0];
@@ -343,7 +350,7 @@ static cudaError_t launch(const TcArgs& a, int njobs, cudaStream_t s) {
     p.tiles_per_job = (a.nb / TC_BM) * p.tiles_n;
     const long long grid = (long long)njobs * p.tiles_per_job;
     if (grid > 0x7fffffffLL) return cudaErrorInvalidConfiguration;
-    tc_gemm_kernel<KIND><<<(unsigned)grid, TC_THREADS, Cfg::SMEM, s>>>(p);
+    tc_gemm_kernel<KIND><<<(unsigned)grid, TcThreads<KIND>::N, Cfg::SMEM, s>>>(p);
     return cudaGetLastError();
 }
 
