@@ -68,6 +68,7 @@ struct Regions {
            wdiag = 0, mtab = 0;
     size_t vec_r = 0, vec_y = 0, partials = 0, norms = 0, ctrl = 0, ctrl_bytes = 0;
     std::vector<size_t> tile_off;  // per (m*nt+k), SIZE_MAX if not stored here
+    size_t pool = 0;               // start of the tile pool
 };
 
 // Peer-memory exchange area of one matrix (multi-GPU only; cudaMalloc'ed by the library so it
@@ -173,6 +174,7 @@ static Regions layout(const mp_matrix* A, const uint8_t* storage) {
     R.oz = take(2 * (size_t)nt * nb2 * 8);         // Ozaki int8 slice planes (S <= 8), two sets
     R.ozexp = take(2 * (size_t)nt * A->nb * 4);    // per-row exponents
     R.tile_off.assign((size_t)nt * nt, SIZE_MAX);
+    R.pool = align_up(off, 256);  // tile pool start (tile offsets from here are whole nb-float rows when 256 | nb)
     for (int k = 0; k < nt; ++k)
         for (int m = k; m < nt; ++m)
             if (A->mine(m, k)) {
@@ -696,6 +698,8 @@ static mp_status plan_potrf(mp_handle* h, mp_matrix* A, const uint8_t* km, const
     double* wb2 = A->at<double>(A->R.wbuf2);
     int* d_info = h->d_info;
     const bool use_tc = h->tc_mode != 0 && tc_gemm_available() && nb % 256 == 0;
+    const float* const cpool = A->at<float>(A->R.pool);                // tcgen05 epilogue C map range
+    const uint64_t crows = (A->R.total - A->R.pool) / ((size_t)nb * 4);
     const int ozS = h->ozaki == 8 && ozaki_available() && nb % 128 == 0 ? 8 : 0;
     const bool oz32 = ozS && h->ozaki32 && nb % 256 == 0;
     int8_t* const ozb = A->at<int8_t>(A->R.oz);
@@ -1037,6 +1041,8 @@ static mp_status plan_potrf(mp_handle* h, mp_matrix* A, const uint8_t* km, const
             TcJob* dj = ar.push(t32);
             const int nj = (int)t32.size();
             TcArgs ta{dj, phi, plo, nb, nt};
+            ta.cbase = cpool;
+            ta.crows = crows;
             cur->push_back({[=](cudaStream_t s) { return tc_gemm_tf32x3_launch(ta, nj, s); }, C_UPD32, 2 * f3 * nj});
         }
         if (!t16.empty()) {
@@ -1044,6 +1050,8 @@ static mp_status plan_potrf(mp_handle* h, mp_matrix* A, const uint8_t* km, const
             const int nj = (int)t16.size();
             TcArgs ta{dj, nullptr, nullptr, nb, nt};
             ta.p16 = p16;
+            ta.cbase = cpool;
+            ta.crows = crows;
             cur->push_back({[=](cudaStream_t s) { return tc_gemm_f16_launch(ta, nj, s); }, C_UPD16, 2 * f3 * nj});
         }
         }  // part

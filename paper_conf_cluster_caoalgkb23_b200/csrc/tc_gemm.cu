@@ -2,27 +2,31 @@
 //
 //   C_mn (FP32, nb x nb, row-major)  -=  P_m P_n^T        P = panel operand cache [nt*nb][nb]
 //
-// One CTA computes a 128 x BN block of C over the full K = nb:
-//   warp 0 (1 lane)  TMA producer: 128-byte-swizzled K-major boxes into a STAGES-deep ring
-//                    guarded by full/empty mbarriers;
-//   warp 1 (1 lane)  MMA issuer: tcgen05.mma.cta_group::1 (M = 128, N = BN), accumulator in TMEM,
-//                    tcgen05.commit releases each stage back to the producer;
-//   warp 2           TMEM allocator (BN FP32 columns);
-//   warps 4-7        epilogue: tcgen05.ld 32x32b (warp w reads TMEM lanes 32(w%4)..+31 = its rows),
-//                    C -= acc with 16-byte loads/stores of the row.
-// KIND 0 (FP16 class, "FP16_32"): kind::f16, BN = 256, BK = 64, 4 stages (48 KB each).
-// KIND 1 (FP32 class, 3xTF32, reading C13): kind::tf32, BN = 256, BK = 32, 2 stages of
-//   {A_hi, A_lo, B_hi, B_lo} (96 KB), 8 epilogue warps; per k-step three MMAs lo.hi + hi.lo + hi.hi; K is split in
-//   chunks of 64 accumulated in two ping-pong TMEM accumulators and summed by the epilogue in FP32.
+// A CTA pair (cluster of 2 on one TPC, tcgen05.mma.cta_group::2, M = 256) computes a 256 x 256
+// block of C over the full K = nb (CL = 1: one CTA, M = 128, 128 x 256):
+//   warp 0 (1 lane)  TMA producer: 128-byte-swizzled K-major boxes into a multi-stage ring guarded
+//                    by full/empty mbarriers; each CTA loads its 128 rows of A and its half of B,
+//                    the bytes of both CTAs complete on the leader's full barrier;
+//   warp 1 (1 lane)  MMA issuer (leader CTA only): accumulator in TMEM, tcgen05.commit (multicast
+//                    to both CTAs) releases each stage and publishes finished accumulators;
+//   warp 2           TMEM allocator;
+//   warps 4-..       epilogue: tcgen05.ld 32x32b (warp w reads TMEM lanes 32(w%4)..+31 = its rows),
+//                    -acc staged in shared memory (128-byte swizzle) and reduced into C with
+//                    cp.reduce.async.bulk.tensor .add (one add per element: RN(C - acc)).
+// KIND 0 (FP16 class, "FP16_32"): kind::f16, BK = 64, 96 KB of stages so two CTAs share an SM.
+// KIND 1 (FP32 class, 3xTF32, reading C13): kind::tf32, BK = 32, stages of {A_hi, A_lo, B_hi, B_lo},
+//   8 epilogue warps; per k-step three MMAs lo.hi + hi.lo + hi.hi; K is split in chunks of 64
+//   accumulated in two ping-pong TMEM accumulators and summed by the epilogue in FP32.
 #include <cudaTypedefs.h>
 #include <stdint.h>
+#include <stdlib.h>
 #include <string.h>
 
 #include "tc_gemm.h"
 
 namespace mpgeo {
 
-constexpr int TC_BM = 128;
+constexpr int TC_BM = 128;  // output rows per CTA (TMEM lanes)
 template <int KIND>
 struct TcThreads {
     static constexpr int EPI_WARPS = KIND == 0 ? 4 : 8;  // 3xTF32: two warpgroups, one per 128-column half
@@ -30,21 +34,30 @@ struct TcThreads {
 };
 
 struct __align__(64) TcParams {
-    CUtensorMap a, b, a_lo, b_lo;
+    CUtensorMap a, b, a_lo, b_lo, c;
     const TcJob* jobs;
+    const float* cbase;
     int nb, tiles_n, tiles_per_job;
 };
 
-template <int KIND>
+// CL = CTAs per MMA: 1 (tcgen05.mma.cta_group::1, M = 128) or 2 (a CTA pair on one TPC,
+// cta_group::2, M = 256).  In a pair each CTA loads its own 128 rows of A and half (BN / 2 rows) of
+// B; the MMA reads B from both CTAs' shared memory, so every byte fetched from L2 feeds twice the
+// flops (the single-CTA kernel is bound by L2 -> SM bandwidth, profiles/r01).
+template <int KIND, int CL>
 struct TcCfg {
-    static constexpr int BN = 256;
+    static constexpr int BN = 256;                 // MMA N = output columns per CTA
+    static constexpr int BM = TC_BM * CL;          // MMA M = output rows per cluster
     static constexpr int ESZ = KIND == 0 ? 2 : 4;
-    static constexpr int BK = 128 / ESZ;          // elements per 128-byte row
+    static constexpr int BK = 128 / ESZ;           // elements per 128-byte row
     static constexpr int UK = KIND == 0 ? 16 : 8;  // K per tcgen05.mma (32 bytes)
     static constexpr int A_BYTES = TC_BM * 128;
-    static constexpr int B_BYTES = BN * 128;
+    static constexpr int B_BYTES = (BN / CL) * 128;
     static constexpr int STAGE_BYTES = KIND == 0 ? A_BYTES + B_BYTES : 2 * (A_BYTES + B_BYTES);
-    static constexpr int STAGES = KIND == 0 ? 4 : 2;
+    // KIND 0: 96 KB of stages so two CTAs share an SM (one's epilogue overlaps the other's main
+    // loop; 2 x 256 TMEM columns); KIND 1: 192 KB, one CTA per SM (512 TMEM columns)
+    static constexpr int STAGES = (KIND == 0 ? 96 * 1024 : 192 * 1024) / STAGE_BYTES;
+    static constexpr int MIN_BLOCKS = KIND == 0 ? 2 : 1;
     static constexpr int SMEM = STAGES * STAGE_BYTES + 1024;
     // KIND 1: accumulate CHUNK_KB k-blocks (64 of K) per TMEM accumulator, two accumulators
     // ping-pong; the epilogue sums the chunks in FP32 registers (round-to-nearest), which keeps
@@ -54,7 +67,7 @@ struct TcCfg {
     // instruction descriptor: D = F32 (bit 4), A/B format (bits 7-9 / 10-12), K-major both,
     // N >> 3 (bits 17-22), M >> 4 (bits 24-28)
     static constexpr uint32_t IDESC = (1u << 4) | ((KIND == 0 ? 0u : 2u) << 7) | ((KIND == 0 ? 0u : 2u) << 10) |
-                                      ((uint32_t)(BN >> 3) << 17) | ((uint32_t)(TC_BM >> 4) << 24);
+                                      ((uint32_t)(BN >> 3) << 17) | ((uint32_t)(BM >> 4) << 24);
 };
 
 __device__ __forceinline__ uint32_t smem_u32(const void* p) { return (uint32_t)__cvta_generic_to_shared(p); }
@@ -74,16 +87,50 @@ __device__ __forceinline__ void mbar_wait(uint32_t bar, uint32_t parity) {
         "r"(parity)
         : "memory");
 }
+// shared::cluster address of the same shared variable in CTA `rank` of the cluster
+__device__ __forceinline__ uint32_t cluster_addr(uint32_t saddr, uint32_t rank) {
+    uint32_t r;
+    asm volatile("mapa.shared::cluster.u32 %0, %1, %2;" : "=r"(r) : "r"(saddr), "r"(rank));
+    return r;
+}
+__device__ __forceinline__ void mbar_arrive_cluster(uint32_t cbar) {
+    asm volatile("mbarrier.arrive.release.cluster.shared::cluster.b64 _, [%0];" ::"r"(cbar) : "memory");
+}
+__device__ __forceinline__ uint32_t cluster_rank() {
+    uint32_t r;
+    asm volatile("mov.u32 %0, %%cluster_ctarank;" : "=r"(r));
+    return r;
+}
+__device__ __forceinline__ void cluster_sync() {
+    asm volatile("barrier.cluster.arrive.release.aligned;\n\tbarrier.cluster.wait.acquire.aligned;" ::: "memory");
+}
+// TMA 2D load into this CTA's shared memory; with CL = 2 the completion is signalled on the
+// leader CTA's mbarrier (cta_group::2 form), which the leader's MMA issuer waits on.
+template <int CL>
 __device__ __forceinline__ void tma_load_2d(uint32_t dst, const CUtensorMap* map, uint32_t bar, int c0, int c1) {
-    asm volatile(
-        "cp.async.bulk.tensor.2d.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1, {%3, %4}], [%2];" ::"r"(dst),
-        "l"((uint64_t)map), "r"(bar), "r"(c0), "r"(c1)
-        : "memory");
+    if (CL == 1)
+        asm volatile(
+            "cp.async.bulk.tensor.2d.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1, {%3, %4}], [%2];" ::"r"(dst),
+            "l"((uint64_t)map), "r"(bar), "r"(c0), "r"(c1)
+            : "memory");
+    else
+        asm volatile(
+            "cp.async.bulk.tensor.2d.cta_group::2.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1, {%3, %4}], [%2];" ::"r"(dst),
+            "l"((uint64_t)map), "r"(bar), "r"(c0), "r"(c1)
+            : "memory");
 }
 __device__ __forceinline__ void tc_fence_before() { asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory"); }
 __device__ __forceinline__ void tc_fence_after() { asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory"); }
+// MMA-completion arrive: CL = 1 on this CTA's barrier; CL = 2 on the barrier at the same offset in
+// both CTAs of the pair
+template <int CL>
 __device__ __forceinline__ void tc_commit(uint32_t bar) {
-    asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];" ::"r"(bar) : "memory");
+    if (CL == 1)
+        asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];" ::"r"(bar) : "memory");
+    else
+        asm volatile("tcgen05.commit.cta_group::2.mbarrier::arrive::one.shared::cluster.multicast::cluster.b64 [%0], %1;" ::"r"(bar),
+                     "h"((uint16_t)3)
+                     : "memory");
 }
 
 // K-major operand, 128-byte swizzle: 8-row x 128-byte atoms stacked every 1024 bytes (SBO),
@@ -97,19 +144,29 @@ __device__ __forceinline__ uint64_t desc_sw128(uint32_t saddr) {
     return d;
 }
 
-template <int KIND>
+template <int KIND, int CL>
 __device__ __forceinline__ void tc_mma(uint32_t tmem, uint64_t a, uint64_t b, uint32_t accum) {
-    if (KIND == 0) {
+    constexpr uint32_t ID = TcCfg<KIND, CL>::IDESC;
+    if (KIND == 0 && CL == 1)
         asm volatile(
             "{\n\t.reg .pred p;\n\tsetp.ne.b32 p, %4, 0;\n\t"
             "tcgen05.mma.cta_group::1.kind::f16 [%0], %1, %2, %3, p;\n\t}" ::"r"(tmem),
-            "l"(a), "l"(b), "r"(TcCfg<KIND>::IDESC), "r"(accum));
-    } else {
+            "l"(a), "l"(b), "r"(ID), "r"(accum));
+    else if (KIND == 0)
+        asm volatile(
+            "{\n\t.reg .pred p;\n\tsetp.ne.b32 p, %4, 0;\n\t"
+            "tcgen05.mma.cta_group::2.kind::f16 [%0], %1, %2, %3, p;\n\t}" ::"r"(tmem),
+            "l"(a), "l"(b), "r"(ID), "r"(accum));
+    else if (CL == 1)
         asm volatile(
             "{\n\t.reg .pred p;\n\tsetp.ne.b32 p, %4, 0;\n\t"
             "tcgen05.mma.cta_group::1.kind::tf32 [%0], %1, %2, %3, p;\n\t}" ::"r"(tmem),
-            "l"(a), "l"(b), "r"(TcCfg<KIND>::IDESC), "r"(accum));
-    }
+            "l"(a), "l"(b), "r"(ID), "r"(accum));
+    else
+        asm volatile(
+            "{\n\t.reg .pred p;\n\tsetp.ne.b32 p, %4, 0;\n\t"
+            "tcgen05.mma.cta_group::2.kind::tf32 [%0], %1, %2, %3, p;\n\t}" ::"r"(tmem),
+            "l"(a), "l"(b), "r"(ID), "r"(accum));
 }
 
 __device__ __forceinline__ void tmem_ld32(uint32_t taddr, uint32_t (&r)[32]) {
@@ -124,9 +181,53 @@ __device__ __forceinline__ void tmem_ld32(uint32_t taddr, uint32_t (&r)[32]) {
     asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
 }
 
-template <int KIND>
-__global__ void __launch_bounds__(TcThreads<KIND>::N, 1) tc_gemm_kernel(const __grid_constant__ TcParams p) {
-    using Cfg = TcCfg<KIND>;
+// C -= acc through the TMA unit: the warp stages -acc for a 32 x 32 box in shared memory
+// (128-byte swizzle: 16-byte chunk j of row r at chunk j ^ (r & 7), conflict-free for the
+// row-per-lane writes) and one lane issues a bulk tensor reduce-add into global C.  Each element
+// of C receives exactly one add, so the result is RN(C - acc), as with a load / subtract / store.
+__device__ __forceinline__ void stage_box_neg(uint32_t buf, int lane, const float* v) {
+#pragma unroll
+    for (int j = 0; j < 8; ++j) {
+        const uint32_t a = buf + (uint32_t)lane * 128u + ((uint32_t)(j ^ (lane & 7)) << 4);
+        asm volatile("st.shared.v4.f32 [%0], {%1, %2, %3, %4};" ::"r"(a), "f"(-v[4 * j]), "f"(-v[4 * j + 1]),
+                     "f"(-v[4 * j + 2]), "f"(-v[4 * j + 3])
+                     : "memory");
+    }
+    asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+    __syncwarp();
+}
+__device__ __forceinline__ void tma_reduce_add(const CUtensorMap* map, uint32_t buf, int c0, int c1) {
+    asm volatile("cp.reduce.async.bulk.tensor.2d.global.shared::cta.add.tile.bulk_group [%0, {%2, %3}], [%1];" ::"l"(
+                     (uint64_t)map),
+                 "r"(buf), "r"(c0), "r"(c1)
+                 : "memory");
+    asm volatile("cp.async.bulk.commit_group;" ::: "memory");
+}
+__device__ __forceinline__ void bulk_wait_read_1() { asm volatile("cp.async.bulk.wait_group.read 1;" ::: "memory"); }
+__device__ __forceinline__ void bulk_wait_all() { asm volatile("cp.async.bulk.wait_group 0;" ::: "memory"); }
+
+template <int CL>
+__device__ __forceinline__ void tmem_alloc(uint32_t slot, uint32_t cols) {
+    if (CL == 1) {
+        asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(slot), "r"(cols) : "memory");
+        asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;" ::: "memory");
+    } else {
+        asm volatile("tcgen05.alloc.cta_group::2.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(slot), "r"(cols) : "memory");
+        asm volatile("tcgen05.relinquish_alloc_permit.cta_group::2.sync.aligned;" ::: "memory");
+    }
+}
+template <int CL>
+__device__ __forceinline__ void tmem_dealloc(uint32_t tmem, uint32_t cols) {
+    if (CL == 1)
+        asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem), "r"(cols) : "memory");
+    else
+        asm volatile("tcgen05.dealloc.cta_group::2.sync.aligned.b32 %0, %1;" ::"r"(tmem), "r"(cols) : "memory");
+}
+
+template <int KIND, int CL>
+__global__ void __launch_bounds__(TcThreads<KIND>::N, TcCfg<KIND, CL>::MIN_BLOCKS) tc_gemm_kernel(const __grid_constant__ TcParams p) {
+    using Cfg = TcCfg<KIND, CL>;
+    constexpr int EPI_WARPS = TcThreads<KIND>::EPI_WARPS;
     extern __shared__ uint8_t smem_raw[];
     uint8_t* smem = (uint8_t*)(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
     __shared__ __align__(8) uint64_t full_bar[Cfg::STAGES], empty_bar[Cfg::STAGES], done_bar;
@@ -134,68 +235,67 @@ __global__ void __launch_bounds__(TcThreads<KIND>::N, 1) tc_gemm_kernel(const __
     __shared__ uint32_t tmem_slot;
 
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-    const int job = blockIdx.x / p.tiles_per_job;
-    const int t = blockIdx.x - job * p.tiles_per_job;
+    const uint32_t crank = CL > 1 ? cluster_rank() : 0;
+    const int cta = blockIdx.x / CL;  // output block (one per CTA pair when CL = 2)
+    const int job = cta / p.tiles_per_job;
+    const int t = cta - job * p.tiles_per_job;
     const int bi = t / p.tiles_n, bj = t - bi * p.tiles_n;
     const TcJob jb = p.jobs[job];
-    const int rowA = jb.m * p.nb + bi * TC_BM;
-    const int rowB = jb.n * p.nb + bj * Cfg::BN;
+    const int rowA = jb.m * p.nb + bi * Cfg::BM + (int)crank * TC_BM;
+    const int rowB = jb.n * p.nb + bj * Cfg::BN + (int)crank * (Cfg::BN / CL);
     const int KB = p.nb / Cfg::BK;
 
     if (threadIdx.x == 0) {
         for (int s = 0; s < Cfg::STAGES; ++s) {
-            mbar_init(smem_u32(&full_bar[s]), 1);
-            mbar_init(smem_u32(&empty_bar[s]), 1);
+            mbar_init(smem_u32(&full_bar[s]), 1);   // leader: its producer's arrive + both CTAs' bytes
+            mbar_init(smem_u32(&empty_bar[s]), 1);  // the leader's MMA commit
         }
         mbar_init(smem_u32(&done_bar), 1);
         for (int i = 0; i < 2; ++i) {
             mbar_init(smem_u32(&acc_full[i]), 1);
-            mbar_init(smem_u32(&acc_empty[i]), TcThreads<KIND>::EPI_WARPS);  // one arrive per epilogue warp
+            mbar_init(smem_u32(&acc_empty[i]), CL * EPI_WARPS);  // one arrive per epilogue warp of the pair
         }
         asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
         asm volatile("prefetch.tensormap [%0];" ::"l"((uint64_t)&p.a) : "memory");
         asm volatile("prefetch.tensormap [%0];" ::"l"((uint64_t)&p.b) : "memory");
     }
-    if (warp == 2) {
-        asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(smem_u32(&tmem_slot)),
-                     "r"(Cfg::TMEM_COLS)
-                     : "memory");
-        asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;" ::: "memory");
-    }
+    if (warp == 2) tmem_alloc<CL>(smem_u32(&tmem_slot), Cfg::TMEM_COLS);
     tc_fence_before();
-    __syncthreads();
+    if (CL > 1) cluster_sync();  // the peer's barriers exist before any remote arrive / multicast
+    else __syncthreads();
     tc_fence_after();
     const uint32_t tmem = tmem_slot;
 
     if (warp == 0 && lane == 0) {
-        // ---------------- TMA producer
+        // ---------------- TMA producer (every CTA loads its own A rows and its share of B)
         for (int kb = 0; kb < KB; ++kb) {
             const int s = kb % Cfg::STAGES;
             const uint32_t ph = (uint32_t)(kb / Cfg::STAGES) & 1u;
             mbar_wait(smem_u32(&empty_bar[s]), ph ^ 1u);
             const uint32_t st = smem_u32(smem + s * Cfg::STAGE_BYTES);
-            const uint32_t fb = smem_u32(&full_bar[s]);
-            mbar_expect_tx(fb, Cfg::STAGE_BYTES);
+            const uint32_t lb = smem_u32(&full_bar[s]);
+            const uint32_t fb = CL > 1 ? cluster_addr(lb, 0) : lb;
+            if (crank == 0) mbar_expect_tx(lb, CL * Cfg::STAGE_BYTES);
             const int kc = kb * Cfg::BK;
             if (KIND == 0) {
-                tma_load_2d(st, &p.a, fb, kc, rowA);
-                tma_load_2d(st + Cfg::A_BYTES, &p.b, fb, kc, rowB);
+                tma_load_2d<CL>(st, &p.a, fb, kc, rowA);
+                tma_load_2d<CL>(st + Cfg::A_BYTES, &p.b, fb, kc, rowB);
             } else {
-                tma_load_2d(st, &p.a, fb, kc, rowA);
-                tma_load_2d(st + Cfg::A_BYTES, &p.a_lo, fb, kc, rowA);
-                tma_load_2d(st + 2 * Cfg::A_BYTES, &p.b, fb, kc, rowB);
-                tma_load_2d(st + 2 * Cfg::A_BYTES + Cfg::B_BYTES, &p.b_lo, fb, kc, rowB);
+                tma_load_2d<CL>(st, &p.a, fb, kc, rowA);
+                tma_load_2d<CL>(st + Cfg::A_BYTES, &p.a_lo, fb, kc, rowA);
+                tma_load_2d<CL>(st + 2 * Cfg::A_BYTES, &p.b, fb, kc, rowB);
+                tma_load_2d<CL>(st + 2 * Cfg::A_BYTES + Cfg::B_BYTES, &p.b_lo, fb, kc, rowB);
             }
         }
-    } else if (warp == 1 && lane == 0) {
-        // ---------------- MMA issuer
+    } else if (warp == 1 && lane == 0 && crank == 0) {
+        // ---------------- MMA issuer (the leader CTA issues for the pair)
         for (int kb = 0; kb < KB; ++kb) {
             const int s = kb % Cfg::STAGES;
             const uint32_t ph = (uint32_t)(kb / Cfg::STAGES) & 1u;
             const int chunk = kb / Cfg::CHUNK_KB, kin = kb % Cfg::CHUNK_KB;
             const uint32_t abuf = (uint32_t)(chunk & 1);
             const uint32_t dacc = KIND == 0 ? tmem : tmem + abuf * Cfg::BN;
-            if (KIND == 1 && kin == 0) {  // wait until the epilogue drained this accumulator
+            if (KIND == 1 && kin == 0) {  // wait until the epilogues drained this accumulator
                 mbar_wait(smem_u32(&acc_empty[abuf]), ((uint32_t)(chunk >> 1) & 1u) ^ 1u);
                 tc_fence_after();
             }
@@ -207,53 +307,56 @@ __global__ void __launch_bounds__(TcThreads<KIND>::N, 1) tc_gemm_kernel(const __
                 const uint32_t koff = k * 32;  // bytes along K inside the 128-byte swizzle atom
                 const uint32_t acc = (kin | k) != 0;
                 if (KIND == 0) {
-                    tc_mma<0>(dacc, desc_sw128(base + koff), desc_sw128(base + Cfg::A_BYTES + koff), acc);
+                    tc_mma<0, CL>(dacc, desc_sw128(base + koff), desc_sw128(base + Cfg::A_BYTES + koff), acc);
                 } else {
                     const uint64_t ahi = desc_sw128(base + koff);
                     const uint64_t alo = desc_sw128(base + Cfg::A_BYTES + koff);
                     const uint64_t bhi = desc_sw128(base + 2 * Cfg::A_BYTES + koff);
                     const uint64_t blo = desc_sw128(base + 2 * Cfg::A_BYTES + Cfg::B_BYTES + koff);
-                    tc_mma<1>(dacc, alo, bhi, acc);  // small terms first
-                    tc_mma<1>(dacc, ahi, blo, 1u);
-                    tc_mma<1>(dacc, ahi, bhi, 1u);
+                    tc_mma<1, CL>(dacc, alo, bhi, acc);  // small terms first
+                    tc_mma<1, CL>(dacc, ahi, blo, 1u);
+                    tc_mma<1, CL>(dacc, ahi, bhi, 1u);
                 }
             }
-            tc_commit(smem_u32(&empty_bar[s]));
-            if (KIND == 1 && (kin == Cfg::CHUNK_KB - 1 || kb == KB - 1)) tc_commit(smem_u32(&acc_full[abuf]));
+            tc_commit<CL>(smem_u32(&empty_bar[s]));
+            if (KIND == 1 && (kin == Cfg::CHUNK_KB - 1 || kb == KB - 1)) tc_commit<CL>(smem_u32(&acc_full[abuf]));
         }
-        if (KIND == 0) tc_commit(smem_u32(&done_bar));
+        if (KIND == 0) tc_commit<CL>(smem_u32(&done_bar));
     } else if (warp >= 4) {
         // ---------------- epilogue: C -= acc.  Warp w reads TMEM lanes 32 (w % 4) .. +31 (its rows);
-        // with 8 epilogue warps the two warpgroups split the columns in halves.
-        constexpr int COLS = Cfg::BN / (TcThreads<KIND>::EPI_WARPS / 4);
+        // with 8 epilogue warps the two warpgroups split the columns in halves.  The stage ring is
+        // idle once the last accumulator is complete, so it doubles as the staging buffer.
+        constexpr int COLS = Cfg::BN / (EPI_WARPS / 4);
         const int q = (warp - 4) & 3;
         const int half = (warp - 4) >> 2;
-        const int row = bi * TC_BM + q * 32 + lane;
-        float* crow = jb.C + (size_t)row * p.nb + bj * Cfg::BN + half * COLS;
+        const int crow0 = (int)((jb.C - p.cbase) / p.nb) + bi * Cfg::BM + (int)crank * TC_BM + q * 32;
+        const int ccol0 = bj * Cfg::BN + half * COLS;
         const uint32_t tl = ((uint32_t)(q * 32) << 16) + (uint32_t)(half * COLS);
+        const uint32_t stg = smem_u32(smem) + (uint32_t)(warp - 4) * 8192u;  // two 4 KB boxes per warp
         if (KIND == 0) {
             mbar_wait(smem_u32(&done_bar), 0);
             tc_fence_after();
 #pragma unroll 1
-            for (int c0 = 0; c0 < COLS; c0 += 32) {
+            for (int g = 0; g < COLS / 32; ++g) {
                 uint32_t r[32];
-                tmem_ld32(tmem + tl + (uint32_t)c0, r);
-                float4* cp = (float4*)(crow + c0);
-#pragma unroll
-                for (int v = 0; v < 8; ++v) {
-                    float4 c = cp[v];
-                    c.x -= __uint_as_float(r[4 * v + 0]);
-                    c.y -= __uint_as_float(r[4 * v + 1]);
-                    c.z -= __uint_as_float(r[4 * v + 2]);
-                    c.w -= __uint_as_float(r[4 * v + 3]);
-                    cp[v] = c;
+                tmem_ld32(tmem + tl + (uint32_t)(g * 32), r);
+                const uint32_t buf = stg + (uint32_t)(g & 1) * 4096u;
+                if (g >= 2) {
+                    if (lane == 0) bulk_wait_read_1();
+                    __syncwarp();
                 }
+                float v[32];
+#pragma unroll
+                for (int i = 0; i < 32; ++i) v[i] = __uint_as_float(r[i]);
+                stage_box_neg(buf, lane, v);
+                if (lane == 0) tma_reduce_add(&p.c, buf, ccol0 + g * 32, crow0);
             }
         } else {
             float sum[COLS];
 #pragma unroll
             for (int i = 0; i < COLS; ++i) sum[i] = 0.f;
             const int nchunks = (KB + Cfg::CHUNK_KB - 1) / Cfg::CHUNK_KB;
+            const uint32_t ae0 = CL > 1 ? cluster_addr(smem_u32(&acc_empty[0]), 0) : smem_u32(&acc_empty[0]);
 #pragma unroll 1
             for (int c = 0; c < nchunks; ++c) {
                 const uint32_t abuf = (uint32_t)(c & 1);
@@ -268,26 +371,32 @@ __global__ void __launch_bounds__(TcThreads<KIND>::N, 1) tc_gemm_kernel(const __
                 }
                 tc_fence_before();
                 __syncwarp();
-                if (lane == 0) asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(&acc_empty[abuf])) : "memory");
+                if (lane == 0) {
+                    if (CL > 1) mbar_arrive_cluster(ae0 + abuf * 8u);
+                    else asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(ae0 + abuf * 8u) : "memory");
+                }
             }
+            // the last acc_full also means every MMA (and so every shared-memory read of the ring,
+            // in both CTAs of a pair) has completed
 #pragma unroll
-            for (int c0 = 0; c0 < COLS; c0 += 4) {
-                float4* cp = (float4*)(crow + c0);
-                float4 cv = *cp;
-                cv.x -= sum[c0];
-                cv.y -= sum[c0 + 1];
-                cv.z -= sum[c0 + 2];
-                cv.w -= sum[c0 + 3];
-                *cp = cv;
+            for (int g = 0; g < COLS / 32; ++g) {
+                const uint32_t buf = stg + (uint32_t)(g & 1) * 4096u;
+                if (g >= 2) {
+                    if (lane == 0) bulk_wait_read_1();
+                    __syncwarp();
+                }
+                stage_box_neg(buf, lane, sum + g * 32);
+                if (lane == 0) tma_reduce_add(&p.c, buf, ccol0 + g * 32, crow0);
             }
         }
+        if (lane == 0) bulk_wait_all();
     }
     tc_fence_before();
-    __syncthreads();
+    if (CL > 1) cluster_sync();  // neither CTA frees TMEM / exits while its peer may still signal it
+    else __syncthreads();
     if (warp == 2) {
         tc_fence_after();
-        asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem), "r"(Cfg::TMEM_COLS)
-                     : "memory");
+        tmem_dealloc<CL>(tmem, Cfg::TMEM_COLS);
     }
 }
 
@@ -319,42 +428,70 @@ static bool make_map(CUtensorMap* m, const void* base, CUtensorMapDataType dt, i
 
 bool tc_gemm_available() { return encode_fn() != nullptr; }
 
-template <int KIND>
+template <int KIND, int CL>
 static cudaError_t launch(const TcArgs& a, int njobs, cudaStream_t s) {
-    using Cfg = TcCfg<KIND>;
+    using Cfg = TcCfg<KIND, CL>;
     if (njobs <= 0) return cudaSuccess;
-    if (a.nb % Cfg::BN || a.nb % TC_BM) return cudaErrorInvalidValue;
+    if (a.nb % Cfg::BN || a.nb % Cfg::BM) return cudaErrorInvalidValue;
     static bool attr = false;
     if (!attr) {
-        cudaError_t e = cudaFuncSetAttribute(tc_gemm_kernel<KIND>, cudaFuncAttributeMaxDynamicSharedMemorySize, Cfg::SMEM);
+        cudaError_t e = cudaFuncSetAttribute(tc_gemm_kernel<KIND, CL>, cudaFuncAttributeMaxDynamicSharedMemorySize, Cfg::SMEM);
         if (e != cudaSuccess) return e;
         attr = true;
     }
     TcParams p;
     memset(&p, 0, sizeof p);
     const uint64_t rows = (uint64_t)a.nt * a.nb;
+    constexpr uint32_t BROWS = Cfg::BN / CL;
     bool ok;
     if (KIND == 0) {
         ok = make_map(&p.a, a.p16, CU_TENSOR_MAP_DATA_TYPE_FLOAT16, 2, rows, a.nb, Cfg::BK, TC_BM) &&
-             make_map(&p.b, a.p16, CU_TENSOR_MAP_DATA_TYPE_FLOAT16, 2, rows, a.nb, Cfg::BK, Cfg::BN);
+             make_map(&p.b, a.p16, CU_TENSOR_MAP_DATA_TYPE_FLOAT16, 2, rows, a.nb, Cfg::BK, BROWS);
     } else {
         ok = make_map(&p.a, a.hi, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 4, rows, a.nb, Cfg::BK, TC_BM) &&
              make_map(&p.a_lo, a.lo, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 4, rows, a.nb, Cfg::BK, TC_BM) &&
-             make_map(&p.b, a.hi, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 4, rows, a.nb, Cfg::BK, Cfg::BN) &&
-             make_map(&p.b_lo, a.lo, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 4, rows, a.nb, Cfg::BK, Cfg::BN);
+             make_map(&p.b, a.hi, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 4, rows, a.nb, Cfg::BK, BROWS) &&
+             make_map(&p.b_lo, a.lo, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 4, rows, a.nb, Cfg::BK, BROWS);
     }
+    // C: FP32 rows of nb over [cbase, cbase + crows * nb), 32 x 32 boxes, 128-byte swizzle
+    ok = ok && a.cbase && make_map(&p.c, a.cbase, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 4, a.crows, a.nb, 32, 32);
     if (!ok) return cudaErrorInvalidValue;
     p.jobs = a.jobs;
+    p.cbase = a.cbase;
     p.nb = a.nb;
     p.tiles_n = a.nb / Cfg::BN;
-    p.tiles_per_job = (a.nb / TC_BM) * p.tiles_n;
-    const long long grid = (long long)njobs * p.tiles_per_job;
+    p.tiles_per_job = (a.nb / Cfg::BM) * p.tiles_n;
+    const long long grid = (long long)njobs * p.tiles_per_job * CL;
     if (grid > 0x7fffffffLL) return cudaErrorInvalidConfiguration;
-    tc_gemm_kernel<KIND><<<(unsigned)grid, TcThreads<KIND>::N, Cfg::SMEM, s>>>(p);
-    return cudaGetLastError();
+    cudaLaunchConfig_t cfg = {};
+    cfg.gridDim = dim3((unsigned)grid);
+    cfg.blockDim = dim3(TcThreads<KIND>::N);
+    cfg.dynamicSmemBytes = Cfg::SMEM;
+    cfg.stream = s;
+    cudaLaunchAttribute at[1];
+    at[0].id = cudaLaunchAttributeClusterDimension;
+    at[0].val.clusterDim.x = CL;
+    at[0].val.clusterDim.y = 1;
+    at[0].val.clusterDim.z = 1;
+    cfg.attrs = at;
+    cfg.numAttrs = 1;
+    return cudaLaunchKernelEx(&cfg, tc_gemm_kernel<KIND, CL>, p);
 }
 
-cudaError_t tc_gemm_f16_launch(const TcArgs& a, int njobs, cudaStream_t s) { return launch<0>(a, njobs, s); }
-cudaError_t tc_gemm_tf32x3_launch(const TcArgs& a, int njobs, cudaStream_t s) { return launch<1>(a, njobs, s); }
+// CTAs per MMA: MPGEO_TC_CLUSTER (3xTF32) and MPGEO_TC16_CLUSTER (FP16); default 2 = CTA pairs (faster
+// than single-CTA for both kinds, profiles/r01/README.md)
+static int env_cluster(const char* name, int dflt) {
+    const char* e = getenv(name);
+    return e ? (atoi(e) == 2 ? 2 : 1) : dflt;
+}
+
+cudaError_t tc_gemm_f16_launch(const TcArgs& a, int njobs, cudaStream_t s) {
+    static const int cl = env_cluster("MPGEO_TC16_CLUSTER", 2);
+    return cl == 2 ? launch<0, 2>(a, njobs, s) : launch<0, 1>(a, njobs, s);
+}
+cudaError_t tc_gemm_tf32x3_launch(const TcArgs& a, int njobs, cudaStream_t s) {
+    static const int cl = env_cluster("MPGEO_TC_CLUSTER", 2);
+    return cl == 2 ? launch<1, 2>(a, njobs, s) : launch<1, 1>(a, njobs, s);
+}
 
 }  // namespace mpgeo

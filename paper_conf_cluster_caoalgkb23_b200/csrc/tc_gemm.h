@@ -21,6 +21,10 @@ struct TcArgs {
     const float* lo;      // TF32 lo panel cache
     int nb, nt;
     const __half* p16;    // FP16 panel cache, [nt * nb][nb]
+    // every TcJob::C lies in [cbase, cbase + crows * nb) at a whole row offset (the epilogue
+    // reduces into C through one TMA tensor map over this range)
+    const float* cbase;
+    uint64_t crows;
 };
 bool tc_gemm_available();
 cudaError_t tc_gemm_tf32x3_launch(const TcArgs& a, int njobs, cudaStream_t s);

@@ -50,6 +50,8 @@ mp_status mp_test_tc_gemm(int kind, const void* d_panel, const void* d_panel_lo,
     a.jobs = dj;
     a.nb = nb;
     a.nt = nt;
+    a.cbase = d_C;
+    a.crows = (uint64_t)nb;
     cudaError_t e;
     if (kind == 1) {
         a.hi = (const float*)d_panel;

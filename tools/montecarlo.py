@@ -5,7 +5,7 @@ FP64 factor (mp_gp_sample), then MLE with the FP64 map and with the adaptive MP 
 bounds [0.01, 2]^3, start at the lower bounds).  Reports every estimate, the per-replica
 max |theta_MP - theta_FP64| and the mean / std of both estimators.
 
-  python tools/montecarlo.py [n] [replicas] [u_req]
+  python tools/montecarlo.py [n] [replicas] [u_req] [beta] [nu]
 """
 import json
 import os
@@ -26,7 +26,9 @@ def main():
     R = int(sys.argv[2]) if len(sys.argv) > 2 else 4
     u_req = float(sys.argv[3]) if len(sys.argv) > 3 else 1e-9
     nb = 2048 if n >= 40000 else 512
-    theta_true = (1.0, 0.03, 0.5)
+    beta = float(sys.argv[4]) if len(sys.argv) > 4 else 0.03
+    nu = float(sys.argv[5]) if len(sys.argv) > 5 else 0.5
+    theta_true = (1.0, beta, nu)
     ev = mp.Evaluator(n, nb)
     reps = []
     for r in range(R):
@@ -52,7 +54,7 @@ def main():
            "max_abs_dtheta": float(max(q["max_abs_dtheta"] for q in reps))}
     print(json.dumps(out))
     os.makedirs("gpurun_out", exist_ok=True)
-    json.dump(out, open(f"gpurun_out/montecarlo_n{n}_R{R}.json", "w"), indent=1)
+    json.dump(out, open(f"gpurun_out/montecarlo_n{n}_R{R}_b{beta}_nu{nu}.json", "w"), indent=1)
 
 
 if __name__ == "__main__":
