@@ -45,13 +45,19 @@ CONFIGS = {
 METRIC = "Tflop/s & joules per MLE log-likelihood eval (n=360k) at 1/2/4/8 B200"
 FP64_NOMINAL, BF16_NOMINAL, INT8_NOMINAL = 40.0, 2250.0, 4500.0  # dense TFLOP/s (TOP/s), B200 nominal
 OZ_PRODUCTS = 36  # int8 GEMMs per FP64 GEMM in the Ozaki split with S = 8 slices (S (S+1) / 2)
+CRT_PRODUCTS = 16  # int8 GEMMs per FP64 GEMM in the CRT (Ozaki scheme II) engine: one per modulus
+# FP64-class engines (mp_handle_config "ozaki" % 100): products per FP64 GEMM, kernel, int8 planes per operand
+ENGINES = {16: (CRT_PRODUCTS, "crt_gemm_kernel (FP64-class update as 16 INT8 tcgen05 GEMMs, CRT / Ozaki scheme II)",
+                "crt-int8 (16 moduli)", 16),
+           8: (OZ_PRODUCTS, "ozaki_gemm_kernel<8> (FP64-class update as 36 INT8 tcgen05 GEMMs)", "ozaki-int8 (S=8)", 8)}
 
 
-def ncu_traffic():
+def ncu_traffic(engine):
     """dram bytes per FP64-equivalent flop of the dominant kernel, from one `ncu --set full` capture of a
-    launch inside a bench run (profiles/r01/ncu_traffic.json records the capture and its command)."""
-    p = os.path.join(ROOT, "profiles", "r01", "ncu_traffic.json")
-    return json.load(open(p)) if os.path.exists(p) else None
+    launch inside a bench run (profiles/r01/ncu_traffic*.json record the capture and its command)."""
+    name = {16: "ncu_traffic_crt.json", 8: "ncu_traffic.json"}.get(engine)
+    p = os.path.join(ROOT, "profiles", "r01", name) if name else None
+    return json.load(open(p)) if p and os.path.exists(p) else None
 
 
 def measured_peaks():
@@ -346,18 +352,20 @@ def main():
     int8_peak = peaks["bf16_tflops_sustained"] * INT8_NOMINAL / BF16_NOMINAL
     fp64_eq = dom["flops"] / (dom["ms"] / 1e3) / 1e12 if dom["ms"] > 0 else 0.0
     flops_per_launch = dom["flops"] / max(1, dom["launches"])
-    tr = ncu_traffic()
-    traffic = (tr["dram_bytes_per_flop"] * flops_per_launch) if tr and engine["ozaki"] % 100 == 8 else None
-    # algorithmic bytes of an FP64-class tile-GEMM on the INT8 path: 8 int8 planes of A and B (8 B/entry each)
-    # + row exponents + the FP64 C tile read and written (16 B/entry)
-    alg_bytes_per_launch = flops_per_launch / (2.0 * nb**3) * (8 + 8 + 16) * nb * nb
+    eng = ENGINES.get(engine["ozaki"] % 100)
+    tr = ncu_traffic(engine["ozaki"] % 100)
+    traffic = (tr["dram_bytes_per_flop"] * flops_per_launch) if tr and eng else None
+    # algorithmic bytes of an FP64-class tile-GEMM on the INT8 path: the int8 planes of A and B (8 or 16
+    # B/entry each) + the FP64 C tile read and written (16 B/entry)
+    planes = eng[3] if eng else 8
+    alg_bytes_per_launch = flops_per_launch / (2.0 * nb**3) * (planes + planes + 16) * nb * nb
     try:
         cub = cublas_dgemm_tflops()
     except Exception:
         cub = None
     last = reps[-1]
     upd = list(last.flops_update)
-    fp64_class_peak = (int8_peak / OZ_PRODUCTS) if engine["ozaki"] % 100 == 8 else fp64_peak
+    fp64_class_peak = (int8_peak / eng[0]) if eng else fp64_peak
     fp32_class_peak = (int8_peak / 10) if engine["ozaki"] >= 100 else peaks["bf16_tflops_sustained"] * 0.5 / 3
     roof_time_s = (upd[0] / (fp64_class_peak * 1e12)
                    + upd[1] / (fp32_class_peak * 1e12)
@@ -371,7 +379,7 @@ def main():
         "config": {"workload": f"{args.config}: n={n} ({int(math.isqrt(n))}^2 jittered grid, Morton order), nb={nb}, "
                                f"theta={list(theta)}, {cfg['map']} map u_req={args.u_req}, comm={args.policy}",
                    "n": n, "nb": nb, "map": cfg["map"], "policy": args.policy,
-                   "fp64_engine": "ozaki-int8 (S=8)" if engine["ozaki"] % 100 == 8 else "dmma",
+                   "fp64_engine": eng[2] if eng else "dmma",
                    "fp32_engine": ("ozaki-int8 (S=4)" if engine["ozaki"] >= 100 else
                                    ("tcgen05 3xTF32" if engine["tc"] else "dmma-rounded")),
                    "fp16_engine": "tcgen05 f16" if engine["tc"] else "dmma-rounded", "lookahead": engine["lookahead"],
@@ -387,16 +395,16 @@ def main():
                     for k, v in p.items()},
         "update_roofline_fraction": roof_time_s / t_upd_s if t_upd_s > 0 else None,
         "roofline": (
-            {"bound": "tensor", "kernel": "ozaki_gemm_kernel<8> (FP64-class update as 36 INT8 tcgen05 GEMMs)",
-             "achieved": OZ_PRODUCTS * fp64_eq, "peak": int8_peak, "unit": "TFLOP/s",
-             "frac": OZ_PRODUCTS * fp64_eq / int8_peak, "traffic": traffic,
+            {"bound": "tensor", "kernel": eng[1],
+             "achieved": eng[0] * fp64_eq, "peak": int8_peak, "unit": "TFLOP/s",
+             "frac": eng[0] * fp64_eq / int8_peak, "traffic": traffic,
              "algorithmic_bytes_per_launch": alg_bytes_per_launch,
              "traffic_source": tr.get("source") if tr else None,
              "peak_source": f"{peak_src} bf16_tflops_sustained x {INT8_NOMINAL}/{BF16_NOMINAL} (INT8 nominal / bf16 nominal); "
                             "achieved = executed int8 multiply-add ops x 2 per second",
              "fp64_equivalent_tflops": fp64_eq, "cublas_dgemm_tflops_live": cub,
              "fp64_equivalent_vs_cublas_dgemm": (fp64_eq / cub) if cub else None}
-            if engine["ozaki"] % 100 == 8 else
+            if eng else
             {"bound": "tensor", "kernel": "dgemm_nt_kernel (FP64 DMMA trailing update)",
              "achieved": fp64_eq, "peak": fp64_peak, "unit": "TFLOP/s",
              "frac": fp64_eq / fp64_peak if fp64_peak else None, "traffic": None,

@@ -23,6 +23,18 @@ mp_status mp_test_tc_gemm(int kind, const void* d_panel, const void* d_panel_lo,
  * int8 slices, then C -= P_m P_n^T using the first S slices: S = 8 (FP64 class, C FP64, lower CTA
  * tiles only if `lower`) or S = 4 (FP32 class, C is FP32). */
 mp_status mp_test_ozaki_gemm(const double* d_panel, double* d_C, int nb, int nt, int m, int n, int S, int lower);
+/* CRT ("Ozaki scheme II") GEMM on INT8 tensor cores: the nt tiles of the FP64 panel [nt*nb][nb]
+ * become nmod int8 residue planes, then C (FP64 nb x nb) -= P_m P_n^T (lower: only 256 x 256 blocks
+ * on or below the diagonal).  nb % 256 == 0, 2 <= nmod <= 16. */
+mp_status mp_test_crt_gemm(const double* d_panel, double* d_C, int nb, int nt, int m, int n, int nmod, int lower);
+/* Isolated timing of the FP64-class INT8 engines (engine 8: 8-slice splitting, 16: CRT with nmod
+ * moduli) on njobs batched nb x nb tile-GEMMs over an nt-tile panel; ms[0] = panel split, ms[1] = GEMM
+ * launch, milliseconds (mean of reps). */
+mp_status mp_bench_fp64_engine(int engine, int nb, int nt, int njobs, int nmod, int reps, float* ms);
+/* Host constants of the CRT engine for nmod (even) moduli and inner dimension K: operand bits, the
+ * nmod moduli, the split CRT weights w_j = H_j + L_j of the nmod/2 paired moduli m_j = p_2j p_2j+1
+ * and M = Mhl[0] + Mhl[1] (host pointers). */
+mp_status mp_test_crt_constants(int nmod, int K, int* bits, int* moduli, double* H, double* L, double* Mhl);
 /* 1 if the tcgen05 kernels are compiled in, else 0. */
 int mp_tc_available(void);
 /* Correctly rounded sum of n doubles (host; the S of the precision rule). */

@@ -10,7 +10,7 @@ import ctypes as C
 import os
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_HERE, "libmpgeo.so")
+LIB_PATH = os.environ.get("MPGEO_LIB") or os.path.join(_HERE, "libmpgeo.so")  # MPGEO_LIB: experiment builds
 
 MP_OK, MP_ERR_ARG, MP_ERR_NOT_SPD, MP_ERR_CUDA, MP_ERR_COMM, MP_ERR_NOMEM, MP_ERR_UNSUPPORTED, MP_ERR_STATE = range(8)
 STATUS_NAMES = ["MP_OK", "MP_ERR_ARG", "MP_ERR_NOT_SPD", "MP_ERR_CUDA", "MP_ERR_COMM", "MP_ERR_NOMEM",
@@ -93,6 +93,9 @@ def _load() -> C.CDLL:
         "mp_test_tc_gemm": (i32, [i32, vp, vp, vp, i32, i32, i32, i32]),
         "mp_tc_available": (i32, []),
         "mp_test_ozaki_gemm": (i32, [vp, vp, i32, i32, i32, i32, i32, i32]),
+        "mp_test_crt_gemm": (i32, [vp, vp, i32, i32, i32, i32, i32, i32]),
+        "mp_bench_fp64_engine": (i32, [i32, i32, i32, i32, i32, i32, C.POINTER(C.c_float)]),
+        "mp_test_crt_constants": (i32, [i32, i32, C.POINTER(i32), C.POINTER(i32), dp, dp, dp]),
     }
     for name, (res, args) in sig.items():
         f = getattr(lib, name)

@@ -29,6 +29,7 @@
 #include "tc_gemm.h"
 #include "dist.h"
 #include "ozaki.h"
+#include "crt.h"
 
 using namespace mpgeo;
 
@@ -37,6 +38,7 @@ struct ProfRec {
     cudaEvent_t e0, e1;
     int cls;
     double flops;
+    int stream;
 };
 struct mp_handle {
     int device = 0, rank = 0, nranks = 1, P = 1, Q = 1;
@@ -49,7 +51,8 @@ struct mp_handle {
     bool broken = false;
     int tc_mode = 1;  // 1: tcgen05 kernels for FP32/FP16 classes when available, 0: DMMA emulation
     int lookahead = 1;  // 1: panel k+1 on the high-priority panel stream overlaps update k
-    int ozaki = 8;      // 8: FP64-class GEMM/SYRK emulated on INT8 tensor cores (S = 8 slices); 0: DMMA
+    int ozaki = 16;     // FP64-class GEMM/SYRK: 16 = CRT (Ozaki-II, 16 moduli) / 8 = 8-slice splitting,
+                        // both on INT8 tensor cores; 0 = DMMA
     int matern_table = 1;  // general nu: tabulated correlation (1) or direct K_nu per entry (0)
     int ozaki32 = 0;    // 1: FP32-class GEMM on INT8 tensor cores (first 4 slices); 0: 3xTF32 tcgen05 (default)
     cudaStream_t pstream = nullptr;
@@ -65,7 +68,7 @@ struct mp_handle {
 struct Regions {
     size_t total = 0;
     size_t inputs = 0, p64 = 0, p16 = 0, phi = 0, plo = 0, ltilde = 0, wbuf = 0, wbuf2 = 0, oz = 0, ozexp = 0,
-           wdiag = 0, mtab = 0;
+           wdiag = 0, mtab = 0, crt = 0, crtflags = 0;
     size_t vec_r = 0, vec_y = 0, partials = 0, norms = 0, ctrl = 0, ctrl_bytes = 0;
     std::vector<size_t> tile_off;  // per (m*nt+k), SIZE_MAX if not stored here
     size_t pool = 0;               // start of the tile pool
@@ -171,7 +174,13 @@ static Regions layout(const mp_matrix* A, const uint8_t* storage) {
     R.p16 = take(2 * (size_t)nt * nb2 * 2);
     R.phi = take(2 * (size_t)nt * nb2 * 4);
     R.plo = take(2 * (size_t)nt * nb2 * 4);
-    R.oz = take(2 * (size_t)nt * nb2 * 8);         // Ozaki int8 slice planes (S <= 8), two sets
+    // int8 operand planes of the FP64-class engine, two sets: 8 slices (splitting) or 16 residues (CRT)
+    const bool crt = A->h && A->h->ozaki == 16 && A->nb % 256 == 0;
+    R.oz = take(2 * (size_t)nt * nb2 * (crt ? CRT_NMAX : 8));
+    if (crt) {  // CRT engine: per-CTA residue staging slots + their busy flags
+        R.crt = take((size_t)crt_scratch_slots() * CRT_SLOT_BYTES);
+        R.crtflags = take((size_t)crt_scratch_slots() * sizeof(int));
+    }
     R.ozexp = take(2 * (size_t)nt * A->nb * 4);    // per-row exponents
     R.tile_off.assign((size_t)nt * nt, SIZE_MAX);
     R.pool = align_up(off, 256);  // tile pool start (tile offsets from here are whole nb-float rows when 256 | nb)
@@ -251,7 +260,7 @@ static mp_status run_plan(mp_handle* h, mp_matrix* A, Arena& ar, std::vector<Op>
             CK(h, cudaEventRecord(e0, st));
             CK(h, op.fn(st));
             CK(h, cudaEventRecord(e1, st));
-            h->prof_pending.push_back(ProfRec{e0, e1, op.cls, op.flops});
+            h->prof_pending.push_back(ProfRec{e0, e1, op.cls, op.flops, op.stream});
         } else {
             CK(h, op.fn(st));
         }
@@ -339,6 +348,21 @@ mp_status mp_set_profiling(mp_handle* h, int enable) {
 mp_status mp_get_profile(mp_handle* h, mp_profile* out) {
     if (!h || !out) return MP_ERR_ARG;
     CK(h, cudaStreamSynchronize(h->stream));
+    // MPGEO_TIMELINE=<path>: append every profiled launch as "class stream start_ms end_ms flops"
+    // (relative to the first one) — the schedule of one call, for tuning the lookahead overlap
+    if (const char* path = getenv("MPGEO_TIMELINE"))
+        if (!h->prof_pending.empty())
+            if (FILE* f = fopen(path, "a")) {
+                const cudaEvent_t t0 = h->prof_pending.front().e0;
+                for (const ProfRec& r : h->prof_pending) {
+                    float a = 0.f, b = 0.f;
+                    cudaEventElapsedTime(&a, t0, r.e0);
+                    cudaEventElapsedTime(&b, t0, r.e1);
+                    fprintf(f, "%d %d %.4f %.4f %.6g\n", r.cls, r.stream, a, b, r.flops);
+                }
+                fprintf(f, "--\n");
+                fclose(f);
+            }
     for (const ProfRec& r : h->prof_pending) {
         float ms = 0.f;
         CK(h, cudaEventElapsedTime(&ms, r.e0, r.e1));
@@ -358,7 +382,9 @@ mp_status mp_handle_config(const mp_handle* h, int* tc, int* lookahead, int* oza
     // ozaki: 0 = DMMA FP64 class; 8 = INT8 FP64 class; +100 if the FP32 class also runs on INT8
     if (tc) *tc = (h->tc_mode != 0 && tc_gemm_available()) ? 1 : 0;
     if (lookahead) *lookahead = h->lookahead;
-    if (ozaki) *ozaki = (h->ozaki == 8 && ozaki_available()) ? (8 + (h->ozaki32 ? 100 : 0)) : 0;
+    if (ozaki)
+        *ozaki = (h->ozaki == 16 && crt_available()) ? 16
+                 : (h->ozaki == 8 && ozaki_available()) ? (8 + (h->ozaki32 ? 100 : 0)) : 0;
     return MP_OK;
 }
 
@@ -700,9 +726,17 @@ static mp_status plan_potrf(mp_handle* h, mp_matrix* A, const uint8_t* km, const
     const bool use_tc = h->tc_mode != 0 && tc_gemm_available() && nb % 256 == 0;
     const float* const cpool = A->at<float>(A->R.pool);                // tcgen05 epilogue C map range
     const uint64_t crows = (A->R.total - A->R.pool) / ((size_t)nb * 4);
-    const int ozS = h->ozaki == 8 && ozaki_available() && nb % 128 == 0 ? 8 : 0;
+    const double* const cpool64 = A->at<double>(A->R.pool);  // FP64 view of the pool (CRT epilogue C map)
+    const uint64_t crows64 = (A->R.total - A->R.pool) / ((size_t)nb * 8);
+    const bool crt = h->ozaki == 16 && crt_available() && nb % 256 == 0 && A->R.crt;
+    CrtConst crtc;
+    if (crt && !crt_constants(CRT_NMAX, nb, &crtc)) FAIL(h, MP_ERR_ARG, "CRT constants for nb=%d", nb);
+    // the 8-slice splitting engine: selected (8), or the fallback of the CRT engine when nb % 256 != 0
+    const int ozS = !crt && (h->ozaki == 8 || h->ozaki == 16) && ozaki_available() && nb % 128 == 0 ? 8 : 0;
     const bool oz32 = ozS && h->ozaki32 && nb % 256 == 0;
     int8_t* const ozb = A->at<int8_t>(A->R.oz);
+    uint8_t* const crt_scr = crt ? A->at<uint8_t>(A->R.crt) : nullptr;
+    int* const crt_flags = crt ? A->at<int>(A->R.crtflags) : nullptr;
     int* const ozeb = A->at<int>(A->R.ozexp);
     auto K = [&](int m, int k) { return km[(size_t)m * nt + k]; };
     auto C = [&](int m, int k) { return cm[(size_t)m * nt + k]; };
@@ -779,7 +813,7 @@ static mp_status plan_potrf(mp_handle* h, mp_matrix* A, const uint8_t* km, const
         __half* p16 = p16b + set * nt * nb2;
         float* phi = phib + set * nt * nb2;
         float* plo = plob + set * nt * nb2;
-        int8_t* ozs = ozb + set * nt * nb2 * 8;
+        int8_t* ozs = ozb + set * nt * nb2 * (crt ? CRT_NMAX : 8);
         int* oze = ozeb + set * (size_t)nt * nb;
         const int64_t ozplane = (int64_t)nt * nb2;
         cur = &pan[k];
@@ -965,6 +999,21 @@ static mp_status plan_potrf(mp_handle* h, mp_matrix* A, const uint8_t* km, const
             cur_push(Op{[=](cudaStream_t s) { return set_flag_launch(df, dv, s); }, C_CONV, 0});
         }
         // ---- 5d. Ozaki: split every panel tile this GPU's FP64-class successors read into int8 slices
+        if (crt) {  // CRT engine: residue planes of every panel tile this GPU's FP64-class successors read
+            std::vector<CrtSplitItem> sp;
+            for (int m = k + 1; m < nt; ++m) {
+                bool need = A->mine(m, m);
+                for (int n = k + 1; n < m && !need; ++n) need |= A->mine(m, n) && K(m, n) == MP_FP64;
+                for (int n = m + 1; n < nt && !need; ++n) need |= A->mine(n, m) && K(n, m) == MP_FP64;
+                if (need)
+                    sp.push_back(CrtSplitItem{p64 + (size_t)m * nb2, ozs + (size_t)m * nb2, oze + (size_t)m * nb, ozplane});
+            }
+            if (!sp.empty()) {
+                CrtSplitItem* dsp = ar.push(sp);
+                const int nsp = (int)sp.size();
+                cur_push(Op{[=](cudaStream_t s) { return crt_split_launch(dsp, nsp, nb, crtc, s); }, C_CONV, 0});
+            }
+        }
         if (ozS) {
             std::vector<OzSplitItem> sp;
             for (int m = k + 1; m < nt; ++m) {
@@ -1009,7 +1058,7 @@ static mp_status plan_potrf(mp_handle* h, mp_matrix* A, const uint8_t* km, const
             }
         }
         const double f3 = fnb * fnb * fnb;
-        if (ozS) {  // FP64 class on INT8 tensor cores
+        if (ozS || crt) {  // FP64 class on INT8 tensor cores
             for (int lower = 1; lower >= 0; --lower) {
                 std::vector<OzJob> oj;
                 for (auto& g : (lower ? syrk : g64)) {
@@ -1020,9 +1069,16 @@ static mp_status plan_potrf(mp_handle* h, mp_matrix* A, const uint8_t* km, const
                 if (oj.empty()) continue;
                 OzJob* dj = ar.push(oj);
                 const int nj = (int)oj.size();
-                OzArgs oa{dj, ozs, oze, ozplane, nb, nt, ozS, lower, 0};
-                cur_push(Op{[=](cudaStream_t s) { return ozaki_gemm_launch(oa, nj, s); }, C_UPD64,
-                            (lower ? f3 : 2 * f3) * nj});
+                if (crt) {
+                    // 64 of the 74 CTA pairs: SMs stay free for the panel stream's POTRF/TRSM (lookahead)
+                    CrtArgs ca{dj, ozs, oze, ozplane, nb, nt, lower, crt_scr, crt_flags, crtc, cpool64, crows64, la ? 64 : 0};
+                    cur_push(Op{[=](cudaStream_t s) { return crt_gemm_launch(ca, nj, s); }, C_UPD64,
+                                (lower ? f3 : 2 * f3) * nj});
+                } else {
+                    OzArgs oa{dj, ozs, oze, ozplane, nb, nt, ozS, lower, 0};
+                    cur_push(Op{[=](cudaStream_t s) { return ozaki_gemm_launch(oa, nj, s); }, C_UPD64,
+                                (lower ? f3 : 2 * f3) * nj});
+                }
             }
             syrk.clear();
             g64.clear();
@@ -1105,6 +1161,7 @@ static mp_status potrf_run(mp_handle* h, mp_matrix* A, const uint8_t* km, const 
         }
     const int big = INT_MAX;
     CK(h, cudaMemcpyAsync(h->d_info, &big, sizeof(int), cudaMemcpyHostToDevice, h->stream));
+    if (A->R.crtflags) CK(h, cudaMemsetAsync(A->ws + A->R.crtflags, 0, (size_t)crt_scratch_slots() * sizeof(int), h->stream));
     Arena ar;
     ar.dev_base = A->ws + A->R.ctrl;
     std::vector<Op> ops;

@@ -1,10 +1,14 @@
 // Kernel-level test hooks (include/mpgeo_test.h).  Not on the hot path.
 #include "../../include/mpgeo_test.h"
+#include <math.h>
+#include <stdio.h>
+#include <stdlib.h>
 #include <vector>
 
 #include "kernels.h"
 #include "tc_gemm.h"
 #include "ozaki.h"
+#include "crt.h"
 
 using namespace mpgeo;
 
@@ -93,6 +97,160 @@ mp_status mp_test_ozaki_gemm(const double* d_panel, double* d_C, int nb, int nt,
     cudaFree(it);
     cudaFree(dj);
     return (e == cudaSuccess && e2 == cudaSuccess) ? MP_OK : MP_ERR_CUDA;
+}
+
+mp_status mp_test_crt_gemm(const double* d_panel, double* d_C, int nb, int nt, int m, int n, int nmod, int lower) {
+    if (!crt_available()) return MP_ERR_UNSUPPORTED;
+    CrtConst c;
+    if (!crt_constants(nmod, nb, &c)) return MP_ERR_ARG;
+    const int64_t plane = (int64_t)nt * nb * nb;
+    const int slots = crt_scratch_slots();
+    int8_t* pl = nullptr;
+    int* ex = nullptr;
+    CrtSplitItem* it = nullptr;
+    OzJob* dj = nullptr;
+    uint8_t* scr = nullptr;
+    int* flags = nullptr;
+    if (cudaMalloc(&pl, plane * nmod) || cudaMalloc(&ex, sizeof(int) * nt * nb) ||
+        cudaMalloc(&it, sizeof(CrtSplitItem) * nt) || cudaMalloc(&dj, sizeof(OzJob)) ||
+        cudaMalloc(&scr, (size_t)slots * CRT_SLOT_BYTES) || cudaMalloc(&flags, sizeof(int) * slots))
+        return MP_ERR_CUDA;
+    cudaMemset(flags, 0, sizeof(int) * slots);
+    std::vector<CrtSplitItem> h(nt);
+    for (int t = 0; t < nt; ++t)
+        h[t] = CrtSplitItem{d_panel + (size_t)t * nb * nb, pl + (size_t)t * nb * nb, ex + (size_t)t * nb, plane};
+    cudaMemcpy(it, h.data(), sizeof(CrtSplitItem) * nt, cudaMemcpyHostToDevice);
+    OzJob j{m, n, d_C};
+    cudaMemcpy(dj, &j, sizeof j, cudaMemcpyHostToDevice);
+    cudaError_t e = crt_split_launch(it, nt, nb, c, 0);
+    CrtArgs a{dj, pl, ex, plane, nb, nt, lower, scr, flags, c, d_C, (uint64_t)nb, 0};
+    if (e == cudaSuccess) e = crt_gemm_launch(a, 1, 0);
+    cudaError_t e2 = cudaDeviceSynchronize();
+    if (const char* path = getenv("MPGEO_CRT_DUMP")) {  // debugging aid: planes, exponents, 8 scratch slots
+        std::vector<char> buf((size_t)plane * nmod + sizeof(int) * nt * nb + 8 * CRT_SLOT_BYTES);
+        cudaMemcpy(buf.data(), pl, (size_t)plane * nmod, cudaMemcpyDeviceToHost);
+        cudaMemcpy(buf.data() + plane * nmod, ex, sizeof(int) * nt * nb, cudaMemcpyDeviceToHost);
+        cudaMemcpy(buf.data() + plane * nmod + sizeof(int) * nt * nb, scr, 8 * CRT_SLOT_BYTES, cudaMemcpyDeviceToHost);
+        if (FILE* f = fopen(path, "wb")) {
+            fwrite(buf.data(), 1, buf.size(), f);
+            fclose(f);
+        }
+    }
+    cudaFree(pl);
+    cudaFree(ex);
+    cudaFree(it);
+    cudaFree(dj);
+    cudaFree(scr);
+    cudaFree(flags);
+    if (e == cudaErrorInvalidValue) return MP_ERR_ARG;
+    return (e == cudaSuccess && e2 == cudaSuccess) ? MP_OK : MP_ERR_CUDA;
+}
+
+/* Isolated timing of the FP64-class engines on a batched trailing-update-like launch: a random FP64
+ * panel of nt tiles, njobs tile-GEMMs C_j -= P_{m_j} P_{n_j}^T (distinct C tiles), engine 8 (8-slice
+ * splitting) or 16 (CRT, nmod moduli).  ms[0] = split of the nt panel tiles, ms[1] = one GEMM launch
+ * (mean over reps after one warm-up). */
+mp_status mp_bench_fp64_engine(int engine, int nb, int nt, int njobs, int nmod, int reps, float* ms) {
+    const int64_t plane = (int64_t)nt * nb * nb;
+    const int np = engine == 16 ? nmod : 8;
+    double *P = nullptr, *Cb = nullptr;
+    int8_t* pl = nullptr;
+    int* ex = nullptr;
+    void* it = nullptr;
+    OzJob* dj = nullptr;
+    uint8_t* scr = nullptr;
+    int* flags = nullptr;
+    const int slots = crt_scratch_slots();
+    if (cudaMalloc(&P, plane * 8) || cudaMalloc(&Cb, (size_t)njobs * nb * nb * 8) || cudaMalloc(&pl, plane * np) ||
+        cudaMalloc(&ex, sizeof(int) * nt * nb) || cudaMalloc(&it, 64 * nt) || cudaMalloc(&dj, sizeof(OzJob) * njobs) ||
+        cudaMalloc(&scr, (size_t)slots * CRT_SLOT_BYTES) || cudaMalloc(&flags, sizeof(int) * slots))
+        return MP_ERR_CUDA;
+    cudaMemset(flags, 0, sizeof(int) * slots);
+    cudaMemset(P, 0, plane * 8);
+    cudaMemset(Cb, 0, (size_t)njobs * nb * nb * 8);
+    {   // deterministic non-trivial panel: x = sin(i * 0.37 + j * 0.11) scaled per row
+        std::vector<double> h((size_t)nb * nb);
+        for (int t = 0; t < nt; ++t) {
+            for (int i = 0; i < nb; ++i)
+                for (int j = 0; j < nb; ++j) h[(size_t)i * nb + j] = sin(0.37 * (i + t * nb) + 0.11 * j) * (1.0 + (i % 7));
+            cudaMemcpy(P + (size_t)t * nb * nb, h.data(), h.size() * 8, cudaMemcpyHostToDevice);
+        }
+    }
+    std::vector<OzJob> jobs(njobs);
+    const bool same = getenv("MPGEO_BENCH_SAMEJOB") != nullptr;  // every job reads panel tiles (0, 1)
+    for (int j = 0; j < njobs; ++j)
+        jobs[j] = same ? OzJob{0, 1, Cb + (size_t)j * nb * nb} : OzJob{j % nt, (j / nt + j + 1) % nt, Cb + (size_t)j * nb * nb};
+    cudaMemcpy(dj, jobs.data(), sizeof(OzJob) * njobs, cudaMemcpyHostToDevice);
+    CrtConst c;
+    if (engine == 16 && !crt_constants(nmod, nb, &c)) return MP_ERR_ARG;
+    if (engine == 16) {
+        std::vector<CrtSplitItem> hs(nt);
+        for (int t = 0; t < nt; ++t)
+            hs[t] = CrtSplitItem{P + (size_t)t * nb * nb, pl + (size_t)t * nb * nb, ex + (size_t)t * nb, plane};
+        cudaMemcpy(it, hs.data(), sizeof(CrtSplitItem) * nt, cudaMemcpyHostToDevice);
+    } else {
+        std::vector<OzSplitItem> hs(nt);
+        for (int t = 0; t < nt; ++t)
+            hs[t] = OzSplitItem{P + (size_t)t * nb * nb, pl + (size_t)t * nb * nb, ex + (size_t)t * nb, plane};
+        cudaMemcpy(it, hs.data(), sizeof(OzSplitItem) * nt, cudaMemcpyHostToDevice);
+    }
+    auto split = [&]() {
+        return engine == 16 ? crt_split_launch((const CrtSplitItem*)it, nt, nb, c, 0)
+                            : ozaki_split_launch((const OzSplitItem*)it, nt, nb, 8, 0);
+    };
+    auto gemm = [&]() {
+        if (engine == 16) {
+            CrtArgs a{dj, pl, ex, plane, nb, nt, 0, scr, flags, c, Cb, (uint64_t)njobs * nb, 0};
+            return crt_gemm_launch(a, njobs, 0);
+        }
+        OzArgs a{dj, pl, ex, plane, nb, nt, 8, 0, 0};
+        return ozaki_gemm_launch(a, njobs, 0);
+    };
+    cudaEvent_t e0, e1, e2;
+    cudaEventCreate(&e0);
+    cudaEventCreate(&e1);
+    cudaEventCreate(&e2);
+    cudaError_t e = split();
+    if (e == cudaSuccess) e = gemm();
+    cudaDeviceSynchronize();
+    cudaEventRecord(e0, 0);
+    for (int r = 0; r < reps && e == cudaSuccess; ++r) e = split();
+    cudaEventRecord(e1, 0);
+    for (int r = 0; r < reps && e == cudaSuccess; ++r) e = gemm();
+    cudaEventRecord(e2, 0);
+    cudaError_t es = cudaEventSynchronize(e2);
+    float a = 0, b = 0;
+    cudaEventElapsedTime(&a, e0, e1);
+    cudaEventElapsedTime(&b, e1, e2);
+    ms[0] = a / reps;
+    ms[1] = b / reps;
+    cudaFree(P);
+    cudaFree(Cb);
+    cudaFree(pl);
+    cudaFree(ex);
+    cudaFree(it);
+    cudaFree(dj);
+    cudaFree(scr);
+    cudaFree(flags);
+    cudaEventDestroy(e0);
+    cudaEventDestroy(e1);
+    cudaEventDestroy(e2);
+    return (e == cudaSuccess && es == cudaSuccess) ? MP_OK : MP_ERR_CUDA;
+}
+
+/* Host constants of the CRT engine (pinned on CPU against big-integer arithmetic). */
+mp_status mp_test_crt_constants(int nmod, int K, int* bits, int* moduli, double* H, double* L, double* Mhl) {
+    CrtConst c;
+    if (!crt_constants(nmod, K, &c)) return MP_ERR_ARG;
+    *bits = c.bits;
+    for (int t = 0; t < nmod; ++t) moduli[t] = c.p[t];
+    for (int j = 0; j < nmod / 2; ++j) {
+        H[j] = c.H[j];
+        L[j] = c.L[j];
+    }
+    Mhl[0] = c.Mh;
+    Mhl[1] = c.Ml;
+    return MP_OK;
 }
 
 }  // extern "C"

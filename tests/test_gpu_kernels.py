@@ -172,3 +172,49 @@ def test_ozaki_int8_fp32_class_gemm(lib):
     err = np.linalg.norm(got - exact) / np.linalg.norm(exact)
     err_sg = np.linalg.norm(sgemm - exact) / np.linalg.norm(exact)
     assert err <= 2 * err_sg, (err, err_sg)
+
+
+@pytest.mark.parametrize("nb,nt,m,n,nmod", [(512, 3, 2, 0, 16), (4096, 2, 1, 0, 16), (2048, 3, 1, 2, 16)])
+def test_crt_int8_fp64_gemm(lib, nb, nt, m, n, nmod):
+    """FP64 GEMM by CRT modular emulation on tcgen05 kind::i8 vs the exact FP64 product: with 16
+    moduli the operands keep b = 56 bits (rounded) per row, so |err| <= K 2^-(b+1) max|a_i| max|b_j|
+    + the final FP64 rounding — within the FP64-GEMM bound 8 K u max|a| max|b| used for the splitting
+    engine.  nb = 4096 gives 256 pair tiles for 74 persistent CTA pairs (several tiles per pair, both
+    accumulator parities, scratch-slot reuse).  Rows of very different scale and an all-zero row."""
+    rng = np.random.default_rng(nb + nmod)
+    P = rng.standard_normal((nt * nb, nb)) * np.exp(rng.uniform(-3, 3, (nt * nb, 1)))
+    P[m * nb + 5] = 0.0
+    Cm = rng.standard_normal((nb, nb))
+    dP, dC = dev(P), dev(Cm)
+    assert lib.mp_test_crt_gemm(C.c_void_p(dP.data_ptr()), C.c_void_p(dC.data_ptr()), nb, nt, m, n, nmod, 0) == 0
+    got = dC.cpu().numpy()
+    A, B = P[m * nb:(m + 1) * nb], P[n * nb:(n + 1) * nb]
+    ref = Cm - A @ B.T
+    ma = np.abs(A).max(axis=1)[:, None]
+    mb = np.abs(B).max(axis=1)[None, :]
+    scale = np.maximum(ma * mb, 1e-300)
+    err = np.max(np.abs(got - ref) / (scale + np.abs(ref) * 1e-300))
+    bound = 8 * nb * 2.0**-53
+    assert err <= bound, (err, bound)
+    assert np.array_equal(got[5], Cm[5])  # zero row of A: C row untouched
+
+
+def test_crt_int8_syrk_lower(lib):
+    """lower = 1 (DSYRK on a diagonal tile): 256 x 256 blocks on or below the diagonal are updated,
+    strictly-upper blocks are left untouched."""
+    nb, nt = 1024, 2
+    rng = np.random.default_rng(3)
+    P = rng.standard_normal((nt * nb, nb))
+    Cm = rng.standard_normal((nb, nb))
+    dP, dC = dev(P), dev(Cm)
+    assert lib.mp_test_crt_gemm(C.c_void_p(dP.data_ptr()), C.c_void_p(dC.data_ptr()), nb, nt, 1, 1, 16, 1) == 0
+    got = dC.cpu().numpy()
+    A = P[nb:]
+    ref = Cm - A @ A.T
+    for bi in range(nb // 256):
+        for bj in range(nb // 256):
+            blk = (slice(bi * 256, (bi + 1) * 256), slice(bj * 256, (bj + 1) * 256))
+            if bj > bi:
+                assert np.array_equal(got[blk], Cm[blk])
+            else:
+                assert np.max(np.abs(got[blk] - ref[blk])) <= 8 * nb * 2.0**-53 * np.abs(A).max() ** 2

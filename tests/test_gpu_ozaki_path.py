@@ -1,5 +1,5 @@
-"""Both FP64-class engines — Ozaki split on INT8 tensor cores (default) and DMMA FP64
-(MPGEO_OZAKI=0) — must meet the all-FP64 tolerances: residual <= 1e-13, l relative error <= 1e-10."""
+"""All three FP64-class engines — CRT modular emulation (MPGEO_OZAKI=16) and the 8-slice Ozaki split
+(MPGEO_OZAKI=8), both on INT8 tensor cores, and DMMA FP64 (MPGEO_OZAKI=0) — must meet the all-FP64 tolerances: residual <= 1e-13, l relative error <= 1e-10."""
 import os
 
 import numpy as np
@@ -15,7 +15,7 @@ from tests.gpu_helpers import to_dev
 pytestmark = pytest.mark.gpu
 
 
-@pytest.fixture(scope="module", params=["8", "0"], ids=["ozaki", "dmma"])
+@pytest.fixture(scope="module", params=["16", "8", "0"], ids=["crt", "ozaki", "dmma"])
 def engine_handle(request):
     import paper_conf_cluster_caoalgkb23_b200 as mp
     os.environ["MPGEO_OZAKI"] = request.param
