@@ -366,7 +366,9 @@ def main():
     last = reps[-1]
     upd = list(last.flops_update)
     fp64_class_peak = (int8_peak / eng[0]) if eng else fp64_peak
-    fp32_class_peak = (int8_peak / 10) if engine["ozaki"] >= 100 else peaks["bf16_tflops_sustained"] * 0.5 / 3
+    # FP32-class engine: CRT-8 (8 INT8 GEMMs, ozaki >= 200), 4-slice split (10 INT8 GEMMs, >= 100), 3xTF32
+    fp32_class_peak = ((int8_peak / 8) if engine["ozaki"] >= 200 else (int8_peak / 10) if engine["ozaki"] >= 100
+                       else peaks["bf16_tflops_sustained"] * 0.5 / 3)
     roof_time_s = (upd[0] / (fp64_class_peak * 1e12)
                    + upd[1] / (fp32_class_peak * 1e12)
                    + upd[2] / (peaks["bf16_tflops_sustained"] * 1e12))
@@ -380,7 +382,8 @@ def main():
                                f"theta={list(theta)}, {cfg['map']} map u_req={args.u_req}, comm={args.policy}",
                    "n": n, "nb": nb, "map": cfg["map"], "policy": args.policy,
                    "fp64_engine": eng[2] if eng else "dmma",
-                   "fp32_engine": ("ozaki-int8 (S=4)" if engine["ozaki"] >= 100 else
+                   "fp32_engine": ("crt-int8 (8 moduli, FP32 C)" if engine["ozaki"] >= 200 else
+                                   "ozaki-int8 (S=4)" if engine["ozaki"] >= 100 else
                                    ("tcgen05 3xTF32" if engine["tc"] else "dmma-rounded")),
                    "fp16_engine": "tcgen05 f16" if engine["tc"] else "dmma-rounded", "lookahead": engine["lookahead"],
                    "parallelism": (f"2D block-cyclic {P}x{Q}, peer-memory panel exchange" if distributed

@@ -24,11 +24,15 @@ mp_status mp_test_tc_gemm(int kind, const void* d_panel, const void* d_panel_lo,
  * tiles only if `lower`) or S = 4 (FP32 class, C is FP32). */
 mp_status mp_test_ozaki_gemm(const double* d_panel, double* d_C, int nb, int nt, int m, int n, int S, int lower);
 /* CRT ("Ozaki scheme II") GEMM on INT8 tensor cores: the nt tiles of the FP64 panel [nt*nb][nb]
- * become nmod int8 residue planes, then C (FP64 nb x nb) -= P_m P_n^T (lower: only 256 x 256 blocks
- * on or below the diagonal).  nb % 256 == 0, 2 <= nmod <= 16. */
-mp_status mp_test_crt_gemm(const double* d_panel, double* d_C, int nb, int nt, int m, int n, int nmod, int lower);
-/* Isolated timing of the FP64-class INT8 engines (engine 8: 8-slice splitting, 16: CRT with nmod
- * moduli) on njobs batched nb x nb tile-GEMMs over an nt-tile panel; ms[0] = panel split, ms[1] = GEMM
+ * become nmod int8 residue planes, then C -= P_m P_n^T (lower: only 256 x 256 blocks on or below the
+ * diagonal).  nb % 256 == 0; nmod = 16: C is FP64 (FP64 class); nmod = 8: C is FP32 (FP32 class). */
+mp_status mp_test_crt_gemm(const double* d_panel, void* d_C, int nb, int nt, int m, int n, int nmod, int lower);
+/* The same with the C type and mode explicit: c_f32 (FP32 C, nmod = 8 only), store = 1: C = P_m P_n^T
+ * (overwrite; the FP32-class TRSM product), else C -= P_m P_n^T. */
+mp_status mp_test_crt_gemm_ex(const double* d_panel, void* d_C, int nb, int nt, int m, int n, int nmod, int lower,
+                              int c_f32, int store);
+/* Isolated timing of the INT8 engines (engine 8: 8-slice splitting, 16: CRT with nmod moduli — nmod
+ * = 16 FP64 C, nmod = 8 the FP32-class instantiation with FP32 C) on njobs batched nb x nb tile-GEMMs over an nt-tile panel; ms[0] = panel split, ms[1] = GEMM
  * launch, milliseconds (mean of reps). */
 mp_status mp_bench_fp64_engine(int engine, int nb, int nt, int njobs, int nmod, int reps, float* ms);
 /* Host constants of the CRT engine for nmod (even) moduli and inner dimension K: operand bits, the

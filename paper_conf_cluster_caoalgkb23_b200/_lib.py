@@ -94,6 +94,7 @@ def _load() -> C.CDLL:
         "mp_tc_available": (i32, []),
         "mp_test_ozaki_gemm": (i32, [vp, vp, i32, i32, i32, i32, i32, i32]),
         "mp_test_crt_gemm": (i32, [vp, vp, i32, i32, i32, i32, i32, i32]),
+        "mp_test_crt_gemm_ex": (i32, [vp, vp, i32, i32, i32, i32, i32, i32, i32, i32]),
         "mp_bench_fp64_engine": (i32, [i32, i32, i32, i32, i32, i32, C.POINTER(C.c_float)]),
         "mp_test_crt_constants": (i32, [i32, i32, C.POINTER(i32), C.POINTER(i32), dp, dp, dp]),
     }

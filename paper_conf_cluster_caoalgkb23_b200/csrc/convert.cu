@@ -70,6 +70,34 @@ __global__ void zero_upper_kernel(double* A, int nb) {
     for (int c = r + 1 + threadIdx.x; c < nb; c += blockDim.x) A[(size_t)r * nb + c] = 0.0;
 }
 
+// A = I (nb x nb): the right-hand side whose TRSM gives L~_kk^-T, the inverse factor of the
+// low-precision-class TRSMs (engine.cu step 4b)
+__global__ void identity_kernel(double* A, int nb) {
+    const int r = blockIdx.x;
+    for (int c = threadIdx.x; c < nb; c += blockDim.x) A[(size_t)r * nb + c] = c == r ? 1.0 : 0.0;
+}
+
+// dst = src^T (nb x nb FP64), 32 x 32 shared-memory tiles (coalesced reads and writes)
+__global__ void __launch_bounds__(256) transpose_kernel(const double* __restrict__ src, double* __restrict__ dst, int nb) {
+    __shared__ double t[32][33];
+    const int bx = blockIdx.x * 32, by = blockIdx.y * 32;
+    const int tx = threadIdx.x & 31, ty = threadIdx.x >> 5;
+    for (int r = ty; r < 32; r += 8) t[r][tx] = src[(size_t)(by + r) * nb + bx + tx];
+    __syncthreads();
+    for (int r = ty; r < 32; r += 8) dst[(size_t)(bx + r) * nb + by + tx] = t[tx][r];
+}
+
+cudaError_t identity_launch(double* A, int nb, cudaStream_t s) {
+    identity_kernel<<<nb, 256, 0, s>>>(A, nb);
+    return cudaGetLastError();
+}
+
+cudaError_t transpose_launch(const double* src, double* dst, int nb, cudaStream_t s) {
+    if (nb % 32) return cudaErrorInvalidValue;
+    transpose_kernel<<<dim3(nb / 32, nb / 32), 256, 0, s>>>(src, dst, nb);
+    return cudaGetLastError();
+}
+
 static unsigned chunks_for(int64_t elems, int ntiles) {
     // about 4 waves of 148 SMs in total, at least one chunk per tile
     int64_t per = (4LL * 148 * 8 + ntiles - 1) / ntiles;

@@ -174,6 +174,7 @@ constexpr int A_BYTES = BM * BK;    // 16 KB
 constexpr int B_BYTES = (BN / 2) * BK;  // 16 KB: each CTA loads half of B
 constexpr int STAGE_BYTES = A_BYTES + B_BYTES;
 constexpr int STAGES = 6;
+constexpr int RING = 4;  // tile-index ring depth (dynamic scheduler)
 // C update staging: per epilogue warp two 32 x 8 FP64 boxes (2 KB, 64-byte swizzle) reduced into C
 // by the TMA unit (cp.reduce.async.bulk.tensor .add on the FP64 C map)
 constexpr int STG_BOX = 32 * 8 * 8;
@@ -192,13 +193,15 @@ constexpr uint32_t IDESC = (2u << 4) | (1u << 7) | (1u << 10) | ((uint32_t)(BN >
 
 struct __align__(64) CrtParams {
     CUtensorMap a, b;  // 3D [N][rows][nb] int8, box {128, 128, 1}
-    CUtensorMap cmap;  // FP64 C rows [crows][nb] from cbase, box {8, 32}, 64-byte swizzle
-    const double* cbase;
+    CUtensorMap cmap;  // C rows [crows][nb] from cbase, box {8, 32}: FP64 (64-byte swizzle) or FP32 (no swizzle)
+    const void* cbase;
     const OzJob* jobs;
     const int* exps;
     uint8_t* scratch;
     int* slot_flags;
     int nslots, nb, tiles_n, tiles_per_job, lower, total;
+    int store;  // 1: C = P_m P_n^T (TMA store), 0: C -= P_m P_n^T (TMA reduce-add)
+    int* tile_counter;  // dynamic tile scheduler (zero before the launch)
     CrtConst c;
 };
 
@@ -230,6 +233,19 @@ __device__ __forceinline__ void mbar_arrive_cluster(uint32_t cbar) {
 // (wait::ld), so no memory ordering of its global stores is needed (a release would add a MEMBAR)
 __device__ __forceinline__ void mbar_arrive_cluster_relaxed(uint32_t cbar) {
     asm volatile("mbarrier.arrive.relaxed.cluster.shared::cluster.b64 _, [%0];" ::"r"(cbar) : "memory");
+}
+// wait with cluster-scope acquire: the awaited data (the tile ring) may be written by the peer CTA
+__device__ __forceinline__ void mbar_wait_cl(uint32_t bar, uint32_t parity) {
+    asm volatile(
+        "{\n\t.reg .pred p;\n\t"
+        "WAIT_%=:\n\t"
+        "mbarrier.try_wait.parity.acquire.cluster.shared::cta.b64 p, [%0], %1;\n\t"
+        "@!p bra WAIT_%=;\n\t}" ::"r"(bar),
+        "r"(parity)
+        : "memory");
+}
+__device__ __forceinline__ void st_cluster_u32(uint32_t addr, int v) {
+    asm volatile("st.shared::cluster.u32 [%0], %1;" ::"r"(addr), "r"(v) : "memory");
 }
 __device__ __forceinline__ uint32_t cluster_rank() {
     uint32_t r;
@@ -351,6 +367,9 @@ __device__ __forceinline__ int mod_canon(int a, int p, int mq) {
 
 }  // namespace
 
+// NMOD moduli (16: FP64 class, b = 56 at K = 2048; 8: FP32 class, b = 25), F32: C is FP32 (the
+// FP32-class tiles, reduce-added in FP32 by the TMA unit) instead of FP64
+template <int NMOD, bool F32>
 __global__ void __launch_bounds__(THREADS, 1) crt_gemm_kernel(const __grid_constant__ CrtParams p) {
     extern __shared__ uint8_t smem_raw[];
     uint8_t* smem = (uint8_t*)(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
@@ -358,11 +377,14 @@ __global__ void __launch_bounds__(THREADS, 1) crt_gemm_kernel(const __grid_const
     __shared__ __align__(8) uint64_t acc_full[2], acc_empty[2];
     __shared__ uint32_t tmem_slot;
     __shared__ int slot_sh;
+    // dynamic tile scheduler: the leader's producer claims pair tiles from a global counter and
+    // publishes them in a ring in both CTAs (late-starting pairs simply claim fewer tiles)
+    __shared__ int tile_ring[RING];
+    __shared__ __align__(8) uint64_t ring_full[RING], ring_empty[RING];
 
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     const uint32_t crank = cluster_rank();
-    const int cid = (int)cluster_id(), ncl = (int)num_clusters();
-    const int N = p.c.nmod;
+    constexpr int N = NMOD;
     const int KB = p.nb / BK;
 
     if (threadIdx.x == 0) {
@@ -373,6 +395,11 @@ __global__ void __launch_bounds__(THREADS, 1) crt_gemm_kernel(const __grid_const
         for (int i = 0; i < 2; ++i) {
             mbar_init(su32(&acc_full[i]), 1);
             mbar_init(su32(&acc_empty[i]), 2 * EPI_WARPS);  // every epilogue warp of the pair
+        }
+        for (int i = 0; i < RING; ++i) {
+            mbar_init(su32(&ring_full[i]), 1);  // the leader producer's publish
+            // readers: leader MMA + CTA-1 producer + every epilogue warp of the pair (leader's barrier)
+            mbar_init(su32(&ring_empty[i]), 2 + 2 * EPI_WARPS);
         }
         asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
         asm volatile("prefetch.tensormap [%0];" ::"l"((uint64_t)&p.a) : "memory");
@@ -397,10 +424,33 @@ __global__ void __launch_bounds__(THREADS, 1) crt_gemm_kernel(const __grid_const
     long long pw_accempty = 0, pw_full = 0, pw_accfull = 0, pw_resid = 0, pw_recon = 0;
 #endif
 
+    // ring slot i % RING: wait for the published tile index, then release the slot to the leader
+    auto ring_take = [&](int i, bool release) {
+        const int s = i % RING;
+        mbar_wait_cl(su32(&ring_full[s]), (uint32_t)(i / RING) & 1u);
+        const int t = tile_ring[s];
+        if (release) mbar_arrive_cluster(cluster_addr(su32(&ring_empty[s]), 0));
+        return t;
+    };
+
     if (warp == 0 && lane == 0) {
         // ---------------- TMA producer: per tile, per modulus, K in 128-byte blocks
         uint32_t it = 0;
-        for (int tile = cid; tile < p.total; tile += ncl) {
+        for (int i = 0;; ++i) {
+            int tile;
+            if (crank == 0) {  // claim the next pair tile and publish it to both CTAs
+                const int s = i % RING;
+                mbar_wait(su32(&ring_empty[s]), ((uint32_t)(i / RING) & 1u) ^ 1u);
+                tile = atomicAdd(p.tile_counter, 1);
+                if (tile >= p.total) tile = -1;
+                tile_ring[s] = tile;
+                st_cluster_u32(cluster_addr(su32(&tile_ring[s]), 1), tile);
+                mbar_arrive_cluster(su32(&ring_full[s]));
+                mbar_arrive_cluster(cluster_addr(su32(&ring_full[s]), 1));
+            } else {
+                tile = ring_take(i, true);
+            }
+            if (tile < 0) break;
             int job, bi, bj;
             tile_coords(p, tile, job, bi, bj);
             const OzJob jb = p.jobs[job];
@@ -422,7 +472,8 @@ __global__ void __launch_bounds__(THREADS, 1) crt_gemm_kernel(const __grid_const
     } else if (warp == 1 && lane == 0 && crank == 0) {
         // ---------------- MMA issuer (leader CTA): one accumulator per modulus, two in flight
         uint32_t it = 0, g = 0;
-        for (int tile = cid; tile < p.total; tile += ncl) {
+        for (int i = 0;; ++i) {
+            if (ring_take(i, true) < 0) break;
             for (int t = 0; t < N; ++t, ++g) {
                 const uint32_t buf = g & 1u;
                 { PROF_T0();
@@ -460,7 +511,7 @@ __global__ void __launch_bounds__(THREADS, 1) crt_gemm_kernel(const __grid_const
         const uint32_t tl = ((uint32_t)(q * 32) << 16) + (uint32_t)(h * 128);
         const uint32_t ae0 = cluster_addr(su32(&acc_empty[0]), 0);
         const uint32_t stg_s = su32(smem + STAGES * STAGE_BYTES + (warp - 4) * STG_WARP);
-        const int NP = N / 2;
+        constexpr int NP = N / 2;
         uint32_t g = 0;       // accumulator-buffer counter (one per modulus)
         uint32_t nred = 0;    // C reduce-adds issued by this warp (staging-buffer parity)
         // the previous tile, whose reconstruction is pending
@@ -470,11 +521,10 @@ __global__ void __launch_bounds__(THREADS, 1) crt_gemm_kernel(const __grid_const
         const int* pv_ecol = nullptr;
 
         // reconstruct groups gi (8 columns each) of the pending tile: X = sum_j R_j w_j - q M, scaled
-        auto load_group = [&](int gi, uint4 (&w)[CRT_NMAX / 2]) {
+        auto load_group = [&](int gi, uint4 (&w)[NP]) {
             const uint8_t* src = scr0 + (size_t)pv_half * CRT_HALF_BYTES + scr_off(0, h, gi >> 2, gi & 3, r);
 #pragma unroll
-            for (int jj = 0; jj < CRT_NMAX / 2; ++jj)
-                if (jj < NP) w[jj] = __ldcs((const uint4*)(src + (size_t)jj * SCR_J_STRIDE));  // last use
+            for (int jj = 0; jj < NP; ++jj) w[jj] = __ldcs((const uint4*)(src + (size_t)jj * SCR_J_STRIDE));  // last use
         };
         // L2 prefetch of groups [g0, g1) of the pending tile (all 128 rows of this column half: one
         // 2 KB bulk prefetch per moduli pair and group, issued by one warp of the half)
@@ -486,24 +536,22 @@ __global__ void __launch_bounds__(THREADS, 1) crt_gemm_kernel(const __grid_const
                         asm volatile("cp.async.bulk.prefetch.L2.global [%0], 2048;" ::"l"(src) : "memory");
                     }
         };
-        auto recon = [&](int gi, const uint4 (&w)[CRT_NMAX / 2]) {
+        auto recon = [&](int gi, const uint4 (&w)[NP]) {
             const int col0 = (gi >> 2) * 32 + (gi & 3) * 8;
             double sh[8], sl[8];
 #pragma unroll
             for (int v = 0; v < 8; ++v) sh[v] = sl[v] = 0.0;
 #pragma unroll
-            for (int jj = 0; jj < CRT_NMAX / 2; ++jj) {
-                if (jj < NP) {
-                    const double Hj = p.c.H[jj], Lj = p.c.L[jj];
-                    const uint32_t wv[4] = {w[jj].x, w[jj].y, w[jj].z, w[jj].w};
+            for (int jj = 0; jj < NP; ++jj) {
+                const double Hj = p.c.H[jj], Lj = p.c.L[jj];
+                const uint32_t wv[4] = {w[jj].x, w[jj].y, w[jj].z, w[jj].w};
 #pragma unroll
-                    for (int v = 0; v < 8; ++v) {
-                        // 2^52 + R exactly (R in the low mantissa bits), minus 2^52
-                        const uint32_t Rv = (v & 1) ? (wv[v >> 1] >> 16) : (wv[v >> 1] & 0xffffu);
-                        const double d = __hiloint2double(0x43300000, (int)Rv) - 4503599627370496.0;
-                        sh[v] = fma(d, Hj, sh[v]);  // exact
-                        sl[v] = fma(d, Lj, sl[v]);
-                    }
+                for (int v = 0; v < 8; ++v) {
+                    // 2^52 + R exactly (R in the low mantissa bits), minus 2^52
+                    const uint32_t Rv = (v & 1) ? (wv[v >> 1] >> 16) : (wv[v >> 1] & 0xffffu);
+                    const double d = __hiloint2double(0x43300000, (int)Rv) - 4503599627370496.0;
+                    sh[v] = fma(d, Hj, sh[v]);  // exact
+                    sl[v] = fma(d, Lj, sl[v]);
                 }
             }
             // stage -out in the warp's 32 x 8 box (64-byte swizzle: 16-byte chunk k of row l at
@@ -513,32 +561,53 @@ __global__ void __launch_bounds__(THREADS, 1) crt_gemm_kernel(const __grid_const
                 if (lane == 0) asm volatile("cp.async.bulk.wait_group.read 1;" ::: "memory");
                 __syncwarp();
             }
+            double o[8];
 #pragma unroll
-            for (int v = 0; v < 8; v += 2) {
-                double o[2];
+            for (int v = 0; v < 8; ++v) {
+                const double qm = rint((sh[v] + sl[v]) * p.c.invM);
+                const double X = fma(-qm, p.c.Mh, sh[v]) + fma(-qm, p.c.Ml, sl[v]);
+                o[v] = (p.store ? X : -X) * pv_rs * exp2i(__ldg(pv_ecol + col0 + v) - p.c.bits);
+            }
+            if constexpr (F32) {  // 32 x 8 FP32 box, rows of 32 bytes (no swizzle)
+                const uint32_t a = sb + (uint32_t)lane * 32u;
+                asm volatile("st.shared.v4.f32 [%0], {%1, %2, %3, %4};" ::"r"(a), "f"((float)o[0]), "f"((float)o[1]),
+                             "f"((float)o[2]), "f"((float)o[3])
+                             : "memory");
+                asm volatile("st.shared.v4.f32 [%0], {%1, %2, %3, %4};" ::"r"(a + 16u), "f"((float)o[4]), "f"((float)o[5]),
+                             "f"((float)o[6]), "f"((float)o[7])
+                             : "memory");
+            } else {
 #pragma unroll
-                for (int u = 0; u < 2; ++u) {
-                    const double qm = rint((sh[v + u] + sl[v + u]) * p.c.invM);
-                    const double X = fma(-qm, p.c.Mh, sh[v + u]) + fma(-qm, p.c.Ml, sl[v + u]);
-                    o[u] = -(X * pv_rs * exp2i(__ldg(pv_ecol + col0 + v + u) - p.c.bits));
+                for (int v = 0; v < 8; v += 2) {
+                    const uint32_t a = sb + (uint32_t)lane * 64u + ((uint32_t)((v >> 1) ^ ((lane >> 1) & 3)) << 4);
+                    asm volatile("st.shared.v2.f64 [%0], {%1, %2};" ::"r"(a), "d"(o[v]), "d"(o[v + 1]) : "memory");
                 }
-                const uint32_t a = sb + (uint32_t)lane * 64u + ((uint32_t)((v >> 1) ^ ((lane >> 1) & 3)) << 4);
-                asm volatile("st.shared.v2.f64 [%0], {%1, %2};" ::"r"(a), "d"(o[0]), "d"(o[1]) : "memory");
             }
             asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
             __syncwarp();
             if (lane == 0) {
-                asm volatile("cp.reduce.async.bulk.tensor.2d.global.shared::cta.add.tile.bulk_group [%0, {%2, %3}], [%1];" ::"l"(
-                                 (uint64_t)&p.cmap),
-                             "r"(sb), "r"(pv_ccol0 + col0), "r"(pv_crow0)
-                             : "memory");
+                if (p.store)
+                    asm volatile("cp.async.bulk.tensor.2d.global.shared::cta.bulk_group [%0, {%2, %3}], [%1];" ::"l"(
+                                     (uint64_t)&p.cmap),
+                                 "r"(sb), "r"(pv_ccol0 + col0), "r"(pv_crow0)
+                                 : "memory");
+                else
+                    asm volatile("cp.reduce.async.bulk.tensor.2d.global.shared::cta.add.tile.bulk_group [%0, {%2, %3}], [%1];" ::"l"(
+                                     (uint64_t)&p.cmap),
+                                 "r"(sb), "r"(pv_ccol0 + col0), "r"(pv_crow0)
+                                 : "memory");
                 asm volatile("cp.async.bulk.commit_group;" ::: "memory");
             }
             ++nred;
         };
 
         int it_tile = 0;
-        for (int tile = cid; tile < p.total; tile += ncl, ++it_tile) {
+        for (;; ++it_tile) {
+            int tile = 0;
+            if (lane == 0) tile = ring_take(it_tile, false);
+            tile = __shfl_sync(0xffffffffu, tile, 0);
+            if (lane == 0) mbar_arrive_cluster(cluster_addr(su32(&ring_empty[it_tile % RING]), 0));
+            if (tile < 0) break;
             int job, bi, bj;
             tile_coords(p, tile, job, bi, bj);
             uint8_t* const scr = scr0 + (size_t)(it_tile & 1) * CRT_HALF_BYTES;
@@ -624,7 +693,7 @@ __global__ void __launch_bounds__(THREADS, 1) crt_gemm_kernel(const __grid_const
                 if (pv) {
                     PROF_T0();
                     const int g0 = (j * 16) / NP, g1 = ((j + 1) * 16) / NP;
-                    uint4 wa[CRT_NMAX / 2], wb[CRT_NMAX / 2];
+                    uint4 wa[NP], wb[NP];
                     load_group(g0, wa);
                     for (int gi = g0; gi < g1; gi += 2) {
                         if (gi + 1 < g1) load_group(gi + 1, wb);
@@ -642,13 +711,14 @@ __global__ void __launch_bounds__(THREADS, 1) crt_gemm_kernel(const __grid_const
             pv_half = it_tile & 1;
             pv_rs = ldexp(1.0, p.exps[jb.m * p.nb + grow] - p.c.bits);
             pv_ecol = p.exps + (size_t)jb.n * p.nb + bj * BN + h * 128;
-            pv_crow0 = (int)(((const double*)jb.C - p.cbase) / p.nb) + bi * 256 + (int)crank * BM + q * 32;
+            pv_crow0 = (int)(((const char*)jb.C - (const char*)p.cbase) / ((size_t)p.nb * (F32 ? 4 : 8))) + bi * 256 +
+                       (int)crank * BM + q * 32;
             pv_ccol0 = bj * BN + h * 128;
         }
         if (pv) {  // drain: the last tile's reconstruction
             PROF_T0();
             prefetch_groups(0, 16);
-            uint4 wa[CRT_NMAX / 2], wb[CRT_NMAX / 2];
+            uint4 wa[NP], wb[NP];
             load_group(0, wa);
             for (int gi = 0; gi < 16; gi += 2) {
                 load_group(gi + 1, wb);
@@ -709,16 +779,16 @@ static bool crt_map(CUtensorMap* m, const int8_t* base, uint64_t planes, uint64_
               CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
 }
 
-static bool crt_cmap(CUtensorMap* m, const double* base, uint64_t rows, uint64_t cols) {
+static bool crt_cmap(CUtensorMap* m, const void* base, uint64_t rows, uint64_t cols, bool f32) {
     auto fn = crt_encode();
     if (!fn) return false;
     cuuint64_t dims[2] = {cols, rows};
-    cuuint64_t strides[1] = {cols * 8};
+    cuuint64_t strides[1] = {cols * (f32 ? 4 : 8)};
     cuuint32_t box[2] = {8, 32};
     cuuint32_t es[2] = {1, 1};
-    return fn(m, CU_TENSOR_MAP_DATA_TYPE_FLOAT64, 2, const_cast<double*>(base), dims, strides, box, es,
-              CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_64B, CU_TENSOR_MAP_L2_PROMOTION_NONE,
-              CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
+    return fn(m, f32 ? CU_TENSOR_MAP_DATA_TYPE_FLOAT32 : CU_TENSOR_MAP_DATA_TYPE_FLOAT64, 2, const_cast<void*>(base), dims,
+              strides, box, es, CU_TENSOR_MAP_INTERLEAVE_NONE, f32 ? CU_TENSOR_MAP_SWIZZLE_NONE : CU_TENSOR_MAP_SWIZZLE_64B,
+              CU_TENSOR_MAP_L2_PROMOTION_NONE, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
 }
 
 static int sm_count() {
@@ -737,20 +807,24 @@ bool crt_available() { return crt_encode() != nullptr; }
 
 cudaError_t crt_gemm_launch(const CrtArgs& a, int njobs, cudaStream_t s) {
     if (njobs <= 0) return cudaSuccess;
-    // the reconstruction slots are tuned for 8 moduli pairs: the kernel is built for N = 16
-    if (a.nb % 256 || a.nb > 8192 || a.c.nmod != CRT_NMAX || !a.scratch || !a.slot_flags) return cudaErrorInvalidValue;
-    static bool attr = false;
-    if (!attr) {
-        cudaError_t e = cudaFuncSetAttribute(crt_gemm_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, SMEM);
+    // instantiations: 16 moduli with an FP64 C (FP64 class); 8 moduli (FP32 class) with an FP32 C
+    // (trailing update) or an FP64 C (the FP32-class TRSM product into the FP64 panel buffer)
+    if (a.nb % 256 || a.nb > 8192 || !a.scratch || !a.slot_flags) return cudaErrorInvalidValue;
+    if (!((a.c.nmod == 16 && !a.c_f32) || a.c.nmod == 8)) return cudaErrorInvalidValue;
+    const int ki = a.c.nmod == 16 ? 0 : a.c_f32 ? 1 : 2;
+    auto kern = ki == 0 ? crt_gemm_kernel<16, false> : ki == 1 ? crt_gemm_kernel<8, true> : crt_gemm_kernel<8, false>;
+    static bool attr[3] = {false, false, false};
+    if (!attr[ki]) {
+        cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, SMEM);
         if (e != cudaSuccess) return e;
-        attr = true;
+        attr[ki] = true;
     }
     CrtParams p;
     memset(&p, 0, sizeof p);
     const uint64_t rows = (uint64_t)a.nt * a.nb;
     if (!crt_map(&p.a, a.planes, (uint64_t)a.c.nmod, rows, a.nb, a.plane_stride, BM) ||
         !crt_map(&p.b, a.planes, (uint64_t)a.c.nmod, rows, a.nb, a.plane_stride, BN / 2) || !a.cbase ||
-        !crt_cmap(&p.cmap, a.cbase, a.crows, a.nb))
+        !crt_cmap(&p.cmap, a.cbase, a.crows, a.nb, a.c_f32 != 0))
         return cudaErrorInvalidValue;
     p.cbase = a.cbase;
     p.jobs = a.jobs;
@@ -761,6 +835,9 @@ cudaError_t crt_gemm_launch(const CrtArgs& a, int njobs, cudaStream_t s) {
     p.nb = a.nb;
     p.tiles_n = a.nb / BN;
     p.lower = a.lower;
+    p.store = a.store;
+    p.tile_counter = a.counter;
+    if (!a.counter) return cudaErrorInvalidValue;
     p.tiles_per_job = a.lower ? p.tiles_n * (p.tiles_n + 1) / 2 : p.tiles_n * p.tiles_n;
     p.c = a.c;
     const long long total = (long long)njobs * p.tiles_per_job;
@@ -784,7 +861,7 @@ cudaError_t crt_gemm_launch(const CrtArgs& a, int njobs, cudaStream_t s) {
     at[0].val.clusterDim.z = 1;
     cfg.attrs = at;
     cfg.numAttrs = 1;
-    return cudaLaunchKernelEx(&cfg, crt_gemm_kernel, p);
+    return cudaLaunchKernelEx(&cfg, kern, p);
 }
 
 }  // namespace mpgeo

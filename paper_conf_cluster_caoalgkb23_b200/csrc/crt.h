@@ -44,9 +44,12 @@ struct CrtArgs {
     uint8_t* scratch;      // residue staging: crt_scratch_slots() x CRT_SLOT_BYTES
     int* slot_flags;       // crt_scratch_slots() ints, zero-initialised
     CrtConst c;            // copied into the launch parameters
-    const double* cbase;   // C tiles lie inside [cbase, cbase + crows * nb) at whole-row offsets
-    uint64_t crows;        //   (the FP64 view of the tile pool; C is updated by TMA reduce-add)
+    const void* cbase;     // C tiles lie inside [cbase, cbase + crows * nb) at whole-row offsets
+    uint64_t crows;        //   (a view of the tile pool in C's type; C is updated by TMA reduce-add)
     int max_pairs;         // persistent grid in CTA pairs (0: one pair per 2 SMs)
+    int c_f32 = 0;         // 0: FP64 C (nmod = 16 or 8); 1: FP32 C (nmod = 8, FP32-class update)
+    int store = 0;         // 1: C = P_m P_n^T (overwrite), 0: C -= P_m P_n^T
+    int* counter = nullptr;  // tile-scheduler counter of this launch (device int, zero at launch)
 };
 // one CTA's 128 x 256 combined residues (N/2 x 2 bytes each) for two tiles (the epilogue reconstructs
 // tile T-1 while it reduces tile T)

@@ -55,6 +55,11 @@ struct mp_handle {
                         // both on INT8 tensor cores; 0 = DMMA
     int matern_table = 1;  // general nu: tabulated correlation (1) or direct K_nu per entry (0)
     int ozaki32 = 0;    // 1: FP32-class GEMM on INT8 tensor cores (first 4 slices); 0: 3xTF32 tcgen05 (default)
+    int crt32 = 0;      // with the CRT FP64 engine: FP32-class GEMM as 8 INT8 GEMMs (CRT-8, FP32 C); opt-in:
+                        // measured slower than 3xTF32 inside the evaluation (profiles/r01/README.md)
+    int crt_trsm = 1;   // with the CRT FP64 engine: TRSM of FP32/FP16-class tiles as the FP32-class product
+                        // A_mk W^T, W = L~_kk^-1 (CRT-8), instead of the blocked DMMA substitution
+    int reserve_pairs = 6;   // lookahead: CTA pairs the persistent update kernels leave to the panel stream
     cudaStream_t pstream = nullptr;
     std::vector<cudaEvent_t> sync_ev;
     // profiling (mp_set_profiling): event pairs per launch, resolved in mp_get_profile
@@ -67,8 +72,8 @@ struct mp_handle {
 
 struct Regions {
     size_t total = 0;
-    size_t inputs = 0, p64 = 0, p16 = 0, phi = 0, plo = 0, ltilde = 0, wbuf = 0, wbuf2 = 0, oz = 0, ozexp = 0,
-           wdiag = 0, mtab = 0, crt = 0, crtflags = 0;
+    size_t inputs = 0, p64 = 0, p16 = 0, phi = 0, plo = 0, oz32 = 0, ltilde = 0, wbuf = 0, wbuf2 = 0, oz = 0, ozexp = 0,
+           wdiag = 0, mtab = 0, crt = 0, crtflags = 0, crtctr = 0;
     size_t vec_r = 0, vec_y = 0, partials = 0, norms = 0, ctrl = 0, ctrl_bytes = 0;
     std::vector<size_t> tile_off;  // per (m*nt+k), SIZE_MAX if not stored here
     size_t pool = 0;               // start of the tile pool
@@ -123,6 +128,9 @@ struct mp_matrix {
     } while (0)
 
 static size_t align_up(size_t v, size_t a) { return (v + a - 1) / a * a; }
+// CRT launches of one factorisation: <= 4 update launches (two parts x SYRK / GEMM) + 1 FP32-class +
+// 1 TRSM per panel
+static size_t crt_counters(int nt) { return 8 * (size_t)nt + 64; }
 constexpr int MT_PIECES_MAX = 512;
 static int ceil_div(int a, int b) { return (a + b - 1) / b; }
 
@@ -172,14 +180,20 @@ static Regions layout(const mp_matrix* A, const uint8_t* storage) {
     // two sets of panel buffers (panel parity) so panel k+1 can be produced while update k reads panel k
     R.p64 = take(2 * (size_t)nt * nb2 * 8);
     R.p16 = take(2 * (size_t)nt * nb2 * 2);
-    R.phi = take(2 * (size_t)nt * nb2 * 4);
-    R.plo = take(2 * (size_t)nt * nb2 * 4);
     // int8 operand planes of the FP64-class engine, two sets: 8 slices (splitting) or 16 residues (CRT)
     const bool crt = A->h && A->h->ozaki == 16 && A->nb % 256 == 0;
+    // FP32-class operands: TF32 hi/lo pairs (3xTF32), or with the CRT engine 8 residue planes (CRT-8)
+    const bool crt32 = crt && A->h->crt32;
+    if (crt32 || (crt && A->h->crt_trsm)) R.oz32 = take(2 * (size_t)nt * nb2 * 8);
+    if (!crt32) {
+        R.phi = take(2 * (size_t)nt * nb2 * 4);
+        R.plo = take(2 * (size_t)nt * nb2 * 4);
+    }
     R.oz = take(2 * (size_t)nt * nb2 * (crt ? CRT_NMAX : 8));
     if (crt) {  // CRT engine: per-CTA residue staging slots + their busy flags
         R.crt = take((size_t)crt_scratch_slots() * CRT_SLOT_BYTES);
         R.crtflags = take((size_t)crt_scratch_slots() * sizeof(int));
+        R.crtctr = take(crt_counters(nt) * sizeof(int));
     }
     R.ozexp = take(2 * (size_t)nt * A->nb * 4);    // per-row exponents
     R.tile_off.assign((size_t)nt * nt, SIZE_MAX);
@@ -288,6 +302,9 @@ mp_status mp_init(int device, int rank, int nranks, int P, int Q, const uint8_t*
     if (const char* e = getenv("MPGEO_LOOKAHEAD")) h->lookahead = atoi(e);
     if (const char* e = getenv("MPGEO_OZAKI")) h->ozaki = atoi(e);
     if (const char* e = getenv("MPGEO_OZAKI32")) h->ozaki32 = atoi(e);
+    if (const char* e = getenv("MPGEO_CRT32")) h->crt32 = atoi(e);
+    if (const char* e = getenv("MPGEO_CRT_TRSM")) h->crt_trsm = atoi(e);
+    if (const char* e = getenv("MPGEO_RESERVE_PAIRS")) h->reserve_pairs = std::max(0, atoi(e));
     if (const char* e = getenv("MPGEO_MATERN_TABLE")) h->matern_table = atoi(e);
     auto fail = [&](mp_status s) {
         if (h->own_stream && h->stream) cudaStreamDestroy(h->stream);
@@ -383,7 +400,7 @@ mp_status mp_handle_config(const mp_handle* h, int* tc, int* lookahead, int* oza
     if (tc) *tc = (h->tc_mode != 0 && tc_gemm_available()) ? 1 : 0;
     if (lookahead) *lookahead = h->lookahead;
     if (ozaki)
-        *ozaki = (h->ozaki == 16 && crt_available()) ? 16
+        *ozaki = (h->ozaki == 16 && crt_available()) ? (16 + (h->crt32 ? 200 : 0))
                  : (h->ozaki == 8 && ozaki_available()) ? (8 + (h->ozaki32 ? 100 : 0)) : 0;
     return MP_OK;
 }
@@ -729,14 +746,24 @@ static mp_status plan_potrf(mp_handle* h, mp_matrix* A, const uint8_t* km, const
     const double* const cpool64 = A->at<double>(A->R.pool);  // FP64 view of the pool (CRT epilogue C map)
     const uint64_t crows64 = (A->R.total - A->R.pool) / ((size_t)nb * 8);
     const bool crt = h->ozaki == 16 && crt_available() && nb % 256 == 0 && A->R.crt;
-    CrtConst crtc;
+    CrtConst crtc, crtc32;
     if (crt && !crt_constants(CRT_NMAX, nb, &crtc)) FAIL(h, MP_ERR_ARG, "CRT constants for nb=%d", nb);
+    // FP32 class on the CRT engine: 8 moduli (b = 25 operand bits at nb = 2048), FP32 C
+    const bool crt32 = crt && h->crt32 && A->R.oz32 && use_tc;
+    // low-precision-class TRSMs as CRT-8 products with the inverse factor (FP32 TRSM there)
+    const bool ctrsm = crt && h->crt_trsm && A->R.oz32 && nb % 32 == 0;
+    if ((crt32 || ctrsm) && !crt_constants(8, nb, &crtc32)) FAIL(h, MP_ERR_ARG, "CRT-8 constants for nb=%d", nb);
+    int8_t* const oz32b = (crt32 || ctrsm) ? A->at<int8_t>(A->R.oz32) : nullptr;
     // the 8-slice splitting engine: selected (8), or the fallback of the CRT engine when nb % 256 != 0
     const int ozS = !crt && (h->ozaki == 8 || h->ozaki == 16) && ozaki_available() && nb % 128 == 0 ? 8 : 0;
     const bool oz32 = ozS && h->ozaki32 && nb % 256 == 0;
     int8_t* const ozb = A->at<int8_t>(A->R.oz);
     uint8_t* const crt_scr = crt ? A->at<uint8_t>(A->R.crt) : nullptr;
     int* const crt_flags = crt ? A->at<int>(A->R.crtflags) : nullptr;
+    // one tile-scheduler counter per CRT launch of this call (zeroed by potrf_run)
+    int* const crt_ctr = crt ? A->at<int>(A->R.crtctr) : nullptr;
+    size_t ctr_next = 0;
+    auto next_ctr = [&]() -> int* { return ctr_next < crt_counters(nt) ? crt_ctr + ctr_next++ : nullptr; };
     int* const ozeb = A->at<int>(A->R.ozexp);
     auto K = [&](int m, int k) { return km[(size_t)m * nt + k]; };
     auto C = [&](int m, int k) { return cm[(size_t)m * nt + k]; };
@@ -746,6 +773,11 @@ static mp_status plan_potrf(mp_handle* h, mp_matrix* A, const uint8_t* km, const
     // ---- multi-rank exchange helpers; unused on one rank
     const bool dist = h->nranks > 1;
     const bool la = h->lookahead != 0;  // also multi-rank: exchange waits run on the panel stream
+    // persistent CRT grids: the update leaves reserve_pairs CTA pairs to the panel stream (lookahead)
+    int nsm = 148;
+    cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, h->device);
+    const int upd_pairs = la ? std::max(1, nsm / 2 - h->reserve_pairs) : 0;
+    const int pan_pairs = la ? std::max(1, h->reserve_pairs) : 0;
     const int R = h->nranks, me = h->rank;
     Comm& X = A->comm;
     auto ST = [&](int step) -> uint64_t { return (epoch << 24) + (uint64_t)(step + 2); };
@@ -911,7 +943,7 @@ static mp_status plan_potrf(mp_handle* h, mp_matrix* A, const uint8_t* km, const
             local_formats(k, m, need16, need32);
             if (use_tc) {
                 if (need16) t.p16 = p16 + (size_t)m * nb2;
-                if (need32 && !oz32) {
+                if (need32 && !oz32 && !crt32) {
                     t.hi = phi + (size_t)m * nb2;
                     t.lo = plo + (size_t)m * nb2;
                 }
@@ -923,26 +955,63 @@ static mp_status plan_potrf(mp_handle* h, mp_matrix* A, const uint8_t* km, const
             PanelTile* d_out = ar.push(pout);
             const int np = (int)pin.size();
             cur->push_back({[=](cudaStream_t s) { return panel_in_launch(d_in, np, (int64_t)nb2, s); }, C_CONV, 0});
-            // ---- 4. TRSM(m,k): L_mk = A_mk L~_kk^{-T}, FP64 arithmetic (reading C12'),
-            //      right-looking over 128-column blocks (X_j = X_j W_j^T) with the updates inside a
-            //      512-column outer block at K = 128 and across outer blocks at K = 512.
+            // ---- 4. TRSM(m,k): L_mk = A_mk L~_kk^{-T}.  FP64-class tiles: FP64 arithmetic (
+            //      reading C12'), right-looking over 128-column blocks (X_j = X_j W_j^T) with the updates
+            //      inside a 512-column outer block at K = 128 and across outer blocks at K = 512.
+            //      FP32/FP16-class tiles (the paper's FP32 TRSM) with ctrsm: 4b below.
+            std::vector<double*> dm;  // DMMA substitution targets (panel slots)
+            std::vector<int> lo;      // low-precision-class tiles (ctrsm)
+            for (auto& t : pin) {
+                const int m = (int)((t.p64 - p64) / (ptrdiff_t)nb2);
+                if (ctrsm && K(m, k) != MP_FP64) lo.push_back(m);
+                else dm.push_back(t.p64);
+            }
+            double* const islot = p64 + (size_t)k * nb2;  // panel slot k is free in panel k
+            if (!lo.empty()) {  // right-hand side I: its substitution gives L~_kk^-T
+                cur->push_back({[=](cudaStream_t s) { return identity_launch(islot, nb, s); }, C_TRSM, 0});
+                dm.push_back(islot);
+            }
             for (int J0 = 0; J0 < nb; J0 += OB) {
                 const int Jend = std::min(nb, J0 + OB), Jb = Jend - J0;
                 for (int j0 = J0; j0 < Jend; j0 += IB) {
                     const int jb = std::min(IB, Jend - j0), jend = j0 + jb;
                     std::vector<GemmJob> ja, jin;
-                    for (auto& t : pin) {
-                        ja.push_back(GemmJob{t.p64 + j0, wb2 + (size_t)(j0 / IB) * IB * IB, t.p64 + j0});
-                        if (Jend > jend) jin.push_back(GemmJob{t.p64 + j0, ltil + (size_t)jend * nb + j0, t.p64 + jend});
+                    for (double* x : dm) {
+                        ja.push_back(GemmJob{x + j0, wb2 + (size_t)(j0 / IB) * IB * IB, x + j0});
+                        if (Jend > jend) jin.push_back(GemmJob{x + j0, ltil + (size_t)jend * nb + j0, x + jend});
                     }
                     gemm(ja, nb, jb, jb, nb, IB, nb, 0, 1.0, 0.0, P64, false, C_TRSM, fnb * jb * jb);
                     gemm(jin, nb, Jend - jend, jb, nb, nb, nb, 0, -1.0, 1.0, P64, false, C_TRSM, 2.0 * fnb * (Jend - jend) * jb);
                 }
                 if (nb > Jend) {
                     std::vector<GemmJob> jo;
-                    for (auto& t : pin) jo.push_back(GemmJob{t.p64 + J0, ltil + (size_t)Jend * nb + J0, t.p64 + Jend});
+                    for (double* x : dm) jo.push_back(GemmJob{x + J0, ltil + (size_t)Jend * nb + J0, x + Jend});
                     gemm(jo, nb, nb - Jend, Jb, nb, nb, nb, 0, -1.0, 1.0, P64, false, C_TRSM, 2.0 * fnb * (nb - Jend) * Jb);
                 }
+            }
+            // ---- 4b. FP32/FP16-class TRSM as the FP32-class product L_mk = A_mk W^T with the inverse
+            //      factor W = L~_kk^-1 (its FP64 substitution above, transposed into the L~ buffer, which
+            //      the substitution no longer reads): both operands as 8 CRT residue planes (b = 25 bits
+            //      per row), one CRT-8 launch over the column with an FP64 C (store mode) into the panel
+            //      slots, where the conversions of step 5 pick the tiles up as before.
+            if (!lo.empty()) {
+                int8_t* const o32s = oz32b + set * nt * nb2 * 8;
+                double* const W = ltil;
+                cur->push_back({[=](cudaStream_t s) { return transpose_launch(islot, W, nb, s); }, C_TRSM, 0});
+                std::vector<CrtSplitItem> sp{CrtSplitItem{W, o32s + (size_t)k * nb2, oze + (size_t)k * nb, ozplane}};
+                std::vector<OzJob> tj;
+                for (int m : lo) {
+                    sp.push_back(CrtSplitItem{p64 + (size_t)m * nb2, o32s + (size_t)m * nb2, oze + (size_t)m * nb, ozplane});
+                    tj.push_back(OzJob{m, k, p64 + (size_t)m * nb2});
+                }
+                CrtSplitItem* dsp = ar.push(sp);
+                const int nsp = (int)sp.size();
+                cur->push_back({[=](cudaStream_t s) { return crt_split_launch(dsp, nsp, nb, crtc32, s); }, C_TRSM, 0});
+                OzJob* dj = ar.push(tj);
+                const int nj = (int)tj.size();
+                CrtArgs ca{dj, o32s, oze, ozplane, nb, nt, 0, crt_scr, crt_flags, crtc32, p64b, (uint64_t)2 * nt * nb,
+                           pan_pairs, 0, 1, next_ctr()};
+                cur->push_back({[=](cudaStream_t s) { return crt_gemm_launch(ca, nj, s); }, C_TRSM, 2.0 * fnb * fnb * fnb * nj});
             }
             fc.trsm += np * fnb * fnb * fnb;
             // ---- 5. panel out (K2)
@@ -981,7 +1050,7 @@ static mp_status plan_potrf(mp_handle* h, mp_matrix* A, const uint8_t* km, const
                 PullItem it{sendslot(o, sp, m), pubflag(o, sp, m), ST(k), p64 + (size_t)m * nb2, nullptr, nullptr,
                             nullptr, C(m, k), 0};
                 if (use_tc && n16) it.p16 = p16 + (size_t)m * nb2;
-                if (use_tc && n32 && !oz32) {
+                if (use_tc && n32 && !oz32 && !crt32) {
                     it.hi = phi + (size_t)m * nb2;
                     it.lo = plo + (size_t)m * nb2;
                 }
@@ -1014,6 +1083,23 @@ static mp_status plan_potrf(mp_handle* h, mp_matrix* A, const uint8_t* km, const
                 cur_push(Op{[=](cudaStream_t s) { return crt_split_launch(dsp, nsp, nb, crtc, s); }, C_CONV, 0});
             }
         }
+        if (crt32) {  // CRT-8 residue planes of every panel tile this GPU's FP32-class GEMMs read
+            std::vector<CrtSplitItem> sp;
+            int8_t* const o32s = oz32b + set * nt * nb2 * 8;
+            for (int m = k + 1; m < nt; ++m) {
+                bool need = false;
+                for (int n = k + 1; n < m && !need; ++n) need |= A->mine(m, n) && K(m, n) == MP_FP32;
+                for (int n = m + 1; n < nt && !need; ++n) need |= A->mine(n, m) && K(n, m) == MP_FP32;
+                // the row exponents are the same function of the panel tile as the 16-modulus split's
+                if (need)
+                    sp.push_back(CrtSplitItem{p64 + (size_t)m * nb2, o32s + (size_t)m * nb2, oze + (size_t)m * nb, ozplane});
+            }
+            if (!sp.empty()) {
+                CrtSplitItem* dsp = ar.push(sp);
+                const int nsp = (int)sp.size();
+                cur_push(Op{[=](cudaStream_t s) { return crt_split_launch(dsp, nsp, nb, crtc32, s); }, C_CONV, 0});
+            }
+        }
         if (ozS) {
             std::vector<OzSplitItem> sp;
             for (int m = k + 1; m < nt; ++m) {
@@ -1036,7 +1122,7 @@ static mp_status plan_potrf(mp_handle* h, mp_matrix* A, const uint8_t* km, const
         cur = part == 0 ? &nxt[k] : &rst[k];
         std::vector<GemmJob> syrk, g64, g32, g16;
         std::vector<TcJob> t32, t16;
-        std::vector<OzJob> o32;
+        std::vector<OzJob> o32, c32;
         for (int m = k + 1; m < nt; ++m) {
             if (A->mine(m, m) && ((m == k + 1) == (part == 0))) {
                 syrk.push_back(GemmJob{p64 + (size_t)m * nb2, p64 + (size_t)m * nb2, A->tile(m, m)});
@@ -1050,6 +1136,8 @@ static mp_status plan_potrf(mp_handle* h, mp_matrix* A, const uint8_t* km, const
                     g64.push_back(GemmJob{p64 + (size_t)m * nb2, p64 + (size_t)n * nb2, A->tile(m, n)});
                 } else if (oz32 && p == MP_FP32) {
                     o32.push_back(OzJob{m, n, A->tile(m, n)});
+                } else if (crt32 && p == MP_FP32) {
+                    c32.push_back(OzJob{m, n, A->tile(m, n)});
                 } else if (use_tc) {
                     (p == MP_FP32 ? t32 : t16).push_back(TcJob{m, n, (float*)A->tile(m, n)});
                 } else {
@@ -1070,8 +1158,9 @@ static mp_status plan_potrf(mp_handle* h, mp_matrix* A, const uint8_t* km, const
                 OzJob* dj = ar.push(oj);
                 const int nj = (int)oj.size();
                 if (crt) {
-                    // 64 of the 74 CTA pairs: SMs stay free for the panel stream's POTRF/TRSM (lookahead)
-                    CrtArgs ca{dj, ozs, oze, ozplane, nb, nt, lower, crt_scr, crt_flags, crtc, cpool64, crows64, la ? 64 : 0};
+                    // upd_pairs of the SM/2 CTA pairs: SMs stay free for the panel stream's POTRF/TRSM (lookahead)
+                    CrtArgs ca{dj, ozs, oze, ozplane, nb, nt, lower, crt_scr, crt_flags, crtc, cpool64, crows64, upd_pairs, 0, 0,
+                               next_ctr()};
                     cur_push(Op{[=](cudaStream_t s) { return crt_gemm_launch(ca, nj, s); }, C_UPD64,
                                 (lower ? f3 : 2 * f3) * nj});
                 } else {
@@ -1092,6 +1181,13 @@ static mp_status plan_potrf(mp_handle* h, mp_matrix* A, const uint8_t* km, const
             const int nj = (int)o32.size();
             OzArgs oa{dj, ozs, oze, ozplane, nb, nt, 4, 0, 1};
             cur_push(Op{[=](cudaStream_t s) { return ozaki_gemm_launch(oa, nj, s); }, C_UPD32, 2 * f3 * nj});
+        }
+        if (!c32.empty()) {  // FP32 class as 8 INT8 GEMMs (CRT-8), FP32 C
+            OzJob* dj = ar.push(c32);
+            const int nj = (int)c32.size();
+            int8_t* const o32s = oz32b + set * nt * nb2 * 8;
+            CrtArgs ca{dj, o32s, oze, ozplane, nb, nt, 0, crt_scr, crt_flags, crtc32, cpool, crows, upd_pairs, 1, 0, next_ctr()};
+            cur_push(Op{[=](cudaStream_t s) { return crt_gemm_launch(ca, nj, s); }, C_UPD32, 2 * f3 * nj});
         }
         if (!t32.empty()) {
             TcJob* dj = ar.push(t32);
@@ -1162,6 +1258,7 @@ static mp_status potrf_run(mp_handle* h, mp_matrix* A, const uint8_t* km, const 
     const int big = INT_MAX;
     CK(h, cudaMemcpyAsync(h->d_info, &big, sizeof(int), cudaMemcpyHostToDevice, h->stream));
     if (A->R.crtflags) CK(h, cudaMemsetAsync(A->ws + A->R.crtflags, 0, (size_t)crt_scratch_slots() * sizeof(int), h->stream));
+    if (A->R.crtctr) CK(h, cudaMemsetAsync(A->ws + A->R.crtctr, 0, crt_counters(A->nt) * sizeof(int), h->stream));
     Arena ar;
     ar.dev_base = A->ws + A->R.ctrl;
     std::vector<Op> ops;

@@ -83,6 +83,9 @@ cudaError_t panel_out_launch(const PanelTile* t, int ntiles, int64_t elems, cuda
 cudaError_t round_copy_launch(const double* src, double* dst, int64_t elems, int prec, cudaStream_t s);
 // zero the strictly upper triangle of an nb x nb row-major tile
 cudaError_t zero_upper_launch(double* A, int nb, cudaStream_t s);
+// A = I (nb x nb FP64); dst = src^T (nb x nb FP64, nb % 32 == 0)
+cudaError_t identity_launch(double* A, int nb, cudaStream_t s);
+cudaError_t transpose_launch(const double* src, double* dst, int nb, cudaStream_t s);
 
 // ---- K8: solve and reductions (solve.cu)
 // y[0..nb) = L^{-1} r[0..nb) for one FP64 lower tile (ld nb), rows >= nreal are identity pads

@@ -99,8 +99,15 @@ mp_status mp_test_ozaki_gemm(const double* d_panel, double* d_C, int nb, int nt,
     return (e == cudaSuccess && e2 == cudaSuccess) ? MP_OK : MP_ERR_CUDA;
 }
 
-mp_status mp_test_crt_gemm(const double* d_panel, double* d_C, int nb, int nt, int m, int n, int nmod, int lower) {
+mp_status mp_test_crt_gemm(const double* d_panel, void* d_C, int nb, int nt, int m, int n, int nmod, int lower) {
+    // nmod = 8: the FP32-class update instantiation (FP32 C)
+    return mp_test_crt_gemm_ex(d_panel, d_C, nb, nt, m, n, nmod, lower, nmod == 8, 0);
+}
+
+mp_status mp_test_crt_gemm_ex(const double* d_panel, void* d_C, int nb, int nt, int m, int n, int nmod, int lower,
+                              int c_f32, int store) {
     if (!crt_available()) return MP_ERR_UNSUPPORTED;
+    const int f32 = c_f32;
     CrtConst c;
     if (!crt_constants(nmod, nb, &c)) return MP_ERR_ARG;
     const int64_t plane = (int64_t)nt * nb * nb;
@@ -113,9 +120,9 @@ mp_status mp_test_crt_gemm(const double* d_panel, double* d_C, int nb, int nt, i
     int* flags = nullptr;
     if (cudaMalloc(&pl, plane * nmod) || cudaMalloc(&ex, sizeof(int) * nt * nb) ||
         cudaMalloc(&it, sizeof(CrtSplitItem) * nt) || cudaMalloc(&dj, sizeof(OzJob)) ||
-        cudaMalloc(&scr, (size_t)slots * CRT_SLOT_BYTES) || cudaMalloc(&flags, sizeof(int) * slots))
+        cudaMalloc(&scr, (size_t)slots * CRT_SLOT_BYTES) || cudaMalloc(&flags, sizeof(int) * (slots + 1)))
         return MP_ERR_CUDA;
-    cudaMemset(flags, 0, sizeof(int) * slots);
+    cudaMemset(flags, 0, sizeof(int) * (slots + 1));  // slot flags + the tile counter
     std::vector<CrtSplitItem> h(nt);
     for (int t = 0; t < nt; ++t)
         h[t] = CrtSplitItem{d_panel + (size_t)t * nb * nb, pl + (size_t)t * nb * nb, ex + (size_t)t * nb, plane};
@@ -123,7 +130,7 @@ mp_status mp_test_crt_gemm(const double* d_panel, double* d_C, int nb, int nt, i
     OzJob j{m, n, d_C};
     cudaMemcpy(dj, &j, sizeof j, cudaMemcpyHostToDevice);
     cudaError_t e = crt_split_launch(it, nt, nb, c, 0);
-    CrtArgs a{dj, pl, ex, plane, nb, nt, lower, scr, flags, c, d_C, (uint64_t)nb, 0};
+    CrtArgs a{dj, pl, ex, plane, nb, nt, lower, scr, flags, c, d_C, (uint64_t)nb, 0, f32, store, flags + slots};
     if (e == cudaSuccess) e = crt_gemm_launch(a, 1, 0);
     cudaError_t e2 = cudaDeviceSynchronize();
     if (const char* path = getenv("MPGEO_CRT_DUMP")) {  // debugging aid: planes, exponents, 8 scratch slots
@@ -163,9 +170,9 @@ mp_status mp_bench_fp64_engine(int engine, int nb, int nt, int njobs, int nmod, 
     const int slots = crt_scratch_slots();
     if (cudaMalloc(&P, plane * 8) || cudaMalloc(&Cb, (size_t)njobs * nb * nb * 8) || cudaMalloc(&pl, plane * np) ||
         cudaMalloc(&ex, sizeof(int) * nt * nb) || cudaMalloc(&it, 64 * nt) || cudaMalloc(&dj, sizeof(OzJob) * njobs) ||
-        cudaMalloc(&scr, (size_t)slots * CRT_SLOT_BYTES) || cudaMalloc(&flags, sizeof(int) * slots))
+        cudaMalloc(&scr, (size_t)slots * CRT_SLOT_BYTES) || cudaMalloc(&flags, sizeof(int) * (slots + 1 + reps)))
         return MP_ERR_CUDA;
-    cudaMemset(flags, 0, sizeof(int) * slots);
+    cudaMemset(flags, 0, sizeof(int) * (slots + 1 + reps));  // slot flags + one tile counter per launch
     cudaMemset(P, 0, plane * 8);
     cudaMemset(Cb, 0, (size_t)njobs * nb * nb * 8);
     {   // deterministic non-trivial panel: x = sin(i * 0.37 + j * 0.11) scaled per row
@@ -198,9 +205,13 @@ mp_status mp_bench_fp64_engine(int engine, int nb, int nt, int njobs, int nmod, 
         return engine == 16 ? crt_split_launch((const CrtSplitItem*)it, nt, nb, c, 0)
                             : ozaki_split_launch((const OzSplitItem*)it, nt, nb, 8, 0);
     };
+    int launch_no = 0;
     auto gemm = [&]() {
         if (engine == 16) {
-            CrtArgs a{dj, pl, ex, plane, nb, nt, 0, scr, flags, c, Cb, (uint64_t)njobs * nb, 0};
+            int* const ctr = flags + slots + std::min(launch_no++, reps);
+            // nmod = 8: the FP32-class instantiation (FP32 C tiles, 2 nb^2 floats apart)
+            CrtArgs a{dj, pl, ex, plane, nb, nt, 0, scr, flags, c, Cb, (uint64_t)njobs * nb * (nmod == 8 ? 2 : 1), 0,
+                      nmod == 8, 0, ctr};
             return crt_gemm_launch(a, njobs, 0);
         }
         OzArgs a{dj, pl, ex, plane, nb, nt, 8, 0, 0};

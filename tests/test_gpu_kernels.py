@@ -199,6 +199,55 @@ def test_crt_int8_fp64_gemm(lib, nb, nt, m, n, nmod):
     assert np.array_equal(got[5], Cm[5])  # zero row of A: C row untouched
 
 
+@pytest.mark.parametrize("nb,nt,m,n", [(512, 2, 1, 0), (2048, 3, 2, 1), (4096, 2, 0, 1)])
+def test_crt8_fp32_class_gemm(lib, nb, nt, m, n):
+    """FP32 class as CRT-8 (8 moduli, b = 25 operand bits per row at K = 2048, FP32 C reduce-added by
+    the TMA unit): error vs the exact product of the FP32 operands within 2x an SGEMM's on the same
+    inputs (the C13 pin), rows of very different scale; plus the same pin against the FP32 C update."""
+    rng = np.random.default_rng(nb + 8)
+    A32 = (rng.standard_normal((nt * nb, nb)) * np.exp(rng.uniform(-2, 2, (nt * nb, 1)))).astype(np.float32)
+    Cm = (rng.standard_normal((nb, nb)) * 0.01).astype(np.float32)
+    dP, dC = dev(A32.astype(np.float64)), dev(Cm)
+    assert lib.mp_test_crt_gemm(C.c_void_p(dP.data_ptr()), C.c_void_p(dC.data_ptr()), nb, nt, m, n, 8, 0) == 0
+    got = dC.cpu().numpy().astype(np.float64)
+    Ad = A32.astype(np.float64)
+    A, B = Ad[m * nb:(m + 1) * nb], Ad[n * nb:(n + 1) * nb]
+    exact = Cm.astype(np.float64) - A @ B.T
+    sgemm = (Cm - A32[m * nb:(m + 1) * nb] @ A32[n * nb:(n + 1) * nb].T).astype(np.float64)
+    err = np.linalg.norm(got - exact) / np.linalg.norm(exact)
+    err_sg = np.linalg.norm(sgemm - exact) / np.linalg.norm(exact)
+    assert err <= 2 * err_sg, (err, err_sg)
+    # entrywise: the operand rounding is 2^-26 of the row / column max
+    ma = np.abs(A).max(axis=1)[:, None]
+    mb = np.abs(B).max(axis=1)[None, :]
+    # two FP32 roundings: the converted product and the reduce-add
+    ent = np.abs(got - exact) - 2.0**-23 * (np.abs(exact) + np.abs(A @ B.T))
+    assert np.all(ent <= 2 * nb * 2.0**-26 * ma * mb), np.max(ent / (ma * mb))
+
+
+@pytest.mark.parametrize("nmod", [8, 16])
+def test_crt_store_mode_fp64_c(lib, nmod):
+    """Store mode (C = P_m P_n^T, the TRSM product X = A_mk W^T with W = L_kk^-1): CRT-8 (the FP32-class
+    TRSM, FP64 C) keeps b = 25 bits per operand row, CRT-16 b = 56; C's previous contents are ignored."""
+    nb, nt, m, n = 2048, 2, 1, 0
+    rng = np.random.default_rng(nmod + 1)
+    P = rng.standard_normal((nt * nb, nb)) * np.exp(rng.uniform(-3, 3, (nt * nb, 1)))
+    P[n * nb:(n + 1) * nb] = np.tril(P[n * nb:(n + 1) * nb])  # a triangular B operand, like the inverse factor
+    Cm = np.full((nb, nb), np.nan)
+    dP, dC = dev(P), dev(Cm)
+    assert lib.mp_test_crt_gemm_ex(C.c_void_p(dP.data_ptr()), C.c_void_p(dC.data_ptr()), nb, nt, m, n, nmod, 0, 0,
+                                   1) == 0
+    got = dC.cpu().numpy()
+    A, B = P[m * nb:(m + 1) * nb], P[n * nb:(n + 1) * nb]
+    ref = A @ B.T
+    b = {8: 25, 16: 56}[nmod]
+    ma = np.abs(A).max(axis=1)[:, None]
+    mb = np.abs(B).max(axis=1)[None, :]
+    assert np.all(np.isfinite(got))
+    err = np.abs(got - ref) - 2.0**-52 * np.abs(ref)
+    assert np.all(err <= nb * 2.0 ** -b * ma * mb), np.max(err / (ma * mb)) / 2.0**-b
+
+
 def test_crt_int8_syrk_lower(lib):
     """lower = 1 (DSYRK on a diagonal tile): 256 x 256 blocks on or below the diagonal are updated,
     strictly-upper blocks are left untouched."""

@@ -1,4 +1,4 @@
-"""All three FP64-class engines — CRT modular emulation (MPGEO_OZAKI=16) and the 8-slice Ozaki split
+"""All FP64-class engines — CRT modular emulation (MPGEO_OZAKI=16) and the 8-slice Ozaki split
 (MPGEO_OZAKI=8), both on INT8 tensor cores, and DMMA FP64 (MPGEO_OZAKI=0) — must meet the all-FP64 tolerances: residual <= 1e-13, l relative error <= 1e-10."""
 import os
 
@@ -15,15 +15,21 @@ from tests.gpu_helpers import to_dev
 pytestmark = pytest.mark.gpu
 
 
-@pytest.fixture(scope="module", params=["16", "8", "0"], ids=["crt", "ozaki", "dmma"])
+@pytest.fixture(scope="module", params=["16", "16t", "8", "0"], ids=["crt", "crt-tf32x3", "ozaki", "dmma"])
 def engine_handle(request):
+    """crt: CRT FP64 class + CRT-8 FP32 class (MPGEO_CRT32=1); crt-tf32x3: CRT FP64 class + 3xTF32 (the
+    default engines)."""
     import paper_conf_cluster_caoalgkb23_b200 as mp
-    os.environ["MPGEO_OZAKI"] = request.param
+    eng = request.param.rstrip("t")
+    os.environ["MPGEO_OZAKI"] = eng
+    os.environ["MPGEO_CRT32"] = "0" if request.param.endswith("t") else "1"  # crt: the CRT-8 FP32 class (opt-in)
     try:
         h = mp.Handle(0)
     finally:
-        del os.environ["MPGEO_OZAKI"]
-    assert h.config()["ozaki"] % 100 == int(request.param)
+        del os.environ["MPGEO_OZAKI"], os.environ["MPGEO_CRT32"]
+    oz = h.config()["ozaki"]
+    assert oz % 100 == int(eng)
+    assert (oz >= 200) == (request.param == "16")
     return h
 
 

@@ -1,4 +1,4 @@
-"""Isolated FP64-class engine timing (mp_bench_fp64_engine): 8-slice splitting vs CRT, batched
+"""Isolated INT8 engine timing (mp_bench_fp64_engine): 8-slice splitting vs CRT, batched
 nb = 2048 tile-GEMMs; prints FP64-equivalent TFLOP/s of the GEMM launch and the split cost."""
 import ctypes as C
 import os
@@ -21,8 +21,8 @@ def run(engine, nb=2048, nt=8, njobs=64, nmod=16, reps=5):
 if __name__ == "__main__":
     import torch
     torch.cuda.init()
-    args = sys.argv[1:] or ["8", "16"]
+    args = sys.argv[1:] or ["8", "16", "16/8"]  # "16/8": CRT with 8 moduli (the FP32-class instantiation)
     for a in args:
-        eng = int(a)
+        eng, _, nm = a.partition("/")
         for nj in (16, 64, 148):
-            run(eng, njobs=nj)
+            run(int(eng), njobs=nj, nmod=int(nm) if nm else 16)
