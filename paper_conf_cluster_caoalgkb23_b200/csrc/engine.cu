@@ -777,7 +777,7 @@ static mp_status plan_potrf(mp_handle* h, mp_matrix* A, const uint8_t* km, const
     int nsm = 148;
     cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, h->device);
     const int upd_pairs = la ? std::max(1, nsm / 2 - h->reserve_pairs) : 0;
-    const int pan_pairs = la ? std::max(1, h->reserve_pairs) : 0;
+    const int pan_pairs = 0;  // panel-stream CRT launches: any free SM (dynamic tiles, high priority)
     const int R = h->nranks, me = h->rank;
     Comm& X = A->comm;
     auto ST = [&](int step) -> uint64_t { return (epoch << 24) + (uint64_t)(step + 2); };
