@@ -201,7 +201,8 @@ struct __align__(64) CrtParams {
     int* slot_flags;
     int nslots, nb, tiles_n, tiles_per_job, lower, total;
     int store;  // 1: C = P_m P_n^T (TMA store), 0: C -= P_m P_n^T (TMA reduce-add)
-    int* tile_counter;  // dynamic tile scheduler (zero before the launch)
+    int* tile_counter;  // [0]: dynamic tile scheduler, [1]: current modulus-pair phase (zero before the launch)
+    int phase_lock;     // 1: start each tile at the current modulus-pair phase (MPGEO_CRT_PHASE, default 1)
     CrtConst c;
 };
 
@@ -442,7 +443,11 @@ __global__ void __launch_bounds__(THREADS, 1) crt_gemm_kernel(const __grid_const
                 const int s = i % RING;
                 mbar_wait(su32(&ring_empty[s]), ((uint32_t)(i / RING) & 1u) ^ 1u);
                 tile = atomicAdd(p.tile_counter, 1);
+                // modulus-pair phase: start where the other pairs currently are (p.tile_counter[1],
+                // written by every MMA issuer), so concurrent tiles read the same residue planes
+                // and the operands of one phase stay L2-resident; any order gives the same result
                 if (tile >= p.total) tile = -1;
+                else if (p.phase_lock) tile |= (*(volatile int*)(p.tile_counter + 1) & (NMOD / 2 - 1)) << 28;
                 tile_ring[s] = tile;
                 st_cluster_u32(cluster_addr(su32(&tile_ring[s]), 1), tile);
                 mbar_arrive_cluster(su32(&ring_full[s]));
@@ -451,12 +456,15 @@ __global__ void __launch_bounds__(THREADS, 1) crt_gemm_kernel(const __grid_const
                 tile = ring_take(i, true);
             }
             if (tile < 0) break;
+            const int j0 = tile >> 28;
+            tile &= (1 << 28) - 1;
             int job, bi, bj;
             tile_coords(p, tile, job, bi, bj);
             const OzJob jb = p.jobs[job];
             const int rowA = jb.m * p.nb + bi * 256 + (int)crank * BM;
             const int rowB = jb.n * p.nb + bj * BN + (int)crank * (BN / 2);
-            for (int t = 0; t < N; ++t)
+            for (int tt = 0; tt < N; ++tt) {
+                const int t = (2 * j0 + tt) & (N - 1);
                 for (int kb = 0; kb < KB; ++kb, ++it) {
                     const uint32_t s = it % STAGES;
                     const uint32_t ph = (it / STAGES) & 1u;
@@ -468,13 +476,17 @@ __global__ void __launch_bounds__(THREADS, 1) crt_gemm_kernel(const __grid_const
                     tma3d_pair(st, &p.a, fb, kb * BK, rowA, t);
                     tma3d_pair(st + A_BYTES, &p.b, fb, kb * BK, rowB, t);
                 }
+            }
         }
     } else if (warp == 1 && lane == 0 && crank == 0) {
         // ---------------- MMA issuer (leader CTA): one accumulator per modulus, two in flight
         uint32_t it = 0, g = 0;
         for (int i = 0;; ++i) {
-            if (ring_take(i, true) < 0) break;
-            for (int t = 0; t < N; ++t, ++g) {
+            const int tv = ring_take(i, true);
+            if (tv < 0) break;
+            const int j0 = tv >> 28;
+            for (int tt = 0; tt < N; ++tt, ++g) {
+                if (p.phase_lock && !(tt & 1)) *(volatile int*)(p.tile_counter + 1) = ((j0 + (tt >> 1)) & (N / 2 - 1));
                 const uint32_t buf = g & 1u;
                 { PROF_T0();
                 mbar_wait(su32(&acc_empty[buf]), ((g >> 1) & 1u) ^ 1u);
@@ -608,11 +620,14 @@ __global__ void __launch_bounds__(THREADS, 1) crt_gemm_kernel(const __grid_const
             tile = __shfl_sync(0xffffffffu, tile, 0);
             if (lane == 0) mbar_arrive_cluster(cluster_addr(su32(&ring_empty[it_tile % RING]), 0));
             if (tile < 0) break;
+            const int j0 = tile >> 28;
+            tile &= (1 << 28) - 1;
             int job, bi, bj;
             tile_coords(p, tile, job, bi, bj);
             uint8_t* const scr = scr0 + (size_t)(it_tile & 1) * CRT_HALF_BYTES;
-            for (int j = 0; j < NP; ++j) {
-                if (pv) prefetch_groups((j * 16) / NP, ((j + 1) * 16) / NP);
+            for (int jj = 0; jj < NP; ++jj) {
+                const int j = (j0 + jj) & (NP - 1);  // moduli pair (phase-rotated order)
+                if (pv) prefetch_groups((jj * 16) / NP, ((jj + 1) * 16) / NP);
                 // ---- first modulus a of pair j: canonical residues r_a kept as bytes (32 registers)
                 uint32_t ra[4][8];
                 {
@@ -692,7 +707,7 @@ __global__ void __launch_bounds__(THREADS, 1) crt_gemm_kernel(const __grid_const
                 // ---- two groups of the pending tile's reconstruction (16 groups over the NP pairs)
                 if (pv) {
                     PROF_T0();
-                    const int g0 = (j * 16) / NP, g1 = ((j + 1) * 16) / NP;
+                    const int g0 = (jj * 16) / NP, g1 = ((jj + 1) * 16) / NP;
                     uint4 wa[NP], wb[NP];
                     load_group(g0, wa);
                     for (int gi = g0; gi < g1; gi += 2) {
@@ -837,11 +852,16 @@ cudaError_t crt_gemm_launch(const CrtArgs& a, int njobs, cudaStream_t s) {
     p.lower = a.lower;
     p.store = a.store;
     p.tile_counter = a.counter;
+    static const int phase_env = [] {
+        const char* e = getenv("MPGEO_CRT_PHASE");
+        return e ? atoi(e) : 1;
+    }();
+    p.phase_lock = phase_env;
     if (!a.counter) return cudaErrorInvalidValue;
     p.tiles_per_job = a.lower ? p.tiles_n * (p.tiles_n + 1) / 2 : p.tiles_n * p.tiles_n;
     p.c = a.c;
     const long long total = (long long)njobs * p.tiles_per_job;
-    if (total > 0x7fffffffLL) return cudaErrorInvalidConfiguration;
+    if (total >= (1LL << 28)) return cudaErrorInvalidConfiguration;  // tile index | phase << 28 in the ring
     p.total = (int)total;
     static const int env_pairs = [] {  // MPGEO_CRT_PAIRS overrides the persistent grid size (CTA pairs)
         const char* e = getenv("MPGEO_CRT_PAIRS");

@@ -49,7 +49,7 @@ struct CrtArgs {
     int max_pairs;         // persistent grid in CTA pairs (0: one pair per 2 SMs)
     int c_f32 = 0;         // 0: FP64 C (nmod = 16 or 8); 1: FP32 C (nmod = 8, FP32-class update)
     int store = 0;         // 1: C = P_m P_n^T (overwrite), 0: C -= P_m P_n^T
-    int* counter = nullptr;  // tile-scheduler counter of this launch (device int, zero at launch)
+    int* counter = nullptr;  // 2 device ints of this launch, zero at launch: tile counter, modulus phase
 };
 // one CTA's 128 x 256 combined residues (N/2 x 2 bytes each) for two tiles (the epilogue reconstructs
 // tile T-1 while it reduces tile T)

@@ -130,7 +130,7 @@ struct mp_matrix {
 static size_t align_up(size_t v, size_t a) { return (v + a - 1) / a * a; }
 // CRT launches of one factorisation: <= 4 update launches (two parts x SYRK / GEMM) + 1 FP32-class +
 // 1 TRSM per panel
-static size_t crt_counters(int nt) { return 8 * (size_t)nt + 64; }
+static size_t crt_counters(int nt) { return 2 * (8 * (size_t)nt + 64); }
 constexpr int MT_PIECES_MAX = 512;
 static int ceil_div(int a, int b) { return (a + b - 1) / b; }
 
@@ -763,7 +763,11 @@ static mp_status plan_potrf(mp_handle* h, mp_matrix* A, const uint8_t* km, const
     // one tile-scheduler counter per CRT launch of this call (zeroed by potrf_run)
     int* const crt_ctr = crt ? A->at<int>(A->R.crtctr) : nullptr;
     size_t ctr_next = 0;
-    auto next_ctr = [&]() -> int* { return ctr_next < crt_counters(nt) ? crt_ctr + ctr_next++ : nullptr; };
+    auto next_ctr = [&]() -> int* {  // two ints per launch
+        if (ctr_next + 2 > crt_counters(nt)) return nullptr;
+        ctr_next += 2;
+        return crt_ctr + ctr_next - 2;
+    };
     int* const ozeb = A->at<int>(A->R.ozexp);
     auto K = [&](int m, int k) { return km[(size_t)m * nt + k]; };
     auto C = [&](int m, int k) { return cm[(size_t)m * nt + k]; };

@@ -120,9 +120,9 @@ mp_status mp_test_crt_gemm_ex(const double* d_panel, void* d_C, int nb, int nt, 
     int* flags = nullptr;
     if (cudaMalloc(&pl, plane * nmod) || cudaMalloc(&ex, sizeof(int) * nt * nb) ||
         cudaMalloc(&it, sizeof(CrtSplitItem) * nt) || cudaMalloc(&dj, sizeof(OzJob)) ||
-        cudaMalloc(&scr, (size_t)slots * CRT_SLOT_BYTES) || cudaMalloc(&flags, sizeof(int) * (slots + 1)))
+        cudaMalloc(&scr, (size_t)slots * CRT_SLOT_BYTES) || cudaMalloc(&flags, sizeof(int) * (slots + 2)))
         return MP_ERR_CUDA;
-    cudaMemset(flags, 0, sizeof(int) * (slots + 1));  // slot flags + the tile counter
+    cudaMemset(flags, 0, sizeof(int) * (slots + 2));  // slot flags + the tile counter and phase
     std::vector<CrtSplitItem> h(nt);
     for (int t = 0; t < nt; ++t)
         h[t] = CrtSplitItem{d_panel + (size_t)t * nb * nb, pl + (size_t)t * nb * nb, ex + (size_t)t * nb, plane};
@@ -170,9 +170,9 @@ mp_status mp_bench_fp64_engine(int engine, int nb, int nt, int njobs, int nmod, 
     const int slots = crt_scratch_slots();
     if (cudaMalloc(&P, plane * 8) || cudaMalloc(&Cb, (size_t)njobs * nb * nb * 8) || cudaMalloc(&pl, plane * np) ||
         cudaMalloc(&ex, sizeof(int) * nt * nb) || cudaMalloc(&it, 64 * nt) || cudaMalloc(&dj, sizeof(OzJob) * njobs) ||
-        cudaMalloc(&scr, (size_t)slots * CRT_SLOT_BYTES) || cudaMalloc(&flags, sizeof(int) * (slots + 1 + reps)))
+        cudaMalloc(&scr, (size_t)slots * CRT_SLOT_BYTES) || cudaMalloc(&flags, sizeof(int) * (slots + 2 * (1 + reps))))
         return MP_ERR_CUDA;
-    cudaMemset(flags, 0, sizeof(int) * (slots + 1 + reps));  // slot flags + one tile counter per launch
+    cudaMemset(flags, 0, sizeof(int) * (slots + 2 * (1 + reps)));  // slot flags + counter pair per launch
     cudaMemset(P, 0, plane * 8);
     cudaMemset(Cb, 0, (size_t)njobs * nb * nb * 8);
     {   // deterministic non-trivial panel: x = sin(i * 0.37 + j * 0.11) scaled per row
@@ -208,7 +208,7 @@ mp_status mp_bench_fp64_engine(int engine, int nb, int nt, int njobs, int nmod, 
     int launch_no = 0;
     auto gemm = [&]() {
         if (engine == 16) {
-            int* const ctr = flags + slots + std::min(launch_no++, reps);
+            int* const ctr = flags + slots + 2 * std::min(launch_no++, reps);
             // nmod = 8: the FP32-class instantiation (FP32 C tiles, 2 nb^2 floats apart)
             CrtArgs a{dj, pl, ex, plane, nb, nt, 0, scr, flags, c, Cb, (uint64_t)njobs * nb * (nmod == 8 ? 2 : 1), 0,
                       nmod == 8, 0, ctr};
