@@ -33,6 +33,8 @@ def sample_z(ev, x, y, theta, seed):
 
 def main():
     n = int(sys.argv[1]) if len(sys.argv) > 1 else 40000
+    modes = (sys.argv[2] if len(sys.argv) > 2 else "fp64,mp").split(",")
+    maxfev = int(sys.argv[3]) if len(sys.argv) > 3 else 600
     nb = 2048
     theta_true = (1.0, 0.03, 0.5)
     x, y = synth.locations(n, 0)
@@ -41,17 +43,26 @@ def main():
     dx, dy, dz = (torch.from_numpy(a).cuda() for a in (x, y, z))
     out = {"n": n, "nb": nb, "theta_true": theta_true, "optimizer": "COBYQA (BOBYQA family), bounds [0.01,2]^3, "
            "start at the lower bounds, final trust radius 1e-9"}
+    os.makedirs("gpurun_out", exist_ok=True)
     for name, mode in [("fp64", mp.MP_MAP_FP64), ("mp", mp.MP_MAP_ADAPTIVE)]:
+        if name not in modes:
+            continue
         t0 = time.time()
-        r = fit(ev, dx, dy, dz, mode=mode, u_req=1e-9, maxfev=600)
+        logf = open(f"gpurun_out/mle_n{n}_{name}.log", "w")
+
+        def log(th, ll, logf=logf):
+            logf.write(f"{th[0]:.10f} {th[1]:.10f} {th[2]:.10f} {ll:.10f}\n")
+            logf.flush()
+
+        r = fit(ev, dx, dy, dz, mode=mode, u_req=1e-9, maxfev=maxfev, log=log)
         rep = ev.eval(dx, dy, dz, tuple(r.theta), mode=mode)
         out[name] = {"theta": list(r.theta), "loglik": r.loglik, "nfev": r.nfev, "seconds": time.time() - t0,
                      "tiles_fp64_fp32_fp16": list(rep.tiles)}
         print(name, out[name], flush=True)
-    out["max_abs_dtheta"] = float(np.max(np.abs(np.array(out["mp"]["theta"]) - np.array(out["fp64"]["theta"]))))
+    if "mp" in out and "fp64" in out:
+        out["max_abs_dtheta"] = float(np.max(np.abs(np.array(out["mp"]["theta"]) - np.array(out["fp64"]["theta"]))))
     print(json.dumps(out))
-    os.makedirs("gpurun_out", exist_ok=True)
-    json.dump(out, open(f"gpurun_out/mle_n{n}.json", "w"), indent=1)
+    json.dump(out, open(f"gpurun_out/mle_n{n}_{'_'.join(modes)}.json", "w"), indent=1)
 
 
 if __name__ == "__main__":
