@@ -19,6 +19,9 @@ mp_status mp_test_dgemm(const double* d_A, const double* d_B, void* d_C, int M, 
  * [nt*nb][nb]: kind 1 = 3xTF32 (panel = hi, panel_lo = lo, float), kind 2 = FP16 (panel = half). */
 mp_status mp_test_tc_gemm(int kind, const void* d_panel, const void* d_panel_lo, float* d_C, int nb, int nt, int m,
                           int n);
+/* 3xFP16 FP32-class GEMM (reading C13c): splits the nt tiles of the FP64 panel [nt*nb][nb] into
+ * row-scaled FP16 hi / lo, then C (FP32 nb x nb) -= P_m P_n^T on tcgen05 kind::f16. */
+mp_status mp_test_tc_gemm_f16x3(const double* d_panel, float* d_C, int nb, int nt, int m, int n);
 /* Ozaki-split GEMM on INT8 tensor cores: splits the nt tiles of the FP64 panel [nt*nb][nb] into 8
  * int8 slices, then C -= P_m P_n^T using the first S slices: S = 8 (FP64 class, C FP64, lower CTA
  * tiles only if `lower`) or S = 4 (FP32 class, C is FP32). */

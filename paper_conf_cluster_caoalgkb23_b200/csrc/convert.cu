@@ -87,6 +87,46 @@ __global__ void __launch_bounds__(256) transpose_kernel(const double* __restrict
     for (int r = ty; r < 32; r += 8) dst[(size_t)(bx + r) * nb + by + tx] = t[tx][r];
 }
 
+// 3xFP16 operands of the FP32 class (reading C13c): row i of the FP64 panel tile, rounded to FP32
+// (the FP32-class operand), is scaled by 2^s_i with max_j |x_ij| 2^s_i < 2^15 and split into FP16
+// hi = rn(x 2^s), lo = rn(x 2^s - hi) (x 2^s - hi is exact in FP32), i.e. the 11 + 11-bit split of
+// 3xTF32, now within FP16 range; e_i = -s_i is stored for the GEMM epilogue.  One warp per row.
+__global__ void __launch_bounds__(256) split16_kernel(const Split16Item* items, int nb) {
+    const Split16Item it = items[blockIdx.y];
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    const int row = blockIdx.x * 8 + warp;
+    if (row >= nb) return;
+    const double* x = it.src + (size_t)row * nb;
+    float mx = 0.f;
+    for (int j = lane * 2; j < nb; j += 64) {
+        const double2 v = *(const double2*)(x + j);
+        mx = fmaxf(mx, fmaxf(fabsf(__double2float_rn(v.x)), fabsf(__double2float_rn(v.y))));
+    }
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) mx = fmaxf(mx, __shfl_xor_sync(0xffffffffu, mx, o));
+    int e = 0;
+    if (mx > 0.f) frexpf(mx, &e);  // mx < 2^e
+    const int sc = min(max(15 - e, -100), 115);  // 2^sc and 2^-sc are normal FP32 numbers
+    if (lane == 0) it.exps[row] = -sc;
+    const float f = ldexpf(1.f, sc);
+    __half* hi = it.hi + (size_t)row * nb;
+    __half* lo = it.lo + (size_t)row * nb;
+    for (int j = lane * 2; j < nb; j += 64) {
+        const double2 v = *(const double2*)(x + j);
+        const float a0 = __double2float_rn(v.x) * f, a1 = __double2float_rn(v.y) * f;
+        const __half h0 = __float2half_rn(a0), h1 = __float2half_rn(a1);
+        *(__half2*)(hi + j) = __halves2half2(h0, h1);
+        *(__half2*)(lo + j) = __halves2half2(__float2half_rn(a0 - __half2float(h0)), __float2half_rn(a1 - __half2float(h1)));
+    }
+}
+
+cudaError_t split16_launch(const Split16Item* items, int n, int nb, cudaStream_t s) {
+    if (n <= 0) return cudaSuccess;
+    if (nb % 64) return cudaErrorInvalidValue;
+    split16_kernel<<<dim3((nb + 7) / 8, n), 256, 0, s>>>(items, nb);
+    return cudaGetLastError();
+}
+
 cudaError_t identity_launch(double* A, int nb, cudaStream_t s) {
     identity_kernel<<<nb, 256, 0, s>>>(A, nb);
     return cudaGetLastError();

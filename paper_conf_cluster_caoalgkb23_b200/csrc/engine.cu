@@ -55,6 +55,7 @@ struct mp_handle {
                         // both on INT8 tensor cores; 0 = DMMA
     int matern_table = 1;  // general nu: tabulated correlation (1) or direct K_nu per entry (0)
     int ozaki32 = 0;    // 1: FP32-class GEMM on INT8 tensor cores (first 4 slices); 0: 3xTF32 tcgen05 (default)
+    int f16x3 = 1;      // FP32-class update as 3xFP16 (row-scaled FP16 hi/lo split, kind::f16; reading C13c); 0: 3xTF32
     int crt32 = 0;      // with the CRT FP64 engine: FP32-class GEMM as 8 INT8 GEMMs (CRT-8, FP32 C); opt-in:
                         // measured slower than 3xTF32 inside the evaluation (profiles/r01/README.md)
     int crt_trsm = 1;   // with the CRT FP64 engine: TRSM of FP32/FP16-class tiles as the FP32-class product
@@ -303,6 +304,7 @@ mp_status mp_init(int device, int rank, int nranks, int P, int Q, const uint8_t*
     if (const char* e = getenv("MPGEO_OZAKI")) h->ozaki = atoi(e);
     if (const char* e = getenv("MPGEO_OZAKI32")) h->ozaki32 = atoi(e);
     if (const char* e = getenv("MPGEO_CRT32")) h->crt32 = atoi(e);
+    if (const char* e = getenv("MPGEO_F16X3")) h->f16x3 = atoi(e);
     if (const char* e = getenv("MPGEO_CRT_TRSM")) h->crt_trsm = atoi(e);
     if (const char* e = getenv("MPGEO_RESERVE_PAIRS")) h->reserve_pairs = std::max(0, atoi(e));
     if (const char* e = getenv("MPGEO_MATERN_TABLE")) h->matern_table = atoi(e);
@@ -750,6 +752,7 @@ static mp_status plan_potrf(mp_handle* h, mp_matrix* A, const uint8_t* km, const
     if (crt && !crt_constants(CRT_NMAX, nb, &crtc)) FAIL(h, MP_ERR_ARG, "CRT constants for nb=%d", nb);
     // FP32 class on the CRT engine: 8 moduli (b = 25 operand bits at nb = 2048), FP32 C
     const bool crt32 = crt && h->crt32 && A->R.oz32 && use_tc;
+    const bool f16x3 = h->f16x3 != 0;
     // low-precision-class TRSMs as CRT-8 products with the inverse factor (FP32 TRSM there)
     const bool ctrsm = crt && h->crt_trsm && A->R.oz32 && nb % 32 == 0;
     if ((crt32 || ctrsm) && !crt_constants(8, nb, &crtc32)) FAIL(h, MP_ERR_ARG, "CRT-8 constants for nb=%d", nb);
@@ -852,6 +855,13 @@ static mp_status plan_potrf(mp_handle* h, mp_matrix* A, const uint8_t* km, const
         int8_t* ozs = ozb + set * nt * nb2 * (crt ? CRT_NMAX : 8);
         int* oze = ozeb + set * (size_t)nt * nb;
         const int64_t ozplane = (int64_t)nt * nb2;
+        // 3xFP16 caches inside the TF32 hi/lo region of this set: hi at phi, lo at phi + nt nb^2
+        // halves, the row exponents at plo
+        auto s16item = [=](int m) {
+            __half* const h = (__half*)phi;
+            return Split16Item{p64 + (size_t)m * nb2, h + (size_t)m * nb2, h + (size_t)nt * nb2 + (size_t)m * nb2,
+                               (int*)plo + (size_t)m * nb};
+        };
         cur = &pan[k];
         // ---- 1. DPOTRF(k,k), FP64: two-level blocking — 128-column blocks
         //      (diagonal block Cholesky + inverse, block column as GEMM with the inverse, update
@@ -934,6 +944,7 @@ static mp_status plan_potrf(mp_handle* h, mp_matrix* A, const uint8_t* km, const
         }
         // ---- 3. panel in
         std::vector<PanelTile> pin, pout;
+        std::vector<Split16Item> s16out;  // 3xFP16 operands derived after panel out
         for (int m = k + 1; m < nt; ++m) {
             if (!A->mine(m, k)) continue;
             PanelTile t{};
@@ -948,8 +959,12 @@ static mp_status plan_potrf(mp_handle* h, mp_matrix* A, const uint8_t* km, const
             if (use_tc) {
                 if (need16) t.p16 = p16 + (size_t)m * nb2;
                 if (need32 && !oz32 && !crt32) {
-                    t.hi = phi + (size_t)m * nb2;
-                    t.lo = plo + (size_t)m * nb2;
+                    if (f16x3) {
+                        s16out.push_back(s16item(m));
+                    } else {
+                        t.hi = phi + (size_t)m * nb2;
+                        t.lo = plo + (size_t)m * nb2;
+                    }
                 }
             }
             pout.push_back(t);
@@ -1020,6 +1035,11 @@ static mp_status plan_potrf(mp_handle* h, mp_matrix* A, const uint8_t* km, const
             fc.trsm += np * fnb * fnb * fnb;
             // ---- 5. panel out (K2)
             cur->push_back({[=](cudaStream_t s) { return panel_out_launch(d_out, np, (int64_t)nb2, s); }, C_CONV, 0});
+            if (!s16out.empty()) {
+                Split16Item* di = ar.push(s16out);
+                const int ns = (int)s16out.size();
+                cur->push_back({[=](cudaStream_t s) { return split16_launch(di, ns, nb, s); }, C_CONV, 0});
+            }
         }
         if (dist) {
             // ---- 5b. publish my L_mk (comm precision) for remote successors
@@ -1045,6 +1065,7 @@ static mp_status plan_potrf(mp_handle* h, mp_matrix* A, const uint8_t* km, const
             // ---- 5c. pull the remote L_mk my tiles need: peer payload -> FP64 panel slot + caches
             std::vector<WaitItem> waits;
             std::vector<PullItem> pulls;
+            std::vector<Split16Item> s16pull;
             for (auto& x : xpull[k]) {
                 const int m = x.m;
                 if (m == k) continue;
@@ -1055,8 +1076,12 @@ static mp_status plan_potrf(mp_handle* h, mp_matrix* A, const uint8_t* km, const
                             nullptr, C(m, k), 0};
                 if (use_tc && n16) it.p16 = p16 + (size_t)m * nb2;
                 if (use_tc && n32 && !oz32 && !crt32) {
-                    it.hi = phi + (size_t)m * nb2;
-                    it.lo = plo + (size_t)m * nb2;
+                    if (f16x3) {
+                        s16pull.push_back(s16item(m));
+                    } else {
+                        it.hi = phi + (size_t)m * nb2;
+                        it.lo = plo + (size_t)m * nb2;
+                    }
                 }
                 waits.push_back(WaitItem{it.flag, it.target});
                 pulls.push_back(it);
@@ -1066,6 +1091,11 @@ static mp_status plan_potrf(mp_handle* h, mp_matrix* A, const uint8_t* km, const
                 PullItem* dp = ar.push(pulls);
                 const int npl = (int)pulls.size();
                 cur_push(Op{[=](cudaStream_t s) { return pull_launch(dp, npl, (int64_t)nb2, s); }, C_CONV, 0});
+            }
+            if (!s16pull.empty()) {
+                Split16Item* di = ar.push(s16pull);
+                const int ns = (int)s16pull.size();
+                cur_push(Op{[=](cudaStream_t s) { return split16_launch(di, ns, nb, s); }, C_CONV, 0});
             }
             uint64_t* df = doneflag(me, sp);
             const uint64_t dv = ST(k);
@@ -1199,7 +1229,14 @@ static mp_status plan_potrf(mp_handle* h, mp_matrix* A, const uint8_t* km, const
             TcArgs ta{dj, phi, plo, nb, nt};
             ta.cbase = cpool;
             ta.crows = crows;
-            cur->push_back({[=](cudaStream_t s) { return tc_gemm_tf32x3_launch(ta, nj, s); }, C_UPD32, 2 * f3 * nj});
+            if (f16x3) {
+                ta.h16hi = (const __half*)phi;
+                ta.h16lo = (const __half*)phi + (size_t)nt * nb2;
+                ta.e16 = (const int*)plo;
+                cur->push_back({[=](cudaStream_t s) { return tc_gemm_f16x3_launch(ta, nj, s); }, C_UPD32, 2 * f3 * nj});
+            } else {
+                cur->push_back({[=](cudaStream_t s) { return tc_gemm_tf32x3_launch(ta, nj, s); }, C_UPD32, 2 * f3 * nj});
+            }
         }
         if (!t16.empty()) {
             TcJob* dj = ar.push(t16);

@@ -75,6 +75,14 @@ struct PanelTile {
     int store_prec;   // P64 / P32
     int comm_prec;    // precision the tile is sent at (P64 / P32 / P16)
 };
+// 3xFP16 FP32-class operands of one FP64 panel tile (split16_kernel, convert.cu)
+struct Split16Item {
+    const double* src;  // FP64 panel slot (nb x nb)
+    __half* hi;         // row-scaled FP16 hi / lo (nb x nb)
+    __half* lo;
+    int* exps;          // [nb]: 2^exps undoes row i's scale
+};
+cudaError_t split16_launch(const Split16Item* items, int n, int nb, cudaStream_t s);
 // p64 = (double) store
 cudaError_t panel_in_launch(const PanelTile* t, int ntiles, int64_t elems, cudaStream_t s);
 // store = round(p64, store_prec); p64 = round(p64, comm_prec); p16/hi/lo = conversions of p64

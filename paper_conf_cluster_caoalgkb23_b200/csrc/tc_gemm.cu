@@ -17,6 +17,9 @@
 // KIND 1 (FP32 class, 3xTF32, reading C13): kind::tf32, BK = 32, stages of {A_hi, A_lo, B_hi, B_lo},
 //   8 epilogue warps; per k-step three MMAs lo.hi + hi.lo + hi.hi; K is split in chunks of 64
 //   accumulated in two ping-pong TMEM accumulators and summed by the epilogue in FP32.
+// KIND 2 (FP32 class, 3xFP16, reading C13c): the same three products with an 11-bit hi/lo split in
+//   FP16 (kind::f16, twice the TF32 rate): each panel row is scaled by a power of two so its max is
+//   below 2^15 (split16_kernel, convert.cu); the epilogue multiplies by 2^(eA_i + eB_j).
 #include <cudaTypedefs.h>
 #include <stdint.h>
 #include <stdlib.h>
@@ -27,6 +30,9 @@
 namespace mpgeo {
 
 constexpr int TC_BM = 128;  // output rows per CTA (TMEM lanes)
+#ifndef TC16X3_CHUNK_KB
+#define TC16X3_CHUNK_KB 1  // KIND 2: k-blocks of 64 per TMEM accumulator chunk (K = 64, as 3xTF32)
+#endif
 template <int KIND>
 struct TcThreads {
     static constexpr int EPI_WARPS = KIND == 0 ? 4 : 8;  // 3xTF32: two warpgroups, one per 128-column half
@@ -37,6 +43,7 @@ struct __align__(64) TcParams {
     CUtensorMap a, b, a_lo, b_lo, c;
     const TcJob* jobs;
     const float* cbase;
+    const int* exps;  // KIND 2: per panel-cache row, 2^exps undoes the operand scale
     int nb, tiles_n, tiles_per_job;
 };
 
@@ -48,9 +55,9 @@ template <int KIND, int CL>
 struct TcCfg {
     static constexpr int BN = 256;                 // MMA N = output columns per CTA
     static constexpr int BM = TC_BM * CL;          // MMA M = output rows per cluster
-    static constexpr int ESZ = KIND == 0 ? 2 : 4;
+    static constexpr int ESZ = KIND == 1 ? 4 : 2;
     static constexpr int BK = 128 / ESZ;           // elements per 128-byte row
-    static constexpr int UK = KIND == 0 ? 16 : 8;  // K per tcgen05.mma (32 bytes)
+    static constexpr int UK = KIND == 1 ? 8 : 16;  // K per tcgen05.mma (32 bytes)
     static constexpr int A_BYTES = TC_BM * 128;
     static constexpr int B_BYTES = (BN / CL) * 128;
     static constexpr int STAGE_BYTES = KIND == 0 ? A_BYTES + B_BYTES : 2 * (A_BYTES + B_BYTES);
@@ -62,11 +69,11 @@ struct TcCfg {
     // KIND 1: accumulate CHUNK_KB k-blocks (64 of K) per TMEM accumulator, two accumulators
     // ping-pong; the epilogue sums the chunks in FP32 registers (round-to-nearest), which keeps
     // the tensor core's non-RN FP32 accumulation error from growing with K (reading C13).
-    static constexpr int CHUNK_KB = KIND == 0 ? 1 << 20 : 2;
+    static constexpr int CHUNK_KB = KIND == 0 ? 1 << 20 : KIND == 1 ? 2 : TC16X3_CHUNK_KB;
     static constexpr uint32_t TMEM_COLS = KIND == 0 ? BN : 2 * BN;  // power of two >= 32
     // instruction descriptor: D = F32 (bit 4), A/B format (bits 7-9 / 10-12), K-major both,
     // N >> 3 (bits 17-22), M >> 4 (bits 24-28)
-    static constexpr uint32_t IDESC = (1u << 4) | ((KIND == 0 ? 0u : 2u) << 7) | ((KIND == 0 ? 0u : 2u) << 10) |
+    static constexpr uint32_t IDESC = (1u << 4) | ((KIND == 1 ? 2u : 0u) << 7) | ((KIND == 1 ? 2u : 0u) << 10) |
                                       ((uint32_t)(BN >> 3) << 17) | ((uint32_t)(BM >> 4) << 24);
 };
 
@@ -147,12 +154,12 @@ __device__ __forceinline__ uint64_t desc_sw128(uint32_t saddr) {
 template <int KIND, int CL>
 __device__ __forceinline__ void tc_mma(uint32_t tmem, uint64_t a, uint64_t b, uint32_t accum) {
     constexpr uint32_t ID = TcCfg<KIND, CL>::IDESC;
-    if (KIND == 0 && CL == 1)
+    if (KIND != 1 && CL == 1)
         asm volatile(
             "{\n\t.reg .pred p;\n\tsetp.ne.b32 p, %4, 0;\n\t"
             "tcgen05.mma.cta_group::1.kind::f16 [%0], %1, %2, %3, p;\n\t}" ::"r"(tmem),
             "l"(a), "l"(b), "r"(ID), "r"(accum));
-    else if (KIND == 0)
+    else if (KIND != 1)
         asm volatile(
             "{\n\t.reg .pred p;\n\tsetp.ne.b32 p, %4, 0;\n\t"
             "tcgen05.mma.cta_group::2.kind::f16 [%0], %1, %2, %3, p;\n\t}" ::"r"(tmem),
@@ -295,7 +302,7 @@ __global__ void __launch_bounds__(TcThreads<KIND>::N, TcCfg<KIND, CL>::MIN_BLOCK
             const int chunk = kb / Cfg::CHUNK_KB, kin = kb % Cfg::CHUNK_KB;
             const uint32_t abuf = (uint32_t)(chunk & 1);
             const uint32_t dacc = KIND == 0 ? tmem : tmem + abuf * Cfg::BN;
-            if (KIND == 1 && kin == 0) {  // wait until the epilogues drained this accumulator
+            if (KIND != 0 && kin == 0) {  // wait until the epilogues drained this accumulator
                 mbar_wait(smem_u32(&acc_empty[abuf]), ((uint32_t)(chunk >> 1) & 1u) ^ 1u);
                 tc_fence_after();
             }
@@ -313,13 +320,13 @@ __global__ void __launch_bounds__(TcThreads<KIND>::N, TcCfg<KIND, CL>::MIN_BLOCK
                     const uint64_t alo = desc_sw128(base + Cfg::A_BYTES + koff);
                     const uint64_t bhi = desc_sw128(base + 2 * Cfg::A_BYTES + koff);
                     const uint64_t blo = desc_sw128(base + 2 * Cfg::A_BYTES + Cfg::B_BYTES + koff);
-                    tc_mma<1, CL>(dacc, alo, bhi, acc);  // small terms first
-                    tc_mma<1, CL>(dacc, ahi, blo, 1u);
-                    tc_mma<1, CL>(dacc, ahi, bhi, 1u);
+                    tc_mma<KIND, CL>(dacc, alo, bhi, acc);  // small terms first
+                    tc_mma<KIND, CL>(dacc, ahi, blo, 1u);
+                    tc_mma<KIND, CL>(dacc, ahi, bhi, 1u);
                 }
             }
             tc_commit<CL>(smem_u32(&empty_bar[s]));
-            if (KIND == 1 && (kin == Cfg::CHUNK_KB - 1 || kb == KB - 1)) tc_commit<CL>(smem_u32(&acc_full[abuf]));
+            if (KIND != 0 && (kin == Cfg::CHUNK_KB - 1 || kb == KB - 1)) tc_commit<CL>(smem_u32(&acc_full[abuf]));
         }
         if (KIND == 0) tc_commit<CL>(smem_u32(&done_bar));
     } else if (warp >= 4) {
@@ -374,6 +381,19 @@ __global__ void __launch_bounds__(TcThreads<KIND>::N, TcCfg<KIND, CL>::MIN_BLOCK
                 if (lane == 0) {
                     if (CL > 1) mbar_arrive_cluster(ae0 + abuf * 8u);
                     else asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(ae0 + abuf * 8u) : "memory");
+                }
+            }
+            if (KIND == 2) {  // undo the operands' power-of-two row scales: 2^(eA_i) 2^(eB_j), exact
+                // exponents lie in [-115, 100] (split16_kernel), so 2^e is built from its bits
+                const float ra = __int_as_float((p.exps[rowA + q * 32 + lane] + 127) << 23);
+                const int4* eb = (const int4*)(p.exps + jb.n * p.nb + ccol0);
+#pragma unroll
+                for (int i = 0; i < COLS / 4; ++i) {
+                    const int4 e4 = __ldg(eb + i);
+                    sum[4 * i] = (sum[4 * i] * ra) * __int_as_float((e4.x + 127) << 23);
+                    sum[4 * i + 1] = (sum[4 * i + 1] * ra) * __int_as_float((e4.y + 127) << 23);
+                    sum[4 * i + 2] = (sum[4 * i + 2] * ra) * __int_as_float((e4.z + 127) << 23);
+                    sum[4 * i + 3] = (sum[4 * i + 3] * ra) * __int_as_float((e4.w + 127) << 23);
                 }
             }
             // the last acc_full also means every MMA (and so every shared-memory read of the ring,
@@ -447,6 +467,13 @@ static cudaError_t launch(const TcArgs& a, int njobs, cudaStream_t s) {
     if (KIND == 0) {
         ok = make_map(&p.a, a.p16, CU_TENSOR_MAP_DATA_TYPE_FLOAT16, 2, rows, a.nb, Cfg::BK, TC_BM) &&
              make_map(&p.b, a.p16, CU_TENSOR_MAP_DATA_TYPE_FLOAT16, 2, rows, a.nb, Cfg::BK, BROWS);
+    } else if (KIND == 2) {
+        ok = a.h16hi && a.h16lo && a.e16 &&
+             make_map(&p.a, a.h16hi, CU_TENSOR_MAP_DATA_TYPE_FLOAT16, 2, rows, a.nb, Cfg::BK, TC_BM) &&
+             make_map(&p.a_lo, a.h16lo, CU_TENSOR_MAP_DATA_TYPE_FLOAT16, 2, rows, a.nb, Cfg::BK, TC_BM) &&
+             make_map(&p.b, a.h16hi, CU_TENSOR_MAP_DATA_TYPE_FLOAT16, 2, rows, a.nb, Cfg::BK, BROWS) &&
+             make_map(&p.b_lo, a.h16lo, CU_TENSOR_MAP_DATA_TYPE_FLOAT16, 2, rows, a.nb, Cfg::BK, BROWS);
+        p.exps = a.e16;
     } else {
         ok = make_map(&p.a, a.hi, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 4, rows, a.nb, Cfg::BK, TC_BM) &&
              make_map(&p.a_lo, a.lo, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 4, rows, a.nb, Cfg::BK, TC_BM) &&
@@ -489,6 +516,7 @@ cudaError_t tc_gemm_f16_launch(const TcArgs& a, int njobs, cudaStream_t s) {
     static const int cl = env_cluster("MPGEO_TC16_CLUSTER", 2);
     return cl == 2 ? launch<0, 2>(a, njobs, s) : launch<0, 1>(a, njobs, s);
 }
+cudaError_t tc_gemm_f16x3_launch(const TcArgs& a, int njobs, cudaStream_t s) { return launch<2, 2>(a, njobs, s); }
 cudaError_t tc_gemm_tf32x3_launch(const TcArgs& a, int njobs, cudaStream_t s) {
     static const int cl = env_cluster("MPGEO_TC_CLUSTER", 2);
     return cl == 2 ? launch<1, 2>(a, njobs, s) : launch<1, 1>(a, njobs, s);

@@ -21,6 +21,11 @@ struct TcArgs {
     const float* lo;      // TF32 lo panel cache
     int nb, nt;
     const __half* p16;    // FP16 panel cache, [nt * nb][nb]
+    // 3xFP16 FP32-class operands (tc_gemm_f16x3_launch): row-scaled FP16 hi / lo panel caches
+    // [nt * nb][nb] and the per-row exponents e (x = 2^e (hi + lo) up to the split error)
+    const __half* h16hi = nullptr;
+    const __half* h16lo = nullptr;
+    const int* e16 = nullptr;
     // every TcJob::C lies in [cbase, cbase + crows * nb) at a whole row offset (the epilogue
     // reduces into C through one TMA tensor map over this range)
     const float* cbase;
@@ -29,4 +34,5 @@ struct TcArgs {
 bool tc_gemm_available();
 cudaError_t tc_gemm_tf32x3_launch(const TcArgs& a, int njobs, cudaStream_t s);
 cudaError_t tc_gemm_f16_launch(const TcArgs& a, int njobs, cudaStream_t s);
+cudaError_t tc_gemm_f16x3_launch(const TcArgs& a, int njobs, cudaStream_t s);
 }  // namespace mpgeo

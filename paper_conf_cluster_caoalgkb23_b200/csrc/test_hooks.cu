@@ -70,6 +70,48 @@ mp_status mp_test_tc_gemm(int kind, const void* d_panel, const void* d_panel_lo,
     return (e == cudaSuccess && e2 == cudaSuccess) ? MP_OK : MP_ERR_CUDA;
 }
 
+mp_status mp_test_tc_gemm_f16x3(const double* d_panel, float* d_C, int nb, int nt, int m, int n) {
+    if (!tc_gemm_available()) return MP_ERR_UNSUPPORTED;
+    const size_t elems = (size_t)nt * nb * nb;
+    __half *hi = nullptr, *lo = nullptr;
+    int* ex = nullptr;
+    TcJob j{m, n, d_C};
+    TcJob* dj = nullptr;
+    Split16Item* di = nullptr;
+    std::vector<Split16Item> items;
+    cudaError_t e = cudaMalloc(&hi, elems * 2);
+    if (e == cudaSuccess) e = cudaMalloc(&lo, elems * 2);
+    if (e == cudaSuccess) e = cudaMalloc(&ex, (size_t)nt * nb * sizeof(int));
+    if (e == cudaSuccess) e = cudaMalloc(&dj, sizeof j);
+    if (e == cudaSuccess) e = cudaMalloc(&di, nt * sizeof(Split16Item));
+    if (e == cudaSuccess) {
+        for (int t = 0; t < nt; ++t)
+            items.push_back({d_panel + (size_t)t * nb * nb, hi + (size_t)t * nb * nb, lo + (size_t)t * nb * nb, ex + (size_t)t * nb});
+        cudaMemcpy(dj, &j, sizeof j, cudaMemcpyHostToDevice);
+        cudaMemcpy(di, items.data(), nt * sizeof(Split16Item), cudaMemcpyHostToDevice);
+        e = split16_launch(di, nt, nb, 0);
+    }
+    if (e == cudaSuccess) {
+        TcArgs a{};
+        a.jobs = dj;
+        a.nb = nb;
+        a.nt = nt;
+        a.h16hi = hi;
+        a.h16lo = lo;
+        a.e16 = ex;
+        a.cbase = d_C;
+        a.crows = (uint64_t)nb;
+        e = tc_gemm_f16x3_launch(a, 1, 0);
+    }
+    cudaError_t e2 = cudaDeviceSynchronize();
+    cudaFree(hi);
+    cudaFree(lo);
+    cudaFree(ex);
+    cudaFree(dj);
+    cudaFree(di);
+    return (e == cudaSuccess && e2 == cudaSuccess) ? MP_OK : MP_ERR_CUDA;
+}
+
 int mp_tc_available(void) { return tc_gemm_available() ? 1 : 0; }
 
 mp_status mp_test_ozaki_gemm(const double* d_panel, double* d_C, int nb, int nt, int m, int n, int S, int lower) {

@@ -125,6 +125,36 @@ def test_tc_gemm_tf32x3_matches_sgemm_accuracy(lib):
     assert err_tc < err_1x / 50  # far better than a single TF32 product
 
 
+@pytest.mark.parametrize("spread", [0, 30])
+def test_tc_gemm_f16x3_matches_sgemm_accuracy(lib, spread):
+    """Reading C13c pin: 3xFP16 (row-scaled FP16 hi/lo split, kind::f16) error vs the exact product of
+    the FP32-rounded operands <= 2x the SGEMM error on the same inputs, also when row magnitudes
+    spread over 2^-spread .. 1 (the per-row power-of-two scales keep every row inside FP16 range);
+    a zero row gives a zero row of the product."""
+    nb, nt = 512, 2
+    rng = np.random.default_rng(5)
+    P = rng.standard_normal((nt * nb, nb)) * np.exp2(-rng.integers(0, spread + 1, size=(nt * nb, 1)))
+    P[nb + 3] = 0.0
+    Cm = np.zeros((nb, nb), np.float32)
+    dP, dC = dev(P), dev(Cm)
+    assert lib.mp_test_tc_gemm_f16x3(C.c_void_p(dP.data_ptr()), C.c_void_p(dC.data_ptr()), nb, nt, 1, 0) == 0
+    got = -dC.cpu().numpy().astype(np.float64)
+    A32 = P.astype(np.float32)
+    Ad = A32.astype(np.float64)
+    exact = Ad[nb:] @ Ad[:nb].T
+    sgemm = (A32[nb:] @ A32[:nb].T).astype(np.float64)
+    # row-wise relative errors (rows of different magnitude must each be accurate)
+    rn = np.linalg.norm(exact, axis=1)
+    ok = rn > 0
+    err_tc = np.max(np.linalg.norm(got - exact, axis=1)[ok] / rn[ok])
+    err_sg = np.max(np.linalg.norm(sgemm - exact, axis=1)[ok] / rn[ok])
+    assert err_tc <= 2 * err_sg + 1e-9, (err_tc, err_sg)
+    assert np.all(got[3] == 0.0)
+    single = (A32[nb:].astype(np.float16).astype(np.float64) @ A32[:nb].astype(np.float16).astype(np.float64).T)
+    if spread == 0:
+        assert err_tc < np.max(np.linalg.norm(single - exact, axis=1)[ok] / rn[ok]) / 50
+
+
 @pytest.mark.parametrize("S", [8])
 def test_ozaki_int8_fp64_gemm(lib, S):
     """FP64 GEMM emulated with int8 slices on tcgen05 kind::i8 vs the exact FP64 product: for S = 8

@@ -15,18 +15,20 @@ from tests.gpu_helpers import to_dev
 pytestmark = pytest.mark.gpu
 
 
-@pytest.fixture(scope="module", params=["16", "16t", "8", "0"], ids=["crt", "crt-tf32x3", "ozaki", "dmma"])
+@pytest.fixture(scope="module", params=["16", "16t", "16f", "8", "0"],
+                ids=["crt", "crt-tf32x3", "crt-f16x3", "ozaki", "dmma"])
 def engine_handle(request):
-    """crt: CRT FP64 class + CRT-8 FP32 class (MPGEO_CRT32=1); crt-tf32x3: CRT FP64 class + 3xTF32 (the
-    default engines)."""
+    """crt: CRT FP64 class + CRT-8 FP32 class (MPGEO_CRT32=1); crt-tf32x3: CRT FP64 class + 3xTF32
+    (MPGEO_F16X3=0); crt-f16x3: CRT FP64 class + 3xFP16 (the default engines)."""
     import paper_conf_cluster_caoalgkb23_b200 as mp
-    eng = request.param.rstrip("t")
+    eng = request.param.rstrip("tf")
     os.environ["MPGEO_OZAKI"] = eng
-    os.environ["MPGEO_CRT32"] = "0" if request.param.endswith("t") else "1"  # crt: the CRT-8 FP32 class (opt-in)
+    os.environ["MPGEO_CRT32"] = "0" if request.param[-1] in "tf" else "1"  # crt: the CRT-8 FP32 class (opt-in)
+    os.environ["MPGEO_F16X3"] = "0" if request.param.endswith("t") else "1"
     try:
         h = mp.Handle(0)
     finally:
-        del os.environ["MPGEO_OZAKI"], os.environ["MPGEO_CRT32"]
+        del os.environ["MPGEO_OZAKI"], os.environ["MPGEO_CRT32"], os.environ["MPGEO_F16X3"]
     oz = h.config()["ozaki"]
     assert oz % 100 == int(eng)
     assert (oz >= 200) == (request.param == "16")
