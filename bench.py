@@ -366,8 +366,9 @@ def main():
     last = reps[-1]
     upd = list(last.flops_update)
     fp64_class_peak = (int8_peak / eng[0]) if eng else fp64_peak
-    # FP32-class engine: CRT-8 (8 INT8 GEMMs, ozaki >= 200), 4-slice split (10 INT8 GEMMs, >= 100), 3xTF32
+    # FP32-class engine: CRT-8 (8 INT8 GEMMs, ozaki >= 200), 4-slice split (10 INT8 GEMMs, >= 100), 3xFP16 (tc 2), 3xTF32
     fp32_class_peak = ((int8_peak / 8) if engine["ozaki"] >= 200 else (int8_peak / 10) if engine["ozaki"] >= 100
+                       else peaks["bf16_tflops_sustained"] / 3 if engine["tc"] == 2  # 3xFP16 at the f16 rate
                        else peaks["bf16_tflops_sustained"] * 0.5 / 3)
     roof_time_s = (upd[0] / (fp64_class_peak * 1e12)
                    + upd[1] / (fp32_class_peak * 1e12)
@@ -384,7 +385,8 @@ def main():
                    "fp64_engine": eng[2] if eng else "dmma",
                    "fp32_engine": ("crt-int8 (8 moduli, FP32 C)" if engine["ozaki"] >= 200 else
                                    "ozaki-int8 (S=4)" if engine["ozaki"] >= 100 else
-                                   ("tcgen05 3xTF32" if engine["tc"] else "dmma-rounded")),
+                                   ("tcgen05 3xFP16 (row-scaled)" if engine["tc"] == 2 else
+                                    "tcgen05 3xTF32" if engine["tc"] else "dmma-rounded")),
                    "fp16_engine": "tcgen05 f16" if engine["tc"] else "dmma-rounded", "lookahead": engine["lookahead"],
                    "parallelism": (f"2D block-cyclic {P}x{Q}, peer-memory panel exchange" if distributed
                                    else ("replicas" if world > 1 else "1 GPU")),

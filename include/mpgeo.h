@@ -263,7 +263,8 @@ mp_status mp_set_profiling(mp_handle* h, int enable);  /* enable also resets the
 mp_status mp_get_profile(mp_handle* h, mp_profile* out);  /* synchronises the stream */
 
 /* Engine configuration of a handle (read from MPGEO_* at mp_init): tcgen05 kernels for the FP32
- * and FP16 classes (1) or DMMA on rounded operands (0); panel lookahead (1/0); FP64-class
+ * and FP16 classes (1: FP32 class as 3xTF32; 2: FP32 class as row-scaled 3xFP16, the default) or DMMA
+ * on rounded operands (0); panel lookahead (1/0); FP64-class
  * engine: 16 = CRT (16 moduli) and 8 = Ozaki split (8 int8 slices), both on tcgen05 kind::i8, 0 = DMMA
  * FP64; + 200 if the FP32 class runs as CRT-8 (8 moduli), + 100 if as the 4-slice split. */
 mp_status mp_handle_config(const mp_handle* h, int* tc, int* lookahead, int* ozaki);

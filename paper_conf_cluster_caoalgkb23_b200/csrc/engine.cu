@@ -399,7 +399,7 @@ int64_t mp_launch_count(const mp_handle* h) { return h ? h->launches : 0; }
 mp_status mp_handle_config(const mp_handle* h, int* tc, int* lookahead, int* ozaki) {
     if (!h) return MP_ERR_ARG;
     // ozaki: 0 = DMMA FP64 class; 8 = INT8 FP64 class; +100 if the FP32 class also runs on INT8
-    if (tc) *tc = (h->tc_mode != 0 && tc_gemm_available()) ? 1 : 0;
+    if (tc) *tc = (h->tc_mode != 0 && tc_gemm_available()) ? (h->f16x3 ? 2 : 1) : 0;
     if (lookahead) *lookahead = h->lookahead;
     if (ozaki)
         *ozaki = (h->ozaki == 16 && crt_available()) ? (16 + (h->crt32 ? 200 : 0))
