@@ -30,12 +30,16 @@
 namespace mpgeo {
 
 constexpr int TC_BM = 128;  // output rows per CTA (TMEM lanes)
+#ifndef TC16X3_EPI_WARPS
+#define TC16X3_EPI_WARPS 8
+#endif
 #ifndef TC16X3_CHUNK_KB
 #define TC16X3_CHUNK_KB 2  // KIND 2: k-blocks of 64 per TMEM accumulator chunk (K = 128; measured 187 vs 181 Tflop/s at K = 64)
 #endif
 template <int KIND>
 struct TcThreads {
-    static constexpr int EPI_WARPS = KIND == 0 ? 4 : 8;  // 3xTF32: two warpgroups, one per 128-column half
+    // 3xTF32: two warpgroups, one per 128-column half; 3xFP16: TC16X3_EPI_WARPS / 4 column groups
+    static constexpr int EPI_WARPS = KIND == 0 ? 4 : KIND == 1 ? 8 : TC16X3_EPI_WARPS;
     static constexpr int N = (4 + EPI_WARPS) * 32;
 };
 
@@ -102,6 +106,12 @@ __device__ __forceinline__ uint32_t cluster_addr(uint32_t saddr, uint32_t rank) 
 }
 __device__ __forceinline__ void mbar_arrive_cluster(uint32_t cbar) {
     asm volatile("mbarrier.arrive.release.cluster.shared::cluster.b64 _, [%0];" ::"r"(cbar) : "memory");
+}
+// relaxed arrive: the epilogue only signals that its tcgen05.ld of the accumulator completed
+// (wait::ld), which orders nothing else, so no release (a release adds a MEMBAR per chunk: 21% of
+// the 3xFP16 kernel's stalls, profiles/r01/s4_ncu_f16x3_summary.txt)
+__device__ __forceinline__ void mbar_arrive_cluster_relaxed(uint32_t cbar) {
+    asm volatile("mbarrier.arrive.relaxed.cluster.shared::cluster.b64 _, [%0];" ::"r"(cbar) : "memory");
 }
 __device__ __forceinline__ uint32_t cluster_rank() {
     uint32_t r;
@@ -379,7 +389,7 @@ __global__ void __launch_bounds__(TcThreads<KIND>::N, TcCfg<KIND, CL>::MIN_BLOCK
                 tc_fence_before();
                 __syncwarp();
                 if (lane == 0) {
-                    if (CL > 1) mbar_arrive_cluster(ae0 + abuf * 8u);
+                    if (CL > 1) mbar_arrive_cluster_relaxed(ae0 + abuf * 8u);
                     else asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(ae0 + abuf * 8u) : "memory");
                 }
             }
