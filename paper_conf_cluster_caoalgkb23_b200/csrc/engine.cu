@@ -1233,6 +1233,7 @@ static mp_status plan_potrf(mp_handle* h, mp_matrix* A, const uint8_t* km, const
                 ta.h16hi = (const __half*)phi;
                 ta.h16lo = (const __half*)phi + (size_t)nt * nb2;
                 ta.e16 = (const int*)plo;
+                ta.pairs = upd_pairs;  // lookahead: leave SMs to the panel stream (0: all)
                 cur->push_back({[=](cudaStream_t s) { return tc_gemm_f16x3_launch(ta, nj, s); }, C_UPD32, 2 * f3 * nj});
             } else {
                 cur->push_back({[=](cudaStream_t s) { return tc_gemm_tf32x3_launch(ta, nj, s); }, C_UPD32, 2 * f3 * nj});

@@ -49,6 +49,7 @@ struct __align__(64) TcParams {
     const float* cbase;
     const int* exps;  // KIND 2: per panel-cache row, 2^exps undoes the operand scale
     int nb, tiles_n, tiles_per_job;
+    int total;        // persistent kernel: pair tiles of the launch
 };
 
 // CL = CTAs per MMA: 1 (tcgen05.mma.cta_group::1, M = 128) or 2 (a CTA pair on one TPC,
@@ -212,6 +213,18 @@ __device__ __forceinline__ void stage_box_neg(uint32_t buf, int lane, const floa
     }
     asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
     __syncwarp();
+}
+// 3xFP16: v_j *= 2^(e_row) 2^(e_col j) for one 32-column group (exponents in [-115, 100], so each
+// power of two is built from its bits)
+__device__ __forceinline__ void scale_group(float* v, float ra, const int4* eb) {
+#pragma unroll
+    for (int i = 0; i < 8; ++i) {
+        const int4 e4 = __ldg(eb + i);
+        v[4 * i] = (v[4 * i] * ra) * __int_as_float((e4.x + 127) << 23);
+        v[4 * i + 1] = (v[4 * i + 1] * ra) * __int_as_float((e4.y + 127) << 23);
+        v[4 * i + 2] = (v[4 * i + 2] * ra) * __int_as_float((e4.z + 127) << 23);
+        v[4 * i + 3] = (v[4 * i + 3] * ra) * __int_as_float((e4.w + 127) << 23);
+    }
 }
 __device__ __forceinline__ void tma_reduce_add(const CUtensorMap* map, uint32_t buf, int c0, int c1) {
     asm volatile("cp.reduce.async.bulk.tensor.2d.global.shared::cta.add.tile.bulk_group [%0, {%2, %3}], [%1];" ::"l"(
@@ -398,13 +411,7 @@ __global__ void __launch_bounds__(TcThreads<KIND>::N, TcCfg<KIND, CL>::MIN_BLOCK
                 const float ra = __int_as_float((p.exps[rowA + q * 32 + lane] + 127) << 23);
                 const int4* eb = (const int4*)(p.exps + jb.n * p.nb + ccol0);
 #pragma unroll
-                for (int i = 0; i < COLS / 4; ++i) {
-                    const int4 e4 = __ldg(eb + i);
-                    sum[4 * i] = (sum[4 * i] * ra) * __int_as_float((e4.x + 127) << 23);
-                    sum[4 * i + 1] = (sum[4 * i + 1] * ra) * __int_as_float((e4.y + 127) << 23);
-                    sum[4 * i + 2] = (sum[4 * i + 2] * ra) * __int_as_float((e4.z + 127) << 23);
-                    sum[4 * i + 3] = (sum[4 * i + 3] * ra) * __int_as_float((e4.w + 127) << 23);
-                }
+                for (int gi = 0; gi < COLS / 32; ++gi) scale_group(sum + gi * 32, ra, eb + gi * 8);
             }
             // the last acc_full also means every MMA (and so every shared-memory read of the ring,
             // in both CTAs of a pair) has completed
@@ -424,6 +431,170 @@ __global__ void __launch_bounds__(TcThreads<KIND>::N, TcCfg<KIND, CL>::MIN_BLOCK
     tc_fence_before();
     if (CL > 1) cluster_sync();  // neither CTA frees TMEM / exits while its peer may still signal it
     else __syncthreads();
+    if (warp == 2) {
+        tc_fence_after();
+        tmem_dealloc<CL>(tmem, Cfg::TMEM_COLS);
+    }
+}
+
+// Persistent 3xFP16 (KIND 2) kernel: CTA pairs loop over the pair tiles of the launch (static
+// round robin), so the MMAs of the next tile run while the epilogue scales the finished FP32 sums
+// (registers) and reduces them into C — the accumulators are free once the last chunk is drained.
+// The staging boxes get their own shared memory (the stage ring stays busy across tiles).
+constexpr int P16_STAGES = 3;
+constexpr int P16_EPI = 8;
+constexpr int P16_STG = 4096;  // one 32 x 32 FP32 box per epilogue warp
+constexpr int P16_SMEM = P16_STAGES * TcCfg<2, 2>::STAGE_BYTES + P16_EPI * P16_STG + 1024;
+
+__global__ void __launch_bounds__((4 + P16_EPI) * 32, 1) tc_f16x3_persistent_kernel(const __grid_constant__ TcParams p) {
+    using Cfg = TcCfg<2, 2>;
+    constexpr int CL = 2;
+    extern __shared__ uint8_t smem_raw[];
+    uint8_t* smem = (uint8_t*)(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
+    __shared__ __align__(8) uint64_t full_bar[P16_STAGES], empty_bar[P16_STAGES];
+    __shared__ __align__(8) uint64_t acc_full[2], acc_empty[2];
+    __shared__ uint32_t tmem_slot;
+
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    const uint32_t crank = cluster_rank();
+    const int pair = blockIdx.x / CL, npairs = gridDim.x / CL;
+    const int KB = p.nb / Cfg::BK;
+    const int nchunks = (KB + Cfg::CHUNK_KB - 1) / Cfg::CHUNK_KB;
+
+    if (threadIdx.x == 0) {
+        for (int s = 0; s < P16_STAGES; ++s) {
+            mbar_init(smem_u32(&full_bar[s]), 1);
+            mbar_init(smem_u32(&empty_bar[s]), 1);
+        }
+        for (int i = 0; i < 2; ++i) {
+            mbar_init(smem_u32(&acc_full[i]), 1);
+            mbar_init(smem_u32(&acc_empty[i]), CL * P16_EPI);
+        }
+        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+        asm volatile("prefetch.tensormap [%0];" ::"l"((uint64_t)&p.a) : "memory");
+        asm volatile("prefetch.tensormap [%0];" ::"l"((uint64_t)&p.b) : "memory");
+    }
+    if (warp == 2) tmem_alloc<CL>(smem_u32(&tmem_slot), Cfg::TMEM_COLS);
+    tc_fence_before();
+    cluster_sync();
+    tc_fence_after();
+    const uint32_t tmem = tmem_slot;
+
+    auto coords = [&](int t, int& job, int& bi, int& bj) {
+        job = t / p.tiles_per_job;
+        const int u = t - job * p.tiles_per_job;
+        bi = u / p.tiles_n;
+        bj = u - bi * p.tiles_n;
+    };
+
+    if (warp == 0 && lane == 0) {
+        uint32_t it = 0;
+        for (int t = pair; t < p.total; t += npairs) {
+            int job, bi, bj;
+            coords(t, job, bi, bj);
+            const TcJob jb = p.jobs[job];
+            const int rowA = jb.m * p.nb + bi * Cfg::BM + (int)crank * TC_BM;
+            const int rowB = jb.n * p.nb + bj * Cfg::BN + (int)crank * (Cfg::BN / CL);
+            for (int kb = 0; kb < KB; ++kb, ++it) {
+                const uint32_t s = it % P16_STAGES;
+                const uint32_t ph = (it / P16_STAGES) & 1u;
+                mbar_wait(smem_u32(&empty_bar[s]), ph ^ 1u);
+                const uint32_t st = smem_u32(smem + s * Cfg::STAGE_BYTES);
+                const uint32_t lb = smem_u32(&full_bar[s]);
+                const uint32_t fb = cluster_addr(lb, 0);
+                if (crank == 0) mbar_expect_tx(lb, CL * Cfg::STAGE_BYTES);
+                const int kc = kb * Cfg::BK;
+                tma_load_2d<CL>(st, &p.a, fb, kc, rowA);
+                tma_load_2d<CL>(st + Cfg::A_BYTES, &p.a_lo, fb, kc, rowA);
+                tma_load_2d<CL>(st + 2 * Cfg::A_BYTES, &p.b, fb, kc, rowB);
+                tma_load_2d<CL>(st + 2 * Cfg::A_BYTES + Cfg::B_BYTES, &p.b_lo, fb, kc, rowB);
+            }
+        }
+    } else if (warp == 1 && lane == 0 && crank == 0) {
+        uint32_t it = 0, g = 0;
+        for (int t = pair; t < p.total; t += npairs) {
+            for (int kb = 0; kb < KB; ++kb, ++it) {
+                const uint32_t s = it % P16_STAGES;
+                const uint32_t ph = (it / P16_STAGES) & 1u;
+                const int kin = kb % Cfg::CHUNK_KB;
+                const uint32_t abuf = g & 1u;
+                const uint32_t dacc = tmem + abuf * Cfg::BN;
+                if (kin == 0) {
+                    mbar_wait(smem_u32(&acc_empty[abuf]), ((g >> 1) & 1u) ^ 1u);
+                    tc_fence_after();
+                }
+                mbar_wait(smem_u32(&full_bar[s]), ph);
+                tc_fence_after();
+                const uint32_t base = smem_u32(smem + s * Cfg::STAGE_BYTES);
+#pragma unroll
+                for (int k = 0; k < Cfg::BK / Cfg::UK; ++k) {
+                    const uint32_t koff = k * 32;
+                    const uint32_t acc = (kin | k) != 0;
+                    const uint64_t ahi = desc_sw128(base + koff);
+                    const uint64_t alo = desc_sw128(base + Cfg::A_BYTES + koff);
+                    const uint64_t bhi = desc_sw128(base + 2 * Cfg::A_BYTES + koff);
+                    const uint64_t blo = desc_sw128(base + 2 * Cfg::A_BYTES + Cfg::B_BYTES + koff);
+                    tc_mma<2, CL>(dacc, alo, bhi, acc);
+                    tc_mma<2, CL>(dacc, ahi, blo, 1u);
+                    tc_mma<2, CL>(dacc, ahi, bhi, 1u);
+                }
+                tc_commit<CL>(smem_u32(&empty_bar[s]));
+                if (kin == Cfg::CHUNK_KB - 1 || kb == KB - 1) {
+                    tc_commit<CL>(smem_u32(&acc_full[abuf]));
+                    ++g;
+                }
+            }
+        }
+    } else if (warp >= 4) {
+        constexpr int COLS = Cfg::BN / (P16_EPI / 4);
+        const int q = (warp - 4) & 3;
+        const int half = (warp - 4) >> 2;
+        const uint32_t tl = ((uint32_t)(q * 32) << 16) + (uint32_t)(half * COLS);
+        const uint32_t stg = smem_u32(smem + P16_STAGES * Cfg::STAGE_BYTES) + (uint32_t)(warp - 4) * P16_STG;
+        const uint32_t ae0 = cluster_addr(smem_u32(&acc_empty[0]), 0);
+        uint32_t g = 0;
+        for (int t = pair; t < p.total; t += npairs) {
+            int job, bi, bj;
+            coords(t, job, bi, bj);
+            const TcJob jb = p.jobs[job];
+            const int rowA = jb.m * p.nb + bi * Cfg::BM + (int)crank * TC_BM;
+            const int crow0 = (int)((jb.C - p.cbase) / p.nb) + bi * Cfg::BM + (int)crank * TC_BM + q * 32;
+            const int ccol0 = bj * Cfg::BN + half * COLS;
+            float sum[COLS];
+#pragma unroll
+            for (int i = 0; i < COLS; ++i) sum[i] = 0.f;
+#pragma unroll 1
+            for (int c = 0; c < nchunks; ++c, ++g) {
+                const uint32_t abuf = g & 1u;
+                mbar_wait(smem_u32(&acc_full[abuf]), (g >> 1) & 1u);
+                tc_fence_after();
+#pragma unroll
+                for (int c0 = 0; c0 < COLS; c0 += 32) {
+                    uint32_t r[32];
+                    tmem_ld32(tmem + tl + abuf * Cfg::BN + (uint32_t)c0, r);
+#pragma unroll
+                    for (int v = 0; v < 32; ++v) sum[c0 + v] += __uint_as_float(r[v]);
+                }
+                tc_fence_before();
+                __syncwarp();
+                if (lane == 0) mbar_arrive_cluster_relaxed(ae0 + abuf * 8u);
+            }
+            // the accumulators are released: the next tile's MMAs overlap the scaling and C update
+            const float ra = __int_as_float((p.exps[rowA + q * 32 + lane] + 127) << 23);
+            const int4* eb = (const int4*)(p.exps + jb.n * p.nb + ccol0);
+#pragma unroll
+            for (int gi = 0; gi < COLS / 32; ++gi) {
+                scale_group(sum + gi * 32, ra, eb + gi * 8);
+                if (lane == 0) asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory");  // box free again
+                __syncwarp();
+                stage_box_neg(stg, lane, sum + gi * 32);
+                if (lane == 0) tma_reduce_add(&p.c, stg, ccol0 + gi * 32, crow0);
+            }
+        }
+        if (lane == 0) bulk_wait_all();
+    }
+    tc_fence_before();
+    cluster_sync();
     if (warp == 2) {
         tc_fence_after();
         tmem_dealloc<CL>(tmem, Cfg::TMEM_COLS);
@@ -457,6 +628,29 @@ static bool make_map(CUtensorMap* m, const void* base, CUtensorMapDataType dt, i
 }
 
 bool tc_gemm_available() { return encode_fn() != nullptr; }
+
+static int tc_sm_count() {
+    static int n = 0;
+    if (!n) {
+        int dev = 0;
+        cudaGetDevice(&dev);
+        cudaDeviceGetAttribute(&n, cudaDevAttrMultiProcessorCount, dev);
+        if (n <= 0) n = 148;
+    }
+    return n;
+}
+// MPGEO_TC16X3_PERSIST=1: the persistent 3xFP16 kernel (opt-in).  Measured at C3 (profiles/r01,
+// s4_persist_*.json): the FP32-class update drops from 1.88 to 1.27-1.35 s, but the evaluation does
+// not gain (183.6-186.5 vs 187.1 Tflop/s): the GPU runs at its power cap, so the denser kernel
+// lowers the clock for the CRT and FP16 launches, and with reserved pairs the panel stream gets
+// fewer SMs (conversions 0.41 -> 0.85 s).  Default: one CTA pair per output tile.
+static bool tc16x3_persistent() {
+    static const int v = [] {
+        const char* e = getenv("MPGEO_TC16X3_PERSIST");
+        return e ? atoi(e) : 0;
+    }();
+    return v != 0;
+}
 
 template <int KIND, int CL>
 static cudaError_t launch(const TcArgs& a, int njobs, cudaStream_t s) {
@@ -498,12 +692,32 @@ static cudaError_t launch(const TcArgs& a, int njobs, cudaStream_t s) {
     p.nb = a.nb;
     p.tiles_n = a.nb / Cfg::BN;
     p.tiles_per_job = (a.nb / Cfg::BM) * p.tiles_n;
-    const long long grid = (long long)njobs * p.tiles_per_job * CL;
+    long long grid = (long long)njobs * p.tiles_per_job * CL;
     if (grid > 0x7fffffffLL) return cudaErrorInvalidConfiguration;
+    void (*kern)(TcParams) = tc_gemm_kernel<KIND, CL>;
+    int smem_bytes = Cfg::SMEM;
+    if (KIND == 2 && CL == 2 && tc16x3_persistent()) {
+        static bool pattr = false;
+        if (!pattr) {
+            cudaError_t e = cudaFuncSetAttribute(tc_f16x3_persistent_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, P16_SMEM);
+            if (e != cudaSuccess) return e;
+            pattr = true;
+        }
+        p.total = (int)(grid / CL);
+        static const int env_pairs = [] {  // MPGEO_TC16X3_PAIRS: override of the pair count
+            const char* e = getenv("MPGEO_TC16X3_PAIRS");
+            return e ? atoi(e) : 0;
+        }();
+        int pairs = env_pairs > 0 ? env_pairs : a.pairs > 0 ? a.pairs : tc_sm_count() / 2;
+        if (pairs > p.total) pairs = p.total;
+        grid = (long long)pairs * CL;
+        kern = tc_f16x3_persistent_kernel;
+        smem_bytes = P16_SMEM;
+    }
     cudaLaunchConfig_t cfg = {};
     cfg.gridDim = dim3((unsigned)grid);
-    cfg.blockDim = dim3(TcThreads<KIND>::N);
-    cfg.dynamicSmemBytes = Cfg::SMEM;
+    cfg.blockDim = dim3(kern == tc_f16x3_persistent_kernel ? (4 + P16_EPI) * 32 : TcThreads<KIND>::N);
+    cfg.dynamicSmemBytes = smem_bytes;
     cfg.stream = s;
     cudaLaunchAttribute at[1];
     at[0].id = cudaLaunchAttributeClusterDimension;
@@ -512,7 +726,7 @@ static cudaError_t launch(const TcArgs& a, int njobs, cudaStream_t s) {
     at[0].val.clusterDim.z = 1;
     cfg.attrs = at;
     cfg.numAttrs = 1;
-    return cudaLaunchKernelEx(&cfg, tc_gemm_kernel<KIND, CL>, p);
+    return cudaLaunchKernelEx(&cfg, kern, p);
 }
 
 // CTAs per MMA: MPGEO_TC_CLUSTER (3xTF32) and MPGEO_TC16_CLUSTER (FP16); default 2 = CTA pairs (faster

@@ -26,6 +26,7 @@ struct TcArgs {
     const __half* h16hi = nullptr;
     const __half* h16lo = nullptr;
     const int* e16 = nullptr;
+    int pairs = 0;  // persistent 3xFP16 kernel: CTA pairs to use (0: all SMs / 2)
     // every TcJob::C lies in [cbase, cbase + crows * nb) at a whole row offset (the epilogue
     // reduces into C through one TMA tensor map over this range)
     const float* cbase;
