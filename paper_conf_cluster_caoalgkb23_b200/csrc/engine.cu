@@ -287,7 +287,9 @@ static mp_status run_plan(mp_handle* h, mp_matrix* A, Arena& ar, std::vector<Op>
 // ------------------------------------------------------------------ lifecycle
 extern "C" {
 
-const char* mp_version(void) { return "mpgeo 0.1 sm_100a (DMMA FP64, tcgen05 TF32x3/FP16)"; }
+const char* mp_version(void) {
+    return "mpgeo 0.1 sm_100a (FP64 class: CRT INT8 tcgen05 | 8-slice | DMMA; FP32 class: 3xFP16 | 3xTF32; FP16 class: tcgen05 f16)";
+}
 
 mp_status mp_init(int device, int rank, int nranks, int P, int Q, const uint8_t* id, void* cuda_stream,
                   mp_handle** out) {
