@@ -20,18 +20,28 @@ Modules (each function cites the passage it follows):
 
 Pins (what fixes each part independently of this code; tests/test_oracle_*.py):
   matern     — closed forms nu = 1/2, 3/2, 5/2; mpmath.besselk at 40 digits;
-               C(0) = sigma^2; Bessel three-term recurrence.               pinned
+               C(0) = sigma^2; monotone decay in h.                         pinned
+  tiles      — tile_sqnorm / global_sqnorm against the dense ||A||_F^2 of the
+               whole symmetric matrix and against hand-derived closed forms of
+               the Kac-Murdock-Szego matrix per tile; correct rounding on
+               hand-built sums (test_oracle_pins.py).                       pinned
   cholesky / loglik — Kac-Murdock-Szego closed forms (L, log|Sigma|, Z^T Sigma^-1 Z);
-               mpmath 50-digit determinant and solve at n <= 48;
-               residual ||A - L L^T||_F / ||A||_F <= 1e-13.                 pinned
+               mpmath 50-digit determinant and solve at n = 40;
+               tile factor vs dense LAPACK; non-SPD `info`.                  pinned
+  residual   — hand-computed 2 x 2 example (both triangles of A).           pinned
   precision (kernel/storage map) — hand-built norm arrays with known
-               answers, tie -> lower precision, monotonicity in u_req.       pinned
+               answers (ties at both thresholds), one tile on each side of
+               each threshold, literal storage table, monotonicity.          pinned
+  precision (band map, reading C21) — hand-built norms with a known band,
+               both too-narrow and too-wide checked.                         pinned
   precision (comm map, Alg. 2) — text claims: all-FP64 map -> comm FP64;
-               extreme FP64/FP16 map -> every communication STC.
-               The paper's Fig. 4b example is an image (absent):  that
-               example is parity unpinned.                                  partially pinned
-  cholesky MP-emulation mode — predicts the MP error only; the MP pass
-               criterion is the FP64 oracle with the north-star tolerance.  parity unpinned (emulation)
+               extreme FP64/FP16 map -> every communication STC (P:294);
+               hand-built successor cases.  The paper's Fig. 4b example is
+               an image (absent): that example is parity unpinned.          partially pinned
+  cholesky MP-emulation mode — predicts the MP error only and is NOT a pass
+               criterion anywhere: the MP tests compare the GPU with the FP64
+               definition (north-star tolerance) and with a backward-error
+               bound computed from the maps.                                parity unpinned (emulation)
 """
 
 FP64, FP32, FP16 = 0, 1, 2  # smaller value = higher precision (SURVEY §8(b) mp_prec)
