@@ -100,17 +100,68 @@ typedef struct {
     int64_t tiles[3];             /* lower off-diagonal tiles per kernel precision */
     int64_t stc_tiles;            /* off-diagonal tiles whose comm precision < storage */
     int64_t gpu_launches;         /* kernels launched by this call */
+    uint64_t workspace_bytes;     /* bytes this evaluation's map needs (set also on MP_ERR_NOMEM) */
 } mp_eval_report;
+
+/* ---------------------------------------------------------------- configuration */
+
+/* Engines of the precision classes (the arithmetic each class of Algorithm 1 runs on). */
+typedef enum {
+    MP_F64_CRT16 = 0,  /* FP64 class (DSYRK, FP64 GEMM) as 16 exact INT8 tcgen05 GEMMs + CRT
+                          reconstruction (Ozaki scheme II): per-row normwise error
+                          <= K 2^-(b+1) max_l|a_il| max_l|b_jl|, b = 56 at nb = 2048 (needs nb % 256 == 0,
+                          else DMMA) */
+    MP_F64_DMMA = 1    /* FP64 class on the FP64 DMMA tensor cores (native FP64, componentwise bound) */
+} mp_fp64_engine;
+typedef enum {
+    MP_F32_3XFP16 = 0, /* FP32 class as 3xFP16 on tcgen05 kind::f16: row-scaled 11 + 11-bit hi/lo split,
+                          FP32 chunk sums (reading C13c); per-row normwise bound (needs nb % 256 == 0) */
+    MP_F32_3XTF32 = 1, /* FP32 class as 3xTF32 on tcgen05 kind::tf32 (reading C13) */
+    MP_F32_DMMA = 2    /* FP32 class on DMMA with FP32-rounded operands and an FP32 C (reference engine) */
+} mp_fp32_engine;
+
+/* Handle configuration (read once by mp_init_config; every field has a default). */
+typedef struct {
+    int fp64_engine;      /* mp_fp64_engine, default MP_F64_CRT16 */
+    int fp32_engine;      /* mp_fp32_engine, default MP_F32_3XFP16 */
+    int fp16_tensor;      /* 1 (default): FP16 class on tcgen05 kind::f16 with row-scaled FP16 operands;
+                             0: DMMA with FP16-rounded operands (reference engine) */
+    int lookahead;        /* 1 (default): panel k+1 (POTRF, TRSM) on a high-priority stream overlaps the
+                             trailing update of panel k; 0: one stream, strict Algorithm 1 order */
+    int reserve_pairs;    /* CTA pairs the persistent update kernels leave to the panel stream (default 6) */
+    int lowp_trsm_product;/* 1 (default, with MP_F64_CRT16): TRSM of FP32/FP16-class tiles as the FP32-class
+                             product A_mk W^T, W = L~_kk^-1 (reading C12'); 0: FP64 substitution */
+    int matern_table;     /* 1 (default): general nu through the per-evaluation Chebyshev table of the
+                             correlation; 0: K_nu evaluated per entry */
+    int f16x3_persistent; /* 1: persistent-CTA 3xFP16 kernel; 0 (default): one CTA pair per output tile */
+    int crt_phase_lock;   /* 1 (default): CRT tiles start at the modulus pair the other CTAs are on */
+} mp_config;
+
+/* Fill *cfg with the defaults above. */
+void mp_config_default(mp_config* cfg);
 
 /* ---------------------------------------------------------------- lifecycle */
 
+/* A 128-byte communicator id (SURVEY §8(b) mp_get_unique_id): random bytes from the OS plus this
+ * host's name and process id.  Rank 0 creates it and broadcasts it to the other ranks (e.g.
+ * torch.distributed); every rank passes it to mp_init.  The multi-rank exchange (mp_matrix_comm_*)
+ * writes it into the header of each rank's exchange area and mp_matrix_comm_connect refuses to map
+ * a peer whose id differs (MP_ERR_COMM), so areas of two different jobs can never be mixed.  The
+ * transport itself is CUDA IPC peer memory, which needs no other bootstrap. */
+mp_status mp_get_unique_id(uint8_t id[128]);
+
 /* Create a handle on CUDA `device` for `rank` of `nranks` (P * Q == nranks,
- * P <= Q, nranks <= 8).  `id` is reserved (pass NULL).  `cuda_stream` is a
- * cudaStream_t (NULL = a stream created and owned by the handle).  *h receives
- * the handle.  Multi-rank matrices exchange panel tiles through peer memory: see
- * mp_matrix_comm_export / mp_matrix_comm_connect. */
+ * P <= Q, nranks <= 8).  `id`: the communicator id of mp_get_unique_id (required when nranks > 1,
+ * may be NULL for one rank).  `cuda_stream` is a cudaStream_t (NULL = a stream created and owned by
+ * the handle).  `cfg` may be NULL (defaults).  *h receives the handle.  Multi-rank matrices exchange
+ * panel tiles through peer memory: see mp_matrix_comm_export / mp_matrix_comm_connect. */
+mp_status mp_init_config(int device, int rank, int nranks, int P, int Q, const uint8_t* id, void* cuda_stream,
+                         const mp_config* cfg, mp_handle** h);
+/* mp_init_config with the default configuration. */
 mp_status mp_init(int device, int rank, int nranks, int P, int Q, const uint8_t* id,
                   void* cuda_stream, mp_handle** h);
+/* The configuration the handle runs with. */
+mp_status mp_handle_get_config(const mp_handle* h, mp_config* cfg);
 mp_status mp_finalize(mp_handle* h);
 const char* mp_last_error(const mp_handle* h);
 
@@ -122,14 +173,22 @@ mp_status mp_matrix_create(mp_handle* h, int64_t n, int nb, mp_matrix** A);
 mp_status mp_matrix_destroy(mp_matrix* A);
 
 /* Device bytes needed to bind A with the given storage map (NULL = all FP64, the
- * worst case): owned tiles in storage precision, the FP64 panel buffer and the
- * low-precision panel caches (K2), communication staging, solve scratch. */
+ * worst case): the map-independent regions (inputs, norms, control arena, the panel buffers and
+ * operand caches of ONE panel — K2 formats are single-buffered) followed by the
+ * owned tiles in storage precision. */
 mp_status mp_matrix_bytes(const mp_matrix* A, const uint8_t* storage_prec, size_t* bytes);
 
 /* Lay out A inside the caller's device workspace (256-byte aligned) for the
  * storage map (NULL = all FP64).  May be called again with a new map on the
  * same workspace (each MLE evaluation has its own map); contents are lost. */
 mp_status mp_matrix_bind(mp_matrix* A, const uint8_t* storage_prec, void* d_workspace, size_t bytes);
+
+/* Give A a caller-owned workspace for mp_eval without laying out a tile pool: every mp_eval then
+ * binds its own map inside it.  `bytes` must cover at least the map-independent regions
+ * (mp_matrix_bytes of the all-FP32 off-diagonal map is a safe minimum); an evaluation whose map
+ * needs more returns MP_ERR_NOMEM with report->workspace_bytes set, so the caller can grow the
+ * workspace (sized by the map, not by an all-FP64 worst case) and repeat the call. */
+mp_status mp_matrix_attach(mp_matrix* A, void* d_workspace, size_t bytes);
 
 /* Multi-rank only (nranks > 1), once per matrix, before its first use:
  * mp_matrix_comm_export allocates this rank's exchange area (send slots in
@@ -191,12 +250,13 @@ mp_status mp_precision_map(int nt, const double* tile_sqnorm, double u_req, cons
                            uint8_t* comm_prec);
 
 /* (3) In-place mixed-precision tile Cholesky A = L L^T (Algorithm 1):
- * DPOTRF (FP64) on diagonal tiles; TRSM(m,k) with L_kk received at
- * comm(k,k) (FP64 arithmetic, result rounded to storage(m,k)); L_mk reaches its
- * successors at comm(m,k) and is converted on the consuming GPU to the
- * successor's kernel precision; DSYRK in FP64; GEMM(m,n,k) at
- * kernel(m,n): FP64 on DMMA tensor cores, FP32 class as 3xTF32 and FP16 class
- * as FP16xFP16->FP32 on tcgen05 tensor cores, accumulating into the FP32 tile.
+ * DPOTRF (FP64) on diagonal tiles; TRSM(m,k) with L_kk received at comm(k,k): FP64 substitution
+ * for FP64-class tiles, the FP32-class product A_mk L~_kk^-T for FP32/FP16-class tiles (reading
+ * C12'), result rounded to storage(m,k); L_mk reaches its successors at comm(m,k) and is
+ * converted once per panel on the consuming GPU to the successor's operand format;
+ * DSYRK and FP64-class GEMMs on the handle's FP64 engine (default: CRT on INT8 tcgen05, see
+ * mp_config), FP32-class GEMMs as 3xFP16 (default) or 3xTF32 on tcgen05, FP16-class GEMMs as
+ * row-scaled FP16 x FP16 -> FP32 on tcgen05, accumulating into the FP32 tile.
  * kernel_prec / comm_prec: host maps (NT*NT, as produced by mp_precision_map
  * and consistent with the storage map A is bound with).  Blocking.
  * *info = 0 on success, else the 1-based global column of the first
@@ -212,7 +272,7 @@ mp_status mp_loglik(mp_handle* h, const mp_matrix* L, const double* d_z,
                     double* loglik, double* logdet, double* quad);
 
 /* Sample the Gaussian field with covariance L L^T: d_z = L d_e (device FP64 [n] each), with L the
- * factor left in A by mp_tile_potrf (read in storage precision).  With e ~ N(0, I) this gives the
+ * factor left in A by mp_tile_potrf (read in storage precision; everything on the device).  With e ~ N(0, I) this gives the
  * synthetic measurement vectors Z = L(theta) e of the Monte-Carlo studies.  One rank only. */
 mp_status mp_gp_sample(mp_handle* h, const mp_matrix* L, const double* d_e, double* d_z);
 
@@ -220,8 +280,8 @@ mp_status mp_gp_sample(mp_handle* h, const mp_matrix* L, const double* d_e, doub
  * (3), (4).  x, y, z are FP64 [n]; if `inputs_on_host` is nonzero they are host
  * pointers and are copied to the device inside the call (pinned memory makes
  * the copy asynchronous), else device pointers.  A must be bound to a
- * workspace sized for the worst case (mp_matrix_bytes with NULL); it is
- * re-bound to the evaluation's storage map.  `mode` picks the kernel map
+ * workspace (mp_matrix_bind or mp_matrix_attach); it is re-bound to the evaluation's storage map,
+ * and MP_ERR_NOMEM (report->workspace_bytes = the bytes needed) if that does not fit.  `mode` picks the kernel map
  * (`user_kernel_prec` is read only for MP_MAP_USER).  Out: report.
  * Returns MP_ERR_NOT_SPD (report->info set, loglik = -inf) for a non-SPD Sigma. */
 mp_status mp_eval(mp_handle* h, mp_matrix* A, const double* x, const double* y, const double* z,
@@ -251,7 +311,7 @@ int mp_matrix_owner(const mp_matrix* A, int m, int k);
 
 /* Per-kernel-class device time accounting (CUDA events recorded on the handle's stream around
  * every launch of the class; enable before the region to measure, read after it).
- * Classes: 0 FP64 trailing update (DMMA GEMM+SYRK), 1 FP32-class update, 2 FP16-class update,
+ * Classes: 0 FP64-class trailing update (GEMM + SYRK), 1 FP32-class update, 2 FP16-class update,
  * 3 POTRF (diagonal tiles), 4 TRSM, 5 conversion (K2), 6 generation (K1), 7 solve (K8). */
 #define MP_PROF_CLASSES 8
 typedef struct {
@@ -260,14 +320,17 @@ typedef struct {
     int64_t launches[MP_PROF_CLASSES];
 } mp_profile;
 mp_status mp_set_profiling(mp_handle* h, int enable);  /* enable also resets the counters */
+/* Profile only the classes whose bit is set in `mask` (bit c = class c; 0 = off); resets the counters.
+ * bench.py times the dominant class inside its timed region this way (one event pair per launch of
+ * that class only). */
+mp_status mp_set_profiling_mask(mp_handle* h, unsigned mask);
 mp_status mp_get_profile(mp_handle* h, mp_profile* out);  /* synchronises the stream */
 
-/* Engine configuration of a handle (read from MPGEO_* at mp_init): tcgen05 kernels for the FP32
- * and FP16 classes (1: FP32 class as 3xTF32; 2: FP32 class as row-scaled 3xFP16, the default) or DMMA
- * on rounded operands (0); panel lookahead (1/0); FP64-class
- * engine: 16 = CRT (16 moduli) and 8 = Ozaki split (8 int8 slices), both on tcgen05 kind::i8, 0 = DMMA
- * FP64; + 200 if the FP32 class runs as CRT-8 (8 moduli), + 100 if as the 4-slice split. */
-mp_status mp_handle_config(const mp_handle* h, int* tc, int* lookahead, int* ozaki);
+/* The engines mp_tile_potrf / mp_eval actually run for this matrix (they depend on nb as well as
+ * on the handle's mp_config: the tcgen05 kernels need nb % 256 == 0).  Out (any may be NULL):
+ * fp64 = mp_fp64_engine, fp32 = mp_fp32_engine, fp16 = 1 for tcgen05 / 0 for DMMA, lowp_trsm = 1
+ * if FP32/FP16-class TRSMs run as the CRT-8 product (reading C12'). */
+mp_status mp_matrix_engines(const mp_matrix* A, int* fp64, int* fp32, int* fp16, int* lowp_trsm);
 
 /* Total kernels launched on this handle since mp_init (for bench accounting). */
 int64_t mp_launch_count(const mp_handle* h);

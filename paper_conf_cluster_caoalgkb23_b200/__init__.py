@@ -6,8 +6,13 @@ precision maps (Alg. 2), the mixed-precision tile Cholesky (Alg. 1) and
 Eq. (1) — runs in the library.
 
     from paper_conf_cluster_caoalgkb23_b200 import Evaluator
-    ev = Evaluator(n, nb)                  # one handle + worst-case workspace
+    ev = Evaluator(n, nb)                  # one handle; the workspace grows to what each map needs
     rep = ev.eval(x, y, z, theta)          # numpy (host) or torch.cuda tensors
+
+Engines and schedule switches are an mp_config (Handle(config={...})): fp64_engine MP_F64_CRT16
+(default) / MP_F64_DMMA, fp32_engine MP_F32_3XFP16 (default) / MP_F32_3XTF32 / MP_F32_DMMA,
+fp16_tensor, lookahead, reserve_pairs, lowp_trsm_product, matern_table, f16x3_persistent,
+crt_phase_lock (include/mpgeo.h).
 """
 from __future__ import annotations
 
@@ -15,11 +20,13 @@ import ctypes as C
 
 import numpy as np
 
-from ._lib import (EvalReport, MpError, Profile, PROF_CLASSES, lib, MP_OK, MP_ERR_NOT_SPD, MP_FP64, MP_FP32, MP_FP16,  # noqa: F401
-                   MP_COMM_TTC, MP_COMM_AUTO, MP_MAP_ADAPTIVE, MP_MAP_FP64, MP_MAP_BAND, MP_MAP_EXTREME,
-                   MP_MAP_USER, MP_COV_MATERN, MP_COV_SQEXP)
+from ._lib import (Config, EvalReport, MpError, Profile, PROF_CLASSES, lib, MP_OK, MP_ERR_NOT_SPD,  # noqa: F401
+                   MP_ERR_NOMEM, MP_FP64, MP_FP32, MP_FP16, MP_COMM_TTC, MP_COMM_AUTO, MP_MAP_ADAPTIVE, MP_MAP_FP64,
+                   MP_MAP_BAND, MP_MAP_EXTREME, MP_MAP_USER, MP_COV_MATERN, MP_COV_SQEXP, MP_F64_CRT16, MP_F64_DMMA,
+                   MP_F32_3XFP16, MP_F32_3XTF32, MP_F32_DMMA)
 
-__all__ = ["Handle", "Matrix", "Evaluator", "precision_map", "exchange_plan", "exact_sum", "MpError", "EvalReport"]
+__all__ = ["Handle", "Matrix", "Evaluator", "precision_map", "exchange_plan", "exact_sum", "unique_id", "MpError",
+           "EvalReport", "default_config", "shared_unique_id"]
 
 _u8p = C.POINTER(C.c_uint8)
 _dp = C.POINTER(C.c_double)
@@ -46,23 +53,55 @@ def _ptr(t) -> int:
     return t.data_ptr()
 
 
+def unique_id() -> bytes:
+    """mp_get_unique_id: the 128-byte communicator id rank 0 creates and broadcasts."""
+    buf = (C.c_uint8 * 128)()
+    st = lib.mp_get_unique_id(C.cast(buf, _u8p))
+    if st != MP_OK:
+        raise MpError(st, "mp_get_unique_id failed")
+    return bytes(buf)
+
+
+def shared_unique_id(group=None) -> bytes:
+    """unique_id() on rank 0, broadcast to every rank of the torch.distributed group."""
+    import torch.distributed as dist
+
+    obj = [unique_id() if dist.get_rank(group) == 0 else None]
+    dist.broadcast_object_list(obj, src=0, group=group)
+    return obj[0]
+
+
+def default_config() -> dict:
+    """mp_config_default as a dict."""
+    c = Config()
+    lib.mp_config_default(C.byref(c))
+    return c.as_dict()
+
+
 class Handle:
-    """mp_init / mp_finalize.  One per process and GPU."""
+    """mp_init_config / mp_finalize.  One per process and GPU.  `config`: dict of mp_config fields
+    overriding the defaults; `uid`: the communicator id (unique_id()) shared by all ranks."""
 
     def __init__(self, device: int = 0, rank: int = 0, nranks: int = 1, P: int = 1, Q: int = 1,
-                 nccl_id: bytes | None = None, stream=None):
+                 uid: bytes | None = None, stream=None, config: dict | None = None):
         import torch
 
         torch.cuda.set_device(device)
         self.stream = stream if stream is not None else torch.cuda.current_stream(device)
         h = C.c_void_p()
-        uid = None
-        if nccl_id is not None:
-            uid = (C.c_uint8 * 128).from_buffer_copy(nccl_id)
-            uid = C.cast(uid, _u8p)
-        st = lib.mp_init(device, rank, nranks, P, Q, uid, C.c_void_p(self.stream.cuda_stream), C.byref(h))
+        cid = None
+        if uid is not None:
+            cid = C.cast((C.c_uint8 * 128).from_buffer_copy(uid), _u8p)
+        cfg = Config()
+        lib.mp_config_default(C.byref(cfg))
+        for k, v in (config or {}).items():
+            if not hasattr(cfg, k):
+                raise ValueError(f"unknown mp_config field {k}")
+            setattr(cfg, k, int(v))
+        st = lib.mp_init_config(device, rank, nranks, P, Q, cid, C.c_void_p(self.stream.cuda_stream), C.byref(cfg),
+                                C.byref(h))
         if st != MP_OK:
-            raise MpError(st, "mp_init failed")
+            raise MpError(st, "mp_init_config failed")
         self.h = h
         self.device = device
         self.rank, self.nranks, self.P, self.Q = rank, nranks, P, Q
@@ -71,8 +110,15 @@ class Handle:
         if st != MP_OK:
             raise MpError(st, lib.mp_last_error(self.h).decode())
 
-    def set_profiling(self, enable: bool):
-        self.check(lib.mp_set_profiling(self.h, int(enable)))
+    def set_profiling(self, enable: bool, classes=None):
+        """All classes, or only `classes` (names of PROF_CLASSES or indices)."""
+        if classes is None:
+            self.check(lib.mp_set_profiling(self.h, int(enable)))
+            return
+        mask = 0
+        for c in classes:
+            mask |= 1 << (PROF_CLASSES.index(c) if isinstance(c, str) else int(c))
+        self.check(lib.mp_set_profiling_mask(self.h, mask if enable else 0))
 
     def profile(self) -> Profile:
         p = Profile()
@@ -80,9 +126,9 @@ class Handle:
         return p
 
     def config(self) -> dict:
-        tc, la, oz = C.c_int(), C.c_int(), C.c_int()
-        self.check(lib.mp_handle_config(self.h, C.byref(tc), C.byref(la), C.byref(oz)))
-        return {"tc": tc.value, "lookahead": la.value, "ozaki": oz.value}
+        c = Config()
+        self.check(lib.mp_handle_get_config(self.h, C.byref(c)))
+        return c.as_dict()
 
     @property
     def launches(self) -> int:
@@ -101,24 +147,56 @@ class Handle:
 
 
 class Matrix:
-    """mp_matrix_*: geometry + a caller-owned (torch) workspace."""
+    """mp_matrix_*: geometry + a caller-owned (torch) workspace.
 
-    def __init__(self, handle: Handle, n: int, nb: int, storage_prec: np.ndarray | None = None, group=None):
-        import torch
+    attach=False: the workspace is sized for `storage_prec` (None = all FP64) and bound to it.
+    attach=True: a workspace for mp_eval only (mp_matrix_attach), sized for the smallest map and grown
+    by Evaluator when an evaluation's map needs more (no all-FP64 worst case)."""
 
+    def __init__(self, handle: Handle, n: int, nb: int, storage_prec: np.ndarray | None = None, group=None,
+                 attach: bool = False):
         self.handle = handle
         A = C.c_void_p()
         handle.check(lib.mp_matrix_create(handle.h, n, nb, C.byref(A)))
         self.A = A
         self.n, self.nb = n, nb
         self.nt = lib.mp_matrix_nt(A)
+        self.ws = None
         if handle.nranks > 1:
             self._connect(group)
+        if attach:
+            nt = self.nt
+            smallest = np.full((nt, nt), 255, np.uint8)  # FP64 diagonal, FP32 elsewhere
+            smallest[np.tril_indices(nt, -1)] = MP_FP32
+            np.fill_diagonal(smallest, MP_FP64)
+            self.attach(self.bytes_for(smallest))
+        else:
+            self._alloc(self.bytes_for(storage_prec))
+            self.bind(storage_prec)
+
+    def bytes_for(self, storage_prec: np.ndarray | None) -> int:
         nbytes = C.c_size_t()
-        handle.check(lib.mp_matrix_bytes(A, _u8(storage_prec), C.byref(nbytes)))
-        self.nbytes = nbytes.value
-        self.ws = torch.empty(self.nbytes, dtype=torch.uint8, device=f"cuda:{handle.device}")
-        self.bind(storage_prec)
+        self.handle.check(lib.mp_matrix_bytes(self.A, _u8(storage_prec), C.byref(nbytes)))
+        return nbytes.value
+
+    def _alloc(self, nbytes: int):
+        import torch
+
+        self.ws = None  # release the old workspace before the new one is allocated
+        torch.cuda.empty_cache()
+        self.nbytes = int(nbytes)
+        self.ws = torch.empty(self.nbytes, dtype=torch.uint8, device=f"cuda:{self.handle.device}")
+
+    def attach(self, nbytes: int):
+        """(Re)allocate a workspace of nbytes and attach it for mp_eval (mp_matrix_attach)."""
+        self._alloc(nbytes)
+        self.handle.check(lib.mp_matrix_attach(self.A, C.c_void_p(self.ws.data_ptr()), self.nbytes))
+
+    def engines(self) -> dict:
+        """mp_matrix_engines: the engines this matrix runs with (handle config + nb)."""
+        f64, f32, f16, tr = C.c_int(), C.c_int(), C.c_int(), C.c_int()
+        self.handle.check(lib.mp_matrix_engines(self.A, C.byref(f64), C.byref(f32), C.byref(f16), C.byref(tr)))
+        return {"fp64": f64.value, "fp32": f32.value, "fp16_tensor": f16.value, "lowp_trsm_product": tr.value}
 
     def _connect(self, group):
         """Exchange the CUDA IPC handles of every rank's exchange area (torch.distributed all-gather)."""
@@ -243,12 +321,14 @@ def exact_sum(v: np.ndarray) -> float:
 
 
 class Evaluator:
-    """One log-likelihood evaluation per call (mp_eval) on a worst-case (all-FP64) workspace."""
+    """One log-likelihood evaluation per call (mp_eval).  One rank: the workspace is sized by the
+    evaluation's storage map and grows when a later map needs more (mp_matrix_attach, MP_ERR_NOMEM);
+    several ranks: each binds its all-FP64 worst case once (the ranks must not disagree mid-call)."""
 
     def __init__(self, n: int, nb: int, device: int = 0, handle: Handle | None = None, group=None,
-                 covariance: int = MP_COV_MATERN):
-        self.handle = handle or Handle(device)
-        self.M = Matrix(self.handle, n, nb, None, group=group)
+                 covariance: int = MP_COV_MATERN, config: dict | None = None):
+        self.handle = handle or Handle(device, config=config)
+        self.M = Matrix(self.handle, n, nb, None, group=group, attach=self.handle.nranks == 1)
         if covariance != MP_COV_MATERN:
             self.M.set_covariance(covariance)
         self.n, self.nb, self.nt = n, nb, self.M.nt
@@ -261,11 +341,15 @@ class Evaluator:
                 assert a.dtype == np.float64 and a.flags.c_contiguous and a.shape == (self.n,)
         th = np.ascontiguousarray(theta, dtype=np.float64)
         e = None if eps is None else np.ascontiguousarray(eps, dtype=np.float64)
-        rep = EvalReport()
-        st = lib.mp_eval(self.handle.h, self.M.A, C.c_void_p(_ptr(x)), C.c_void_p(_ptr(y)), C.c_void_p(_ptr(z)),
-                         int(on_host), _d(th), float(u_req), _d(e), policy, mode,
-                         _u8(None if kernel_prec is None else np.ascontiguousarray(kernel_prec, np.uint8)),
-                         C.byref(rep))
+        km = None if kernel_prec is None else np.ascontiguousarray(kernel_prec, np.uint8)
+        for _ in range(2):
+            rep = EvalReport()
+            st = lib.mp_eval(self.handle.h, self.M.A, C.c_void_p(_ptr(x)), C.c_void_p(_ptr(y)), C.c_void_p(_ptr(z)),
+                             int(on_host), _d(th), float(u_req), _d(e), policy, mode, _u8(km), C.byref(rep))
+            if st == MP_ERR_NOMEM and self.handle.nranks == 1 and rep.workspace_bytes > self.M.nbytes:
+                self.M.attach(rep.workspace_bytes)  # this map needs a larger workspace: grow, repeat
+                continue
+            break
         if st not in (MP_OK, MP_ERR_NOT_SPD):
             self.handle.check(st)
         return rep

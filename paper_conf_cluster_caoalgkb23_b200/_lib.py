@@ -10,7 +10,7 @@ import ctypes as C
 import os
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.environ.get("MPGEO_LIB") or os.path.join(_HERE, "libmpgeo.so")  # MPGEO_LIB: experiment builds
+LIB_PATH = os.path.join(_HERE, "libmpgeo.so")
 
 MP_OK, MP_ERR_ARG, MP_ERR_NOT_SPD, MP_ERR_CUDA, MP_ERR_COMM, MP_ERR_NOMEM, MP_ERR_UNSUPPORTED, MP_ERR_STATE = range(8)
 STATUS_NAMES = ["MP_OK", "MP_ERR_ARG", "MP_ERR_NOT_SPD", "MP_ERR_CUDA", "MP_ERR_COMM", "MP_ERR_NOMEM",
@@ -19,6 +19,8 @@ MP_FP64, MP_FP32, MP_FP16 = 0, 1, 2
 MP_COMM_TTC, MP_COMM_AUTO = 0, 1
 MP_MAP_ADAPTIVE, MP_MAP_FP64, MP_MAP_BAND, MP_MAP_EXTREME, MP_MAP_USER = range(5)
 MP_COV_MATERN, MP_COV_SQEXP = 0, 1
+MP_F64_CRT16, MP_F64_DMMA = 0, 1
+MP_F32_3XFP16, MP_F32_3XTF32, MP_F32_DMMA = 0, 1, 2
 
 
 class EvalReport(C.Structure):
@@ -29,7 +31,18 @@ class EvalReport(C.Structure):
         ("t_solve_ms", C.c_double), ("t_total_ms", C.c_double),
         ("flops_potrf", C.c_double), ("flops_update", C.c_double * 3),
         ("tiles", C.c_int64 * 3), ("stc_tiles", C.c_int64), ("gpu_launches", C.c_int64),
+        ("workspace_bytes", C.c_uint64),
     ]
+
+
+class Config(C.Structure):
+    """mp_config (include/mpgeo.h): engines and schedule switches of a handle."""
+    _fields_ = [("fp64_engine", C.c_int), ("fp32_engine", C.c_int), ("fp16_tensor", C.c_int), ("lookahead", C.c_int),
+                ("reserve_pairs", C.c_int), ("lowp_trsm_product", C.c_int), ("matern_table", C.c_int),
+                ("f16x3_persistent", C.c_int), ("crt_phase_lock", C.c_int)]
+
+    def as_dict(self):
+        return {name: getattr(self, name) for name, _ in self._fields_}
 
 
 PROF_CLASSES = ["upd_fp64", "upd_fp32", "upd_fp16", "potrf", "trsm", "convert", "generate", "solve"]
@@ -61,6 +74,12 @@ def _load() -> C.CDLL:
     vp, i32, i64, dbl, u8p, dp = C.c_void_p, C.c_int, C.c_int64, C.c_double, C.POINTER(C.c_uint8), C.POINTER(C.c_double)
     sig = {
         "mp_init": (i32, [i32, i32, i32, i32, i32, u8p, vp, C.POINTER(vp)]),
+        "mp_init_config": (i32, [i32, i32, i32, i32, i32, u8p, vp, C.POINTER(Config), C.POINTER(vp)]),
+        "mp_config_default": (None, [C.POINTER(Config)]),
+        "mp_handle_get_config": (i32, [vp, C.POINTER(Config)]),
+        "mp_get_unique_id": (i32, [u8p]),
+        "mp_matrix_attach": (i32, [vp, vp, C.c_size_t]),
+        "mp_matrix_engines": (i32, [vp, C.POINTER(i32), C.POINTER(i32), C.POINTER(i32), C.POINTER(i32)]),
         "mp_finalize": (i32, [vp]),
         "mp_last_error": (C.c_char_p, [vp]),
         "mp_matrix_create": (i32, [vp, i64, i32, C.POINTER(vp)]),
@@ -83,19 +102,18 @@ def _load() -> C.CDLL:
         "mp_matrix_nt": (i32, [vp]),
         "mp_matrix_owner": (i32, [vp, i32, i32]),
         "mp_launch_count": (i64, [vp]),
-        "mp_handle_config": (i32, [vp, C.POINTER(i32), C.POINTER(i32), C.POINTER(i32)]),
         "mp_set_profiling": (i32, [vp, i32]),
+        "mp_set_profiling_mask": (i32, [vp, C.c_uint]),
         "mp_get_profile": (i32, [vp, C.POINTER(Profile)]),
         "mp_version": (C.c_char_p, []),
         "mpgeo_exact_sum": (dbl, [dp, i64]),
         "mp_test_bessel_k": (i32, [dbl, vp, vp, i32]),
         "mp_test_dgemm": (i32, [vp, vp, vp, i32, i32, i32, i32, i32, i32, i32, dbl, dbl, i32, i32]),
         "mp_test_tc_gemm": (i32, [i32, vp, vp, vp, i32, i32, i32, i32]),
+        "mp_test_tc_gemm_split": (i32, [i32, vp, vp, i32, i32, i32, i32, i32]),
         "mp_tc_available": (i32, []),
-        "mp_test_ozaki_gemm": (i32, [vp, vp, i32, i32, i32, i32, i32, i32]),
-        "mp_test_crt_gemm": (i32, [vp, vp, i32, i32, i32, i32, i32, i32]),
-        "mp_test_crt_gemm_ex": (i32, [vp, vp, i32, i32, i32, i32, i32, i32, i32, i32]),
-        "mp_bench_fp64_engine": (i32, [i32, i32, i32, i32, i32, i32, C.POINTER(C.c_float)]),
+        "mp_test_crt_gemm": (i32, [vp, vp, i32, i32, i32, i32, i32, i32, i32]),
+        "mp_bench_fp64_engine": (i32, [i32, i32, i32, i32, i32, C.POINTER(C.c_float)]),
         "mp_test_crt_constants": (i32, [i32, i32, C.POINTER(i32), C.POINTER(i32), dp, dp, dp]),
     }
     for name, (res, args) in sig.items():

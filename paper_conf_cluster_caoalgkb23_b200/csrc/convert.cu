@@ -3,12 +3,13 @@
 // After TRSM(m, k) the tile L_mk exists once, in FP64, in the GPU's panel buffer.  panel_out
 //   * writes it back to the tile pool in its storage precision (the factor the solve reads),
 //   * rounds the panel copy to the communication precision comm(m, k) — what the successors
-//     receive (STC when comm < storage, TTC otherwise; Algorithm 2),
-//   * and derives, once per panel per GPU, the operand formats its consuming GEMMs need:
-//     FP16 (FP16-class successors) and the TF32 hi/lo pair (FP32-class successors, 3xTF32).
-// Consumers therefore convert on the GPU they run on (target-side conversion), but at
-// most once per tile instead of once per GEMM.  All kernels are elementwise, 16-byte
-// vectorised and HBM-bound.
+//     receive (STC when comm < storage, TTC otherwise; Algorithm 2).
+// Once per panel and GPU, after the previous trailing update has released the (single-buffered)
+// operand caches, the format kernels derive from the panel copy the operands its consuming GEMMs
+// need: the row-scaled FP16 hi/lo split (FP16 class: hi; FP32 class as 3xFP16: hi + lo), the TF32
+// hi/lo pair (FP32 class as 3xTF32) and, in crt.cu, the CRT residue planes (FP64 class).
+// Consumers therefore convert on the GPU they run on (target-side conversion), but at most
+// once per tile instead of once per GEMM.  All kernels are elementwise and HBM-bound.
 #include "common.cuh"
 #include "kernels.h"
 
@@ -47,15 +48,20 @@ __global__ void __launch_bounds__(CV_T) panel_out_kernel(const PanelTile* tiles,
         } else {
             *(float2*)((float*)t.store + i) = make_float2(__double2float_rn(v.x), __double2float_rn(v.y));
         }
-        const double w0 = round_to(v.x, t.comm_prec), w1 = round_to(v.y, t.comm_prec);
-        if (t.comm_prec != P64) *(double2*)(t.p64 + i) = make_double2(w0, w1);
-        if (t.p16) *(__half2*)(t.p16 + i) = __halves2half2(__double2half(w0), __double2half(w1));
-        if (t.hi) {
-            const float f0 = __double2float_rn(w0), f1 = __double2float_rn(w1);
-            const float h0 = tf32_rna(f0), h1 = tf32_rna(f1);
-            *(float2*)(t.hi + i) = make_float2(h0, h1);
-            *(float2*)(t.lo + i) = make_float2(tf32_rna(f0 - h0), tf32_rna(f1 - h1));
-        }
+        if (t.comm_prec != P64) *(double2*)(t.p64 + i) = make_double2(round_to(v.x, t.comm_prec), round_to(v.y, t.comm_prec));
+    }
+}
+
+// 3xTF32 operands of the FP32 class (reading C13): hi = rna_tf32(fp32(x)), lo = rna_tf32(fp32(x) - hi)
+__global__ void __launch_bounds__(CV_T) tf32_split_kernel(const Tf32Item* items, int64_t elems) {
+    const Tf32Item t = items[blockIdx.y];
+    const int64_t stride = (int64_t)gridDim.x * CV_T * 2;
+    for (int64_t i = ((int64_t)blockIdx.x * CV_T + threadIdx.x) * 2; i < elems; i += stride) {
+        const double2 v = *(const double2*)(t.src + i);
+        const float f0 = __double2float_rn(v.x), f1 = __double2float_rn(v.y);
+        const float h0 = tf32_rna(f0), h1 = tf32_rna(f1);
+        *(float2*)(t.hi + i) = make_float2(h0, h1);
+        *(float2*)(t.lo + i) = make_float2(tf32_rna(f0 - h0), tf32_rna(f1 - h1));
     }
 }
 
@@ -87,10 +93,13 @@ __global__ void __launch_bounds__(256) transpose_kernel(const double* __restrict
     for (int r = ty; r < 32; r += 8) dst[(size_t)(bx + r) * nb + by + tx] = t[tx][r];
 }
 
-// 3xFP16 operands of the FP32 class (reading C13c): row i of the FP64 panel tile, rounded to FP32
+// Row-scaled FP16 operands (reading C13c): row i of the FP64 panel tile, rounded to FP32
 // (the FP32-class operand), is scaled by 2^s_i with max_j |x_ij| 2^s_i < 2^15 and split into FP16
 // hi = rn(x 2^s), lo = rn(x 2^s - hi) (x 2^s - hi is exact in FP32), i.e. the 11 + 11-bit split of
-// 3xTF32, now within FP16 range; e_i = -s_i is stored for the GEMM epilogue.  One warp per row.
+// 3xTF32, now within FP16 range; e_i = -s_i is stored for the GEMM epilogue.  hi + lo are the
+// 3xFP16 FP32-class operands; hi alone is the FP16-class operand (FP16 = 11 significant bits, with
+// the power-of-two row scale keeping small entries out of the FP16 subnormal range).  lo may be
+// null (FP16 class only).  One warp per row.
 __global__ void __launch_bounds__(256) split16_kernel(const Split16Item* items, int nb) {
     const Split16Item it = items[blockIdx.y];
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
@@ -110,13 +119,13 @@ __global__ void __launch_bounds__(256) split16_kernel(const Split16Item* items, 
     if (lane == 0) it.exps[row] = -sc;
     const float f = ldexpf(1.f, sc);
     __half* hi = it.hi + (size_t)row * nb;
-    __half* lo = it.lo + (size_t)row * nb;
+    __half* lo = it.lo ? it.lo + (size_t)row * nb : nullptr;
     for (int j = lane * 2; j < nb; j += 64) {
         const double2 v = *(const double2*)(x + j);
         const float a0 = __double2float_rn(v.x) * f, a1 = __double2float_rn(v.y) * f;
         const __half h0 = __float2half_rn(a0), h1 = __float2half_rn(a1);
         *(__half2*)(hi + j) = __halves2half2(h0, h1);
-        *(__half2*)(lo + j) = __halves2half2(__float2half_rn(a0 - __half2float(h0)), __float2half_rn(a1 - __half2float(h1)));
+        if (lo) *(__half2*)(lo + j) = __halves2half2(__float2half_rn(a0 - __half2float(h0)), __float2half_rn(a1 - __half2float(h1)));
     }
 }
 
@@ -158,6 +167,13 @@ cudaError_t panel_out_launch(const PanelTile* t, int ntiles, int64_t elems, cuda
     if (ntiles <= 0) return cudaSuccess;
     dim3 grid(chunks_for(elems, ntiles), ntiles);
     panel_out_kernel<<<grid, CV_T, 0, s>>>(t, elems);
+    return cudaGetLastError();
+}
+
+cudaError_t tf32_split_launch(const Tf32Item* t, int ntiles, int64_t elems, cudaStream_t s) {
+    if (ntiles <= 0) return cudaSuccess;
+    dim3 grid(chunks_for(elems, ntiles), ntiles);
+    tf32_split_kernel<<<grid, CV_T, 0, s>>>(t, elems);
     return cudaGetLastError();
 }
 

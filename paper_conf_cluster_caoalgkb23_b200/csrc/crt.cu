@@ -16,7 +16,7 @@
 // (|X| ~ 2^{2b}).  Then C_ij -= X 2^{e_i - b} 2^{f_j - b} (exact scalings, one FP64 rounding).
 // Accuracy: the operand rounding is 2^-(b+1) of the row max (b = 56 for N = 16, K = 2048), i.e.
 // the product error is <= K 2^-(b+1) (max_k|a_ik| max_k|b_jk|) — FP64-GEMM level (K 2^-53 sum|a||b|).
-// N = 16 GEMMs per tile product instead of the 36 of the 8-slice splitting engine (ozaki.cu).
+// N = 16 GEMMs per tile product (an 8-slice Ozaki split needs 36).
 //
 // Kernel: persistent CTA pairs (cluster of 2 on a TPC, tcgen05.mma.cta_group::2, M = 256, N = 256,
 // K = 32 per MMA), 128-byte-swizzled K-major TMA boxes of 128 x 128 int8 per CTA and operand, six
@@ -195,14 +195,14 @@ struct __align__(64) CrtParams {
     CUtensorMap a, b;  // 3D [N][rows][nb] int8, box {128, 128, 1}
     CUtensorMap cmap;  // C rows [crows][nb] from cbase, box {8, 32}: FP64 (64-byte swizzle) or FP32 (no swizzle)
     const void* cbase;
-    const OzJob* jobs;
+    const CrtJob* jobs;
     const int* exps;
     uint8_t* scratch;
     int* slot_flags;
     int nslots, nb, tiles_n, tiles_per_job, lower, total;
     int store;  // 1: C = P_m P_n^T (TMA store), 0: C -= P_m P_n^T (TMA reduce-add)
     int* tile_counter;  // [0]: dynamic tile scheduler, [1]: current modulus-pair phase (zero before the launch)
-    int phase_lock;     // 1: start each tile at the current modulus-pair phase (MPGEO_CRT_PHASE, default 1)
+    int phase_lock;     // 1: start each tile at the current modulus-pair phase (CrtArgs::phase_lock)
     CrtConst c;
 };
 
@@ -368,9 +368,8 @@ __device__ __forceinline__ int mod_canon(int a, int p, int mq) {
 
 }  // namespace
 
-// NMOD moduli (16: FP64 class, b = 56 at K = 2048; 8: FP32 class, b = 25), F32: C is FP32 (the
-// FP32-class tiles, reduce-added in FP32 by the TMA unit) instead of FP64
-template <int NMOD, bool F32>
+// NMOD moduli (16: FP64 class, b = 56 at K = 2048; 8: the FP32-class TRSM product, b = 25); C is FP64
+template <int NMOD>
 __global__ void __launch_bounds__(THREADS, 1) crt_gemm_kernel(const __grid_constant__ CrtParams p) {
     extern __shared__ uint8_t smem_raw[];
     uint8_t* smem = (uint8_t*)(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
@@ -460,7 +459,7 @@ __global__ void __launch_bounds__(THREADS, 1) crt_gemm_kernel(const __grid_const
             tile &= (1 << 28) - 1;
             int job, bi, bj;
             tile_coords(p, tile, job, bi, bj);
-            const OzJob jb = p.jobs[job];
+            const CrtJob jb = p.jobs[job];
             const int rowA = jb.m * p.nb + bi * 256 + (int)crank * BM;
             const int rowB = jb.n * p.nb + bj * BN + (int)crank * (BN / 2);
             for (int tt = 0; tt < N; ++tt) {
@@ -580,20 +579,10 @@ __global__ void __launch_bounds__(THREADS, 1) crt_gemm_kernel(const __grid_const
                 const double X = fma(-qm, p.c.Mh, sh[v]) + fma(-qm, p.c.Ml, sl[v]);
                 o[v] = (p.store ? X : -X) * pv_rs * exp2i(__ldg(pv_ecol + col0 + v) - p.c.bits);
             }
-            if constexpr (F32) {  // 32 x 8 FP32 box, rows of 32 bytes (no swizzle)
-                const uint32_t a = sb + (uint32_t)lane * 32u;
-                asm volatile("st.shared.v4.f32 [%0], {%1, %2, %3, %4};" ::"r"(a), "f"((float)o[0]), "f"((float)o[1]),
-                             "f"((float)o[2]), "f"((float)o[3])
-                             : "memory");
-                asm volatile("st.shared.v4.f32 [%0], {%1, %2, %3, %4};" ::"r"(a + 16u), "f"((float)o[4]), "f"((float)o[5]),
-                             "f"((float)o[6]), "f"((float)o[7])
-                             : "memory");
-            } else {
 #pragma unroll
-                for (int v = 0; v < 8; v += 2) {
-                    const uint32_t a = sb + (uint32_t)lane * 64u + ((uint32_t)((v >> 1) ^ ((lane >> 1) & 3)) << 4);
-                    asm volatile("st.shared.v2.f64 [%0], {%1, %2};" ::"r"(a), "d"(o[v]), "d"(o[v + 1]) : "memory");
-                }
+            for (int v = 0; v < 8; v += 2) {
+                const uint32_t a = sb + (uint32_t)lane * 64u + ((uint32_t)((v >> 1) ^ ((lane >> 1) & 3)) << 4);
+                asm volatile("st.shared.v2.f64 [%0], {%1, %2};" ::"r"(a), "d"(o[v]), "d"(o[v + 1]) : "memory");
             }
             asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
             __syncwarp();
@@ -720,13 +709,13 @@ __global__ void __launch_bounds__(THREADS, 1) crt_gemm_kernel(const __grid_const
                 }
             }
             // this tile becomes the pending one
-            const OzJob jb = p.jobs[job];
+            const CrtJob jb = p.jobs[job];
             const int grow = bi * 256 + (int)crank * BM + r;  // row inside the tile
             pv = true;
             pv_half = it_tile & 1;
             pv_rs = ldexp(1.0, p.exps[jb.m * p.nb + grow] - p.c.bits);
             pv_ecol = p.exps + (size_t)jb.n * p.nb + bj * BN + h * 128;
-            pv_crow0 = (int)(((const char*)jb.C - (const char*)p.cbase) / ((size_t)p.nb * (F32 ? 4 : 8))) + bi * 256 +
+            pv_crow0 = (int)(((const char*)jb.C - (const char*)p.cbase) / ((size_t)p.nb * 8)) + bi * 256 +
                        (int)crank * BM + q * 32;
             pv_ccol0 = bj * BN + h * 128;
         }
@@ -772,15 +761,6 @@ static PFN_cuTensorMapEncodeTiled_v12000 crt_encode() {
     return fn;
 }
 
-static CUtensorMapL2promotion crt_promo() {  // MPGEO_CRT_PROMO: 0 none, 1 64B, 2 128B, 3 256B (default)
-    static const int v = [] {
-        const char* e = getenv("MPGEO_CRT_PROMO");
-        return e ? atoi(e) : 3;
-    }();
-    return v == 0 ? CU_TENSOR_MAP_L2_PROMOTION_NONE : v == 1 ? CU_TENSOR_MAP_L2_PROMOTION_L2_64B
-           : v == 2 ? CU_TENSOR_MAP_L2_PROMOTION_L2_128B : CU_TENSOR_MAP_L2_PROMOTION_L2_256B;
-}
-
 static bool crt_map(CUtensorMap* m, const int8_t* base, uint64_t planes, uint64_t rows, uint64_t cols,
                     uint64_t plane_stride, uint32_t box_rows) {
     auto fn = crt_encode();
@@ -790,7 +770,7 @@ static bool crt_map(CUtensorMap* m, const int8_t* base, uint64_t planes, uint64_
     cuuint32_t box[3] = {(cuuint32_t)BK, box_rows, 1};
     cuuint32_t es[3] = {1, 1, 1};
     return fn(m, CU_TENSOR_MAP_DATA_TYPE_UINT8, 3, const_cast<int8_t*>(base), dims, strides, box, es,
-              CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B, crt_promo(),
+              CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
               CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
 }
 
@@ -822,13 +802,13 @@ bool crt_available() { return crt_encode() != nullptr; }
 
 cudaError_t crt_gemm_launch(const CrtArgs& a, int njobs, cudaStream_t s) {
     if (njobs <= 0) return cudaSuccess;
-    // instantiations: 16 moduli with an FP64 C (FP64 class); 8 moduli (FP32 class) with an FP32 C
-    // (trailing update) or an FP64 C (the FP32-class TRSM product into the FP64 panel buffer)
+    // instantiations: 16 moduli (FP64 class: trailing update, DSYRK) and 8 moduli (the FP32-class
+    // TRSM product A_mk W^T, reading C12'), both with an FP64 C
     if (a.nb % 256 || a.nb > 8192 || !a.scratch || !a.slot_flags) return cudaErrorInvalidValue;
-    if (!((a.c.nmod == 16 && !a.c_f32) || a.c.nmod == 8)) return cudaErrorInvalidValue;
-    const int ki = a.c.nmod == 16 ? 0 : a.c_f32 ? 1 : 2;
-    auto kern = ki == 0 ? crt_gemm_kernel<16, false> : ki == 1 ? crt_gemm_kernel<8, true> : crt_gemm_kernel<8, false>;
-    static bool attr[3] = {false, false, false};
+    if (a.c.nmod != 16 && a.c.nmod != 8) return cudaErrorInvalidValue;
+    const int ki = a.c.nmod == 16 ? 0 : 1;
+    auto kern = ki == 0 ? crt_gemm_kernel<16> : crt_gemm_kernel<8>;
+    static bool attr[2] = {false, false};
     if (!attr[ki]) {
         cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, SMEM);
         if (e != cudaSuccess) return e;
@@ -839,7 +819,7 @@ cudaError_t crt_gemm_launch(const CrtArgs& a, int njobs, cudaStream_t s) {
     const uint64_t rows = (uint64_t)a.nt * a.nb;
     if (!crt_map(&p.a, a.planes, (uint64_t)a.c.nmod, rows, a.nb, a.plane_stride, BM) ||
         !crt_map(&p.b, a.planes, (uint64_t)a.c.nmod, rows, a.nb, a.plane_stride, BN / 2) || !a.cbase ||
-        !crt_cmap(&p.cmap, a.cbase, a.crows, a.nb, a.c_f32 != 0))
+        !crt_cmap(&p.cmap, a.cbase, a.crows, a.nb, false))
         return cudaErrorInvalidValue;
     p.cbase = a.cbase;
     p.jobs = a.jobs;
@@ -852,22 +832,14 @@ cudaError_t crt_gemm_launch(const CrtArgs& a, int njobs, cudaStream_t s) {
     p.lower = a.lower;
     p.store = a.store;
     p.tile_counter = a.counter;
-    static const int phase_env = [] {
-        const char* e = getenv("MPGEO_CRT_PHASE");
-        return e ? atoi(e) : 1;
-    }();
-    p.phase_lock = phase_env;
+    p.phase_lock = a.phase_lock;
     if (!a.counter) return cudaErrorInvalidValue;
     p.tiles_per_job = a.lower ? p.tiles_n * (p.tiles_n + 1) / 2 : p.tiles_n * p.tiles_n;
     p.c = a.c;
     const long long total = (long long)njobs * p.tiles_per_job;
     if (total >= (1LL << 28)) return cudaErrorInvalidConfiguration;  // tile index | phase << 28 in the ring
     p.total = (int)total;
-    static const int env_pairs = [] {  // MPGEO_CRT_PAIRS overrides the persistent grid size (CTA pairs)
-        const char* e = getenv("MPGEO_CRT_PAIRS");
-        return e && atoi(e) > 0 ? atoi(e) : 0;
-    }();
-    const int max_pairs = env_pairs ? env_pairs : (a.max_pairs > 0 ? std::min(a.max_pairs, sm_count() / 2) : sm_count() / 2);
+    const int max_pairs = a.max_pairs > 0 ? std::min(a.max_pairs, sm_count() / 2) : sm_count() / 2;
     const int pairs = (int)std::min<long long>(total, max_pairs);
     cudaLaunchConfig_t cfg = {};
     cfg.gridDim = dim3((unsigned)(2 * pairs));

@@ -5,7 +5,6 @@
 #include <cuda_runtime.h>
 #include <stdint.h>
 
-#include "ozaki.h"  // OzJob (m, n, C): the same job records as the splitting engine
 
 namespace mpgeo {
 
@@ -29,6 +28,10 @@ struct CrtConst {
 // 2b + log2(K) + 1 < log2(M), so |sum_k x'_ik y'_jk| < M/2 and the CRT result is unique).
 bool crt_constants(int nmod, int K, CrtConst* c);
 
+struct CrtJob {
+    int m, n;   // panel rows of the operands (residue-cache rows m*nb.., n*nb..)
+    void* C;    // nb x nb output tile (FP64)
+};
 struct CrtSplitItem {
     const double* src;     // FP64 nb x nb tile (panel slot)
     int8_t* dst;           // residue planes: plane i at dst + i * plane_stride, row-major nb x nb
@@ -36,7 +39,7 @@ struct CrtSplitItem {
     int64_t plane_stride;  // bytes between planes
 };
 struct CrtArgs {
-    const OzJob* jobs;
+    const CrtJob* jobs;
     const int8_t* planes;  // residue cache: nmod planes of [nt*nb][nb] int8
     const int* exps;       // [nt*nb] row exponents
     int64_t plane_stride;  // = nt*nb*nb
@@ -47,9 +50,9 @@ struct CrtArgs {
     const void* cbase;     // C tiles lie inside [cbase, cbase + crows * nb) at whole-row offsets
     uint64_t crows;        //   (a view of the tile pool in C's type; C is updated by TMA reduce-add)
     int max_pairs;         // persistent grid in CTA pairs (0: one pair per 2 SMs)
-    int c_f32 = 0;         // 0: FP64 C (nmod = 16 or 8); 1: FP32 C (nmod = 8, FP32-class update)
     int store = 0;         // 1: C = P_m P_n^T (overwrite), 0: C -= P_m P_n^T
     int* counter = nullptr;  // 2 device ints of this launch, zero at launch: tile counter, modulus phase
+    int phase_lock = 1;    // 1: each tile starts at the modulus pair the other CTAs are on
 };
 // one CTA's 128 x 256 combined residues (N/2 x 2 bytes each) for two tiles (the epilogue reconstructs
 // tile T-1 while it reduces tile T)

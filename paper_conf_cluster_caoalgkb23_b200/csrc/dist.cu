@@ -6,9 +6,11 @@
 // storage or comm precision, never wider) and PUBLISHES a stamp (k + 1) with a system-scope
 // release store.  Each consumer runs one fused kernel that waits for the stamp with a
 // system-scope acquire load, reads the payload straight from the producer's memory (NVLink
-// peer load; across processes on one device it is the same-device IPC mapping) and converts it
-// on the fly into its own FP64 panel slot and, if its successors need them, the FP16 and TF32
-// hi/lo operand caches — the transfer and the target-side conversion (TTC) are one kernel.
+// peer load; across processes on one device it is the same-device IPC mapping) and up-converts it
+// on the fly into its own FP64 panel slot — the transfer and the target-side conversion (TTC,
+// P:156) are one kernel; the consumer's operand formats are derived from that slot once per panel
+// (engine.cu, step 5e).  Both kernels move 32 bytes of FP64 (4 elements) per thread and iteration
+// and size their grids to a few waves of the SMs.
 // A consumer stamps `done` when it has pulled everything of a panel; a producer waits for every
 // peer's `done` of panel k-2 before reusing that send slot (two slot sets, panel parity).
 #include "common.cuh"
@@ -23,12 +25,6 @@ __device__ __forceinline__ uint64_t ld_acquire_sys(const volatile uint64_t* p) {
 }
 __device__ __forceinline__ void st_release_sys(volatile uint64_t* p, uint64_t v) {
     asm volatile("st.release.sys.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
-}
-
-__device__ __forceinline__ float tf32_rna_d(float x) {
-    uint32_t r;
-    asm("cvt.rna.tf32.f32 %0, %1;" : "=r"(r) : "f"(x));
-    return __uint_as_float(r);
 }
 
 // Wait until every flag[i] >= target[i] (one thread; the list is short).
@@ -46,39 +42,51 @@ __global__ void set_flag_kernel(uint64_t* flag, uint64_t v) {
     st_release_sys(flag, v);
 }
 
-// Pack FP64 sources (already rounded to their communication precision) into payloads.
-__global__ void pack_kernel(const PackItem* items, int64_t elems) {
+// Pack FP64 sources (already rounded to their communication precision) into payloads (elems % 4 == 0).
+__global__ void __launch_bounds__(256) pack_kernel(const PackItem* items, int64_t elems) {
     const PackItem it = items[blockIdx.y];
-    const int64_t stride = (int64_t)gridDim.x * blockDim.x;
-    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < elems; i += stride) {
-        const double v = it.src[i];
-        if (it.prec == P64) ((double*)it.dst)[i] = v;
-        else if (it.prec == P32) ((float*)it.dst)[i] = __double2float_rn(v);
-        else ((__half*)it.dst)[i] = __double2half(v);
+    const int64_t stride = (int64_t)gridDim.x * blockDim.x * 4;
+    for (int64_t i = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) * 4; i < elems; i += stride) {
+        const double2 a = *(const double2*)(it.src + i), b = *(const double2*)(it.src + i + 2);
+        if (it.prec == P64) {
+            *(double2*)((double*)it.dst + i) = a;
+            *(double2*)((double*)it.dst + i + 2) = b;
+        } else if (it.prec == P32) {
+            *(float4*)((float*)it.dst + i) =
+                make_float4(__double2float_rn(a.x), __double2float_rn(a.y), __double2float_rn(b.x), __double2float_rn(b.y));
+        } else {
+            __half2 h[2] = {__halves2half2(__double2half(a.x), __double2half(a.y)),
+                            __halves2half2(__double2half(b.x), __double2half(b.y))};
+            *(uint2*)((__half*)it.dst + i) = *(const uint2*)h;
+        }
     }
 }
 
-// Fused pull + convert: peer payload (comm precision) -> local FP64 panel slot (+ caches).
-__global__ void pull_kernel(const PullItem* items, int64_t elems) {
+// Fused pull + up-convert: peer payload (comm precision) -> local FP64 panel slot (elems % 4 == 0).
+__global__ void __launch_bounds__(256) pull_kernel(const PullItem* items, int64_t elems) {
     const PullItem it = items[blockIdx.y];
     if (threadIdx.x == 0) {  // acquire the producer's stamp (already reached: wait_flags ran first)
         while (ld_acquire_sys(it.flag) < it.target) __nanosleep(64);
     }
     __syncthreads();
-    const int64_t stride = (int64_t)gridDim.x * blockDim.x;
-    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < elems; i += stride) {
-        double v;
-        if (it.prec == P64) v = ((const double*)it.src)[i];
-        else if (it.prec == P32) v = (double)((const float*)it.src)[i];
-        else v = (double)__half2float(((const __half*)it.src)[i]);
-        it.p64[i] = v;
-        if (it.p16) it.p16[i] = __double2half(v);
-        if (it.hi) {
-            const float f = __double2float_rn(v);
-            const float h = tf32_rna_d(f);
-            it.hi[i] = h;
-            it.lo[i] = tf32_rna_d(f - h);
+    const int64_t stride = (int64_t)gridDim.x * blockDim.x * 4;
+    for (int64_t i = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) * 4; i < elems; i += stride) {
+        double2 a, b;
+        if (it.prec == P64) {
+            a = *(const double2*)((const double*)it.src + i);
+            b = *(const double2*)((const double*)it.src + i + 2);
+        } else if (it.prec == P32) {
+            const float4 f = *(const float4*)((const float*)it.src + i);
+            a = make_double2(f.x, f.y);
+            b = make_double2(f.z, f.w);
+        } else {
+            const uint2 u = *(const uint2*)((const __half*)it.src + i);
+            const __half2 h0 = *(const __half2*)&u.x, h1 = *(const __half2*)&u.y;
+            a = make_double2(__low2float(h0), __high2float(h0));
+            b = make_double2(__low2float(h1), __high2float(h1));
         }
+        *(double2*)(it.p64 + i) = a;
+        *(double2*)(it.p64 + i + 2) = b;
     }
 }
 
@@ -102,17 +110,25 @@ cudaError_t set_flag_launch(uint64_t* flag, uint64_t v, cudaStream_t s) {
     return cudaGetLastError();
 }
 
+// grid: about four waves of 148 SMs x 8 CTAs over all items, at least one CTA per item
+static dim3 xfer_grid(int64_t elems, int n) {
+    int64_t per = (4LL * 148 * 8 + n - 1) / n;
+    const int64_t maxc = (elems / 4 + 255) / 256;
+    per = std::max<int64_t>(1, std::min(per, maxc));
+    return dim3((unsigned)per, n);
+}
+
 cudaError_t pack_launch(const PackItem* items, int n, int64_t elems, cudaStream_t s) {
     if (n <= 0) return cudaSuccess;
-    dim3 grid((unsigned)std::min<int64_t>((elems + 255) / 256, 64), n);
-    pack_kernel<<<grid, 256, 0, s>>>(items, elems);
+    if (elems % 4) return cudaErrorInvalidValue;
+    pack_kernel<<<xfer_grid(elems, n), 256, 0, s>>>(items, elems);
     return cudaGetLastError();
 }
 
 cudaError_t pull_launch(const PullItem* items, int n, int64_t elems, cudaStream_t s) {
     if (n <= 0) return cudaSuccess;
-    dim3 grid((unsigned)std::min<int64_t>((elems + 255) / 256, 64), n);
-    pull_kernel<<<grid, 256, 0, s>>>(items, elems);
+    if (elems % 4) return cudaErrorInvalidValue;
+    pull_kernel<<<xfer_grid(elems, n), 256, 0, s>>>(items, elems);
     return cudaGetLastError();
 }
 

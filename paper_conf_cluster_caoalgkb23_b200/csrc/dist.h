@@ -21,10 +21,7 @@ struct PullItem {
     const void* src;       // peer payload (comm precision)
     const uint64_t* flag;  // peer stamp for that payload
     uint64_t target;
-    double* p64;           // local FP64 panel slot
-    __half* p16;           // optional caches (null if no local successor needs them)
-    float* hi;
-    float* lo;
+    double* p64;           // local FP64 panel slot (the operand formats are derived from it later)
     int prec;
     int pad;
 };

@@ -6,11 +6,14 @@
 //      block column as an in-place DMMA GEMM with the inverse, the trailing block SYRK;
 //   2. L~_kk = L_kk rounded to comm(k,k) (what the TRSMs receive, Alg. 2) + block inverses;
 //   3. panel in: the column's tiles (m,k), m > k, up-converted into the FP64 panel buffer;
-//   4. TRSM(m,k): blocked right-looking, two DMMA GEMMs per 128-column block, batched over m;
-//   5. panel out (K2): write back in storage precision, round to comm(m,k), derive the FP16 /
-//      TF32-pair operand copies for low-precision successors;
+//   4. TRSM(m,k): FP64-class tiles by blocked DMMA substitution, FP32/FP16-class tiles as the
+//      FP32-class product A_mk W^T with W = L~_kk^-1 (reading C12');
+//   5. panel out (K2): write back in storage precision, round to comm(m,k); multi-rank: publish /
+//      pull the panel tiles in comm precision;
+//   5e. operand formats (K2), once per panel and GPU: row-scaled FP16 hi/lo, TF32 pairs, CRT
+//      residue planes — single-buffered, produced on the update stream right before the update;
 //   6. trailing update: DSYRK(m,k) + GEMM(m,n,k) grouped by the kernel precision of the
-//      output tile: FP64 (DMMA), FP32 class and FP16 class.
+//      output tile: FP64 class (CRT INT8 / DMMA), FP32 class, FP16 class.
 // Everything for one call is planned on the host first (job arrays for the batched kernels),
 // uploaded once into the control arena of the workspace, then enqueued.
 #include <unistd.h>
@@ -28,7 +31,6 @@
 #include "kernels.h"
 #include "tc_gemm.h"
 #include "dist.h"
-#include "ozaki.h"
 #include "crt.h"
 
 using namespace mpgeo;
@@ -49,32 +51,49 @@ struct mp_handle {
     int* d_info = nullptr;
     cudaEvent_t ev[8] = {};
     bool broken = false;
-    int tc_mode = 1;  // 1: tcgen05 kernels for FP32/FP16 classes when available, 0: DMMA emulation
-    int lookahead = 1;  // 1: panel k+1 on the high-priority panel stream overlaps update k
-    int ozaki = 16;     // FP64-class GEMM/SYRK: 16 = CRT (Ozaki-II, 16 moduli) / 8 = 8-slice splitting,
-                        // both on INT8 tensor cores; 0 = DMMA
-    int matern_table = 1;  // general nu: tabulated correlation (1) or direct K_nu per entry (0)
-    int ozaki32 = 0;    // 1: FP32-class GEMM on INT8 tensor cores (first 4 slices); 0: 3xTF32 tcgen05 (default)
-    int f16x3 = 1;      // FP32-class update as 3xFP16 (row-scaled FP16 hi/lo split, kind::f16; reading C13c); 0: 3xTF32
-    int crt32 = 0;      // with the CRT FP64 engine: FP32-class GEMM as 8 INT8 GEMMs (CRT-8, FP32 C); opt-in:
-                        // measured slower than 3xTF32 inside the evaluation (profiles/r01/README.md)
-    int crt_trsm = 1;   // with the CRT FP64 engine: TRSM of FP32/FP16-class tiles as the FP32-class product
-                        // A_mk W^T, W = L~_kk^-1 (CRT-8), instead of the blocked DMMA substitution
-    int reserve_pairs = 6;   // lookahead: CTA pairs the persistent update kernels leave to the panel stream
+    mp_config cfg{};       // engines and schedule switches (mp_init_config)
+    uint8_t id[128] = {};  // communicator id (mp_get_unique_id); all zero = none
+    bool has_id = false;
     cudaStream_t pstream = nullptr;
     std::vector<cudaEvent_t> sync_ev;
     // profiling (mp_set_profiling): event pairs per launch, resolved in mp_get_profile
     bool profiling = false;
+    unsigned prof_mask = 0;  // classes whose launches get event pairs (mp_set_profiling_mask)
     std::vector<cudaEvent_t> prof_pool;
     size_t prof_free = 0;
     std::vector<ProfRec> prof_pending;
     mp_profile prof = {};
 };
 
+// The engines one matrix runs with: the handle's configuration where the tile size allows it
+// (the tcgen05 kernels tile nb by 256).  plan_potrf, the workspace layout and mp_matrix_engines all
+// read this one predicate.
+struct Engines {
+    bool crt = false;        // FP64 class: CRT (16 moduli) on INT8 tcgen05; else DMMA
+    bool tc16 = false;       // FP16 class: row-scaled FP16 on tcgen05; else DMMA on FP16-rounded operands
+    int f32 = MP_F32_DMMA;   // FP32 class engine (mp_fp32_engine)
+    bool ctrsm = false;      // FP32/FP16-class TRSM as the CRT-8 product with the inverse factor
+    bool h16 = false;        // row-scaled FP16 hi (+ lo) caches exist
+    bool p64_double = false; // the update reads the FP64 panel buffer (a DMMA class): two panel sets
+};
+static Engines engines_for(const mp_handle* h, int nb) {
+    Engines e;
+    const bool tcok = tc_gemm_available() && nb % 256 == 0;
+    e.crt = h->cfg.fp64_engine == MP_F64_CRT16 && crt_available() && nb % 256 == 0;
+    e.tc16 = h->cfg.fp16_tensor != 0 && tcok;
+    e.f32 = (h->cfg.fp32_engine == MP_F32_3XFP16 || h->cfg.fp32_engine == MP_F32_3XTF32) && tcok ? h->cfg.fp32_engine
+                                                                                                : MP_F32_DMMA;
+    e.ctrsm = e.crt && h->cfg.lowp_trsm_product != 0;
+    e.h16 = e.tc16 || e.f32 == MP_F32_3XFP16;
+    e.p64_double = h->cfg.lookahead != 0 && (!e.crt || !e.tc16 || e.f32 == MP_F32_DMMA);
+    return e;
+}
+
 struct Regions {
     size_t total = 0;
-    size_t inputs = 0, p64 = 0, p16 = 0, phi = 0, plo = 0, oz32 = 0, ltilde = 0, wbuf = 0, wbuf2 = 0, oz = 0, ozexp = 0,
-           wdiag = 0, mtab = 0, crt = 0, crtflags = 0, crtctr = 0;
+    size_t inputs = 0, p64 = 0, h16 = 0, e16 = 0, phi = 0, plo = 0, oz32 = 0, e32 = 0, ltilde = 0, wbuf = 0,
+           wbuf2 = 0, wfac = 0, oz = 0, ozexp = 0, wdiag = 0, mtab = 0, crt = 0, crtflags = 0, crtctr = 0;
+    int p64_sets = 1;              // 2 when the update reads the FP64 panel buffer (Engines::p64_double)
     size_t vec_r = 0, vec_y = 0, partials = 0, norms = 0, ctrl = 0, ctrl_bytes = 0;
     std::vector<size_t> tile_off;  // per (m*nt+k), SIZE_MAX if not stored here
     size_t pool = 0;               // start of the tile pool
@@ -88,8 +107,8 @@ struct Comm {
     std::vector<char*> peer;  // base of every rank's area (own = base)
     bool connected = false;
     uint64_t epoch = 0;       // incremented per collective call; stamps = epoch << 24 | step
-    size_t send = 0, pub = 0, done = 0, bar = 0, part = 0, yv = 0, pflag = 0, yflag = 0, norms = 0, nflag = 0,
-           scal = 0, sflag = 0, tmp = 0;
+    size_t hdr = 0, send = 0, pub = 0, done = 0, bar = 0, part = 0, yv = 0, pflag = 0, yflag = 0, norms = 0,
+           nflag = 0, scal = 0, sflag = 0, tmp = 0;
 };
 
 struct mp_matrix {
@@ -146,17 +165,21 @@ static size_t ctrl_bytes_for(int nt, int nb) {
     bytes += T * T * sizeof(GemvTile);
     bytes += T * (sizeof(double*) + sizeof(int));
     bytes += T * T * (sizeof(PackItem) + sizeof(PullItem) + 2 * sizeof(WaitItem)) + T * 8 * sizeof(WaitItem);
-    bytes += T * T * sizeof(OzSplitItem) + T * (T + 1) * (T + 2) / 6 * sizeof(OzJob);
+    bytes += T * T * (sizeof(CrtSplitItem) + sizeof(Split16Item) + sizeof(Tf32Item)) + T * (T + 1) * (T + 2) / 6 * sizeof(CrtJob);
     bytes += 64 * 1024 + 32 * 256;  // alignment slack
     return bytes;
 }
 
+// storage == NULL: all FP64 (the worst case); storage == NO_POOL: no tile pool (mp_matrix_attach)
+static const uint8_t* const NO_POOL = (const uint8_t*)1;
+
 static Regions layout(const mp_matrix* A, const uint8_t* storage) {
-    // Map-independent regions first (their offsets depend only on n, nb, NT), then the tile
-    // pool, whose slots depend on the storage map (re-laid out per evaluation).
+    // Map-independent regions first (their offsets depend only on n, nb, NT and the engines), then
+    // the tile pool, whose slots depend on the storage map (re-laid out per evaluation).
     Regions R;
     const int nt = A->nt;
     const size_t nb2 = A->nb2();
+    const Engines E = engines_for(A->h, A->nb);
     size_t off = 0;
     auto take = [&](size_t bytes) {
         off = align_up(off, 256);
@@ -165,6 +188,7 @@ static Regions layout(const mp_matrix* A, const uint8_t* storage) {
         return o;
     };
     const size_t nvec = (size_t)nt * A->nb;
+    const size_t slots = (size_t)nt * nb2;  // one panel: slot m holds tile (m, k)
     R.inputs = take(3 * nvec * 8);
     R.vec_r = take(nvec * 8);
     R.vec_y = take(nvec * 8);
@@ -178,33 +202,40 @@ static Regions layout(const mp_matrix* A, const uint8_t* storage) {
     R.wbuf2 = take((size_t)ceil_div(A->nb, POTRF_IB) * POTRF_IB * POTRF_IB * 8);
     R.wdiag = take((size_t)nt * ceil_div(A->nb, POTRF_IB) * POTRF_IB * POTRF_IB * 8);  // solve: block inverses
     R.mtab = take((size_t)MT_PIECES_MAX * (MT_DEG + 1) * 8);  // general-nu Matern table
-    // two sets of panel buffers (panel parity) so panel k+1 can be produced while update k reads panel k
-    R.p64 = take(2 * (size_t)nt * nb2 * 8);
-    R.p16 = take(2 * (size_t)nt * nb2 * 2);
-    // int8 operand planes of the FP64-class engine, two sets: 8 slices (splitting) or 16 residues (CRT)
-    const bool crt = A->h && A->h->ozaki == 16 && A->nb % 256 == 0;
-    // FP32-class operands: TF32 hi/lo pairs (3xTF32), or with the CRT engine 8 residue planes (CRT-8)
-    const bool crt32 = crt && A->h->crt32;
-    if (crt32 || (crt && A->h->crt_trsm)) R.oz32 = take(2 * (size_t)nt * nb2 * 8);
-    if (!crt32) {
-        R.phi = take(2 * (size_t)nt * nb2 * 4);
-        R.plo = take(2 * (size_t)nt * nb2 * 4);
+    // FP64 panel buffer: written by panel k+1's POTRF/TRSM (panel stream) while update k runs, so
+    // two sets only if update k reads it (a DMMA class); the operand formats below are derived from
+    // it after update k and are single-buffered
+    R.p64_sets = E.p64_double ? 2 : 1;
+    R.p64 = take(R.p64_sets * slots * 8);
+    if (E.h16) {  // row-scaled FP16 hi and lo planes + row exponents (3xFP16 FP32 class, FP16 class)
+        R.h16 = take(2 * slots * 2);
+        R.e16 = take(nvec * 4);
     }
-    R.oz = take(2 * (size_t)nt * nb2 * (crt ? CRT_NMAX : 8));
-    if (crt) {  // CRT engine: per-CTA residue staging slots + their busy flags
+    if (E.f32 == MP_F32_3XTF32) {
+        R.phi = take(slots * 4);
+        R.plo = take(slots * 4);
+    }
+    if (E.crt) {  // FP64 class: 16 residue planes + row exponents; per-CTA residue staging slots
+        R.oz = take(slots * CRT_NMAX);
+        R.ozexp = take(nvec * 4);
         R.crt = take((size_t)crt_scratch_slots() * CRT_SLOT_BYTES);
         R.crtflags = take((size_t)crt_scratch_slots() * sizeof(int));
         R.crtctr = take(crt_counters(nt) * sizeof(int));
     }
-    R.ozexp = take(2 * (size_t)nt * A->nb * 4);    // per-row exponents
+    if (E.ctrsm) {  // the TRSM product's operands (8 residue planes, own exponents) and W = L~_kk^-1
+        R.oz32 = take(slots * 8);
+        R.e32 = take(nvec * 4);
+        R.wfac = take(nb2 * 8);
+    }
     R.tile_off.assign((size_t)nt * nt, SIZE_MAX);
     R.pool = align_up(off, 256);  // tile pool start (tile offsets from here are whole nb-float rows when 256 | nb)
-    for (int k = 0; k < nt; ++k)
-        for (int m = k; m < nt; ++m)
-            if (A->mine(m, k)) {
-                const uint8_t p = storage ? storage[(size_t)m * nt + k] : (uint8_t)MP_FP64;
-                R.tile_off[(size_t)m * nt + k] = take(nb2 * (p == MP_FP64 ? 8 : 4));
-            }
+    if (storage != NO_POOL)
+        for (int k = 0; k < nt; ++k)
+            for (int m = k; m < nt; ++m)
+                if (A->mine(m, k)) {
+                    const uint8_t p = storage ? storage[(size_t)m * nt + k] : (uint8_t)MP_FP64;
+                    R.tile_off[(size_t)m * nt + k] = take(nb2 * (p == MP_FP64 ? 8 : 4));
+                }
     R.total = align_up(off, 256);
     return R;
 }
@@ -270,7 +301,7 @@ static mp_status run_plan(mp_handle* h, mp_matrix* A, Arena& ar, std::vector<Op>
             CK(h, cudaStreamWaitEvent(st, h->sync_ev[op.ev], 0));
             continue;
         }
-        if (h->profiling) {
+        if (h->profiling && ((h->prof_mask >> op.cls) & 1u)) {
             cudaEvent_t e0 = prof_event(h), e1 = prof_event(h);
             CK(h, cudaEventRecord(e0, st));
             CK(h, op.fn(st));
@@ -288,32 +319,66 @@ static mp_status run_plan(mp_handle* h, mp_matrix* A, Arena& ar, std::vector<Op>
 extern "C" {
 
 const char* mp_version(void) {
-    return "mpgeo 0.1 sm_100a (FP64 class: CRT INT8 tcgen05 | 8-slice | DMMA; FP32 class: 3xFP16 | 3xTF32; FP16 class: tcgen05 f16)";
+    return "mpgeo 0.2 sm_100a (FP64 class: CRT INT8 tcgen05 | DMMA; FP32 class: 3xFP16 | 3xTF32 tcgen05 | DMMA; "
+           "FP16 class: row-scaled f16 tcgen05 | DMMA)";
 }
 
-mp_status mp_init(int device, int rank, int nranks, int P, int Q, const uint8_t* id, void* cuda_stream,
-                  mp_handle** out) {
+void mp_config_default(mp_config* c) {
+    if (!c) return;
+    c->fp64_engine = MP_F64_CRT16;
+    c->fp32_engine = MP_F32_3XFP16;
+    c->fp16_tensor = 1;
+    c->lookahead = 1;
+    c->reserve_pairs = 6;
+    c->lowp_trsm_product = 1;
+    c->matern_table = 1;
+    c->f16x3_persistent = 0;
+    c->crt_phase_lock = 1;
+}
+
+mp_status mp_get_unique_id(uint8_t id[128]) {
+    if (!id) return MP_ERR_ARG;
+    memset(id, 0, 128);
+    FILE* f = fopen("/dev/urandom", "rb");
+    if (!f || fread(id, 1, 32, f) != 32) {
+        if (f) fclose(f);
+        return MP_ERR_UNSUPPORTED;
+    }
+    fclose(f);
+    const long pid = (long)getpid();
+    memcpy(id + 32, &pid, sizeof pid);
+    gethostname((char*)id + 48, 79);
+    id[127] = 0;
+    return MP_OK;
+}
+
+mp_status mp_init_config(int device, int rank, int nranks, int P, int Q, const uint8_t* id, void* cuda_stream,
+                         const mp_config* cfg, mp_handle** out) {
     if (!out || nranks < 1 || rank < 0 || rank >= nranks || P < 1 || Q < 1 || P * Q != nranks || P > Q)
         return MP_ERR_ARG;
+    *out = nullptr;
+    if (nranks > MAX_PEERS) return MP_ERR_UNSUPPORTED;
+    if (nranks > 1 && !id) return MP_ERR_ARG;  // multi-rank: the communicator id of mp_get_unique_id
     mp_handle* h = new mp_handle();
     h->device = device;
     h->rank = rank;
     h->nranks = nranks;
     h->P = P;
     h->Q = Q;
-    if (const char* e = getenv("MPGEO_TC")) h->tc_mode = atoi(e);
-    if (const char* e = getenv("MPGEO_LOOKAHEAD")) h->lookahead = atoi(e);
-    if (const char* e = getenv("MPGEO_OZAKI")) h->ozaki = atoi(e);
-    if (const char* e = getenv("MPGEO_OZAKI32")) h->ozaki32 = atoi(e);
-    if (const char* e = getenv("MPGEO_CRT32")) h->crt32 = atoi(e);
-    if (const char* e = getenv("MPGEO_F16X3")) h->f16x3 = atoi(e);
-    if (const char* e = getenv("MPGEO_CRT_TRSM")) h->crt_trsm = atoi(e);
-    if (const char* e = getenv("MPGEO_RESERVE_PAIRS")) h->reserve_pairs = std::max(0, atoi(e));
-    if (const char* e = getenv("MPGEO_MATERN_TABLE")) h->matern_table = atoi(e);
-    auto fail = [&](mp_status s) {
+    mp_config_default(&h->cfg);
+    if (cfg) h->cfg = *cfg;
+    if (h->cfg.reserve_pairs < 0) h->cfg.reserve_pairs = 0;
+    if (id) {
+        memcpy(h->id, id, 128);
+        h->has_id = true;
+    }
+    auto fail = [&](mp_status s) {  // release everything created so far
+        for (auto& e : h->ev)
+            if (e) cudaEventDestroy(e);
+        if (h->d_info) cudaFree(h->d_info);
+        if (h->pstream) cudaStreamDestroy(h->pstream);
         if (h->own_stream && h->stream) cudaStreamDestroy(h->stream);
         delete h;
-        *out = nullptr;
         return s;
     };
     if (cudaSetDevice(device) != cudaSuccess) return fail(MP_ERR_CUDA);
@@ -331,9 +396,18 @@ mp_status mp_init(int device, int rank, int nranks, int P, int Q, const uint8_t*
     if (cudaMalloc(&h->d_info, sizeof(int)) != cudaSuccess) return fail(MP_ERR_CUDA);
     for (auto& e : h->ev)
         if (cudaEventCreate(&e) != cudaSuccess) return fail(MP_ERR_CUDA);
-    (void)id;  // reserved: the panel exchange is peer memory (mp_matrix_comm_export/connect)
-    if (nranks > MAX_PEERS) return fail(MP_ERR_UNSUPPORTED);
     *out = h;
+    return MP_OK;
+}
+
+mp_status mp_init(int device, int rank, int nranks, int P, int Q, const uint8_t* id, void* cuda_stream,
+                  mp_handle** out) {
+    return mp_init_config(device, rank, nranks, P, Q, id, cuda_stream, nullptr, out);
+}
+
+mp_status mp_handle_get_config(const mp_handle* h, mp_config* cfg) {
+    if (!h || !cfg) return MP_ERR_ARG;
+    *cfg = h->cfg;
     return MP_OK;
 }
 
@@ -356,14 +430,19 @@ mp_status mp_finalize(mp_handle* h) {
 
 const char* mp_last_error(const mp_handle* h) { return h ? h->err.c_str() : "null handle"; }
 
-mp_status mp_set_profiling(mp_handle* h, int enable) {
+mp_status mp_set_profiling_mask(mp_handle* h, unsigned mask) {
     if (!h) return MP_ERR_ARG;
     if (!h->prof_pending.empty()) CK(h, cudaStreamSynchronize(h->stream));
     h->prof_pending.clear();
     h->prof_free = 0;
     h->prof = mp_profile{};
-    h->profiling = enable != 0;
+    h->prof_mask = mask & ((1u << MP_PROF_CLASSES) - 1);
+    h->profiling = h->prof_mask != 0;
     return MP_OK;
+}
+
+mp_status mp_set_profiling(mp_handle* h, int enable) {
+    return mp_set_profiling_mask(h, enable ? (1u << MP_PROF_CLASSES) - 1 : 0u);
 }
 
 mp_status mp_get_profile(mp_handle* h, mp_profile* out) {
@@ -398,14 +477,13 @@ mp_status mp_get_profile(mp_handle* h, mp_profile* out) {
 }
 int64_t mp_launch_count(const mp_handle* h) { return h ? h->launches : 0; }
 
-mp_status mp_handle_config(const mp_handle* h, int* tc, int* lookahead, int* ozaki) {
-    if (!h) return MP_ERR_ARG;
-    // ozaki: 0 = DMMA FP64 class; 8 = INT8 FP64 class; +100 if the FP32 class also runs on INT8
-    if (tc) *tc = (h->tc_mode != 0 && tc_gemm_available()) ? (h->f16x3 ? 2 : 1) : 0;
-    if (lookahead) *lookahead = h->lookahead;
-    if (ozaki)
-        *ozaki = (h->ozaki == 16 && crt_available()) ? (16 + (h->crt32 ? 200 : 0))
-                 : (h->ozaki == 8 && ozaki_available()) ? (8 + (h->ozaki32 ? 100 : 0)) : 0;
+mp_status mp_matrix_engines(const mp_matrix* A, int* fp64, int* fp32, int* fp16, int* lowp_trsm) {
+    if (!A) return MP_ERR_ARG;
+    const Engines e = engines_for(A->h, A->nb);
+    if (fp64) *fp64 = e.crt ? MP_F64_CRT16 : MP_F64_DMMA;
+    if (fp32) *fp32 = e.f32;
+    if (fp16) *fp16 = e.tc16 ? 1 : 0;
+    if (lowp_trsm) *lowp_trsm = e.ctrsm ? 1 : 0;
     return MP_OK;
 }
 
@@ -443,6 +521,7 @@ static size_t comm_layout(mp_matrix* A) {
         off += bytes;
         return o;
     };
+    c.hdr = take(128);  // the communicator id (mp_get_unique_id), checked by every peer at connect
     c.send = take(2 * nt * nb2 * 8);
     c.pub = take(2 * nt * 8);
     c.done = take(2 * 8);
@@ -468,6 +547,7 @@ mp_status mp_matrix_comm_export(mp_matrix* A, void* handle_out) {
         c.bytes = comm_layout(A);
         CK(h, cudaMalloc(&c.base, c.bytes));
         CK(h, cudaMemset(c.base, 0, c.bytes));
+        CK(h, cudaMemcpy(c.base + c.hdr, h->id, 128, cudaMemcpyHostToDevice));
         CK(h, cudaDeviceSynchronize());
     }
     cudaIpcMemHandle_t ih;
@@ -492,6 +572,10 @@ mp_status mp_matrix_comm_connect(mp_matrix* A, const void* all_handles) {
         void* p = nullptr;
         CK(h, cudaIpcOpenMemHandle(&p, ih, cudaIpcMemLazyEnablePeerAccess));
         c.peer[r] = (char*)p;
+        uint8_t pid[128];
+        CK(h, cudaMemcpy(pid, c.peer[r] + c.hdr, 128, cudaMemcpyDeviceToHost));
+        if (memcmp(pid, h->id, 128) != 0)
+            FAIL(h, MP_ERR_COMM, "rank %d's exchange area carries another communicator id (mp_get_unique_id)", r);
     }
     c.connected = true;
     return MP_OK;
@@ -532,6 +616,21 @@ mp_status mp_matrix_bind(mp_matrix* A, const uint8_t* storage_prec, void* d_work
     return MP_OK;
 }
 
+mp_status mp_matrix_attach(mp_matrix* A, void* d_workspace, size_t bytes) {
+    if (!A || !d_workspace) return MP_ERR_ARG;
+    mp_handle* h = A->h;
+    if ((uintptr_t)d_workspace % 256) FAIL(h, MP_ERR_ARG, "workspace must be 256-byte aligned");
+    Regions R = layout(A, NO_POOL);
+    if (R.total > bytes) FAIL(h, MP_ERR_NOMEM, "workspace %zu bytes < map-independent regions %zu", bytes, R.total);
+    A->R = std::move(R);
+    A->ws = (char*)d_workspace;
+    A->ws_bytes = bytes;
+    A->storage.assign((size_t)A->nt * A->nt, 255);
+    A->bound = true;  // pass 1 of the generation (norms) needs only the map-independent regions
+    A->generated = A->factored = false;
+    return MP_OK;
+}
+
 mp_status mp_matrix_maps(const mp_matrix* A, uint8_t* kernel_prec, uint8_t* storage_prec, uint8_t* comm_prec) {
     if (!A) return MP_ERR_ARG;
     const size_t NN = (size_t)A->nt * A->nt;
@@ -544,6 +643,7 @@ mp_status mp_matrix_maps(const mp_matrix* A, uint8_t* kernel_prec, uint8_t* stor
 mp_status mp_matrix_get_tile(mp_handle* h, const mp_matrix* A, int m, int k, double* h_tile) {
     if (!h || !A || !h_tile || !A->bound || m < k || m >= A->nt || k < 0) return MP_ERR_ARG;
     if (!A->mine(m, k)) FAIL(h, MP_ERR_ARG, "tile (%d,%d) not owned by rank %d", m, k, h->rank);
+    if (A->R.tile_off[(size_t)m * A->nt + k] == SIZE_MAX) FAIL(h, MP_ERR_STATE, "no tile pool laid out");
     const size_t nb2 = A->nb2();
     if (A->st(m, k) == MP_FP64) {
         CK(h, cudaMemcpyAsync(h_tile, A->tile(m, k), nb2 * 8, cudaMemcpyDeviceToHost, h->stream));
@@ -560,6 +660,7 @@ mp_status mp_matrix_get_tile(mp_handle* h, const mp_matrix* A, int m, int k, dou
 mp_status mp_matrix_set_tile(mp_handle* h, mp_matrix* A, int m, int k, const double* h_tile) {
     if (!h || !A || !h_tile || !A->bound || m < k || m >= A->nt || k < 0) return MP_ERR_ARG;
     if (!A->mine(m, k)) FAIL(h, MP_ERR_ARG, "tile (%d,%d) not owned by rank %d", m, k, h->rank);
+    if (A->R.tile_off[(size_t)m * A->nt + k] == SIZE_MAX) FAIL(h, MP_ERR_STATE, "no tile pool laid out");
     const size_t nb2 = A->nb2();
     if (A->st(m, k) == MP_FP64) {
         CK(h, cudaMemcpyAsync(A->tile(m, k), h_tile, nb2 * 8, cudaMemcpyHostToDevice, h->stream));
@@ -642,7 +743,7 @@ mp_status mp_matern_gen(mp_handle* h, mp_matrix* A, const double* d_x, const dou
     if (h->nranks > 1 && !A->comm.connected) FAIL(h, MP_ERR_COMM, "multi-rank matrix not connected");
     const int nt = A->nt;
     MaternArgs a = matern_args(A, d_x, d_y, theta);
-    if (a.kind == 3 && A->bound && h->matern_table) {
+    if (a.kind == 3 && A->bound && h->cfg.matern_table) {
         // pieces of width w = 1/8 in u = log(r/2) on [-w*split, log(r_max/2)]; r_max bounds every
         // distance of points in the unit square (sqrt 2) — outside points fall back to direct K_nu
         const double w = 0.125;
@@ -736,44 +837,42 @@ static mp_status plan_potrf(mp_handle* h, mp_matrix* A, const uint8_t* km, const
                             std::vector<Op>& ops, FlopCount& fc, uint64_t epoch) {
     const int nt = A->nt, nb = A->nb, IB = POTRF_IB, OB = 4 * POTRF_IB;
     const size_t nb2 = A->nb2();
-    double* const p64b = A->at<double>(A->R.p64);
-    __half* const p16b = A->at<__half>(A->R.p16);
-    float* const phib = A->at<float>(A->R.phi);
-    float* const plob = A->at<float>(A->R.plo);
-    double* ltil = A->at<double>(A->R.ltilde);
-    double* wb = A->at<double>(A->R.wbuf);
-    double* wb2 = A->at<double>(A->R.wbuf2);
+    const size_t slots = (size_t)nt * nb2;  // elements of one panel's worth of slots
+    const Engines E = engines_for(h, nb);
+    const Regions& RG = A->R;
+    double* const p64b = A->at<double>(RG.p64);
+    __half* const h16hi = E.h16 ? A->at<__half>(RG.h16) : nullptr;  // [nt*nb][nb] hi planes, then lo
+    __half* const h16lo = E.h16 ? h16hi + slots : nullptr;
+    int* const e16 = E.h16 ? A->at<int>(RG.e16) : nullptr;
+    float* const phi = RG.phi ? A->at<float>(RG.phi) : nullptr;
+    float* const plo = RG.plo ? A->at<float>(RG.plo) : nullptr;
+    double* ltil = A->at<double>(RG.ltilde);
+    double* wb = A->at<double>(RG.wbuf);
+    double* wb2 = A->at<double>(RG.wbuf2);
     int* d_info = h->d_info;
-    const bool use_tc = h->tc_mode != 0 && tc_gemm_available() && nb % 256 == 0;
-    const float* const cpool = A->at<float>(A->R.pool);                // tcgen05 epilogue C map range
-    const uint64_t crows = (A->R.total - A->R.pool) / ((size_t)nb * 4);
-    const double* const cpool64 = A->at<double>(A->R.pool);  // FP64 view of the pool (CRT epilogue C map)
-    const uint64_t crows64 = (A->R.total - A->R.pool) / ((size_t)nb * 8);
-    const bool crt = h->ozaki == 16 && crt_available() && nb % 256 == 0 && A->R.crt;
+    const float* const cpool = A->at<float>(RG.pool);  // tcgen05 epilogue C map range (FP32 view of the pool)
+    const uint64_t crows = (RG.total - RG.pool) / ((size_t)nb * 4);
+    const double* const cpool64 = A->at<double>(RG.pool);  // FP64 view of the pool (CRT epilogue C map)
+    const uint64_t crows64 = (RG.total - RG.pool) / ((size_t)nb * 8);
     CrtConst crtc, crtc32;
-    if (crt && !crt_constants(CRT_NMAX, nb, &crtc)) FAIL(h, MP_ERR_ARG, "CRT constants for nb=%d", nb);
-    // FP32 class on the CRT engine: 8 moduli (b = 25 operand bits at nb = 2048), FP32 C
-    const bool crt32 = crt && h->crt32 && A->R.oz32 && use_tc;
-    const bool f16x3 = h->f16x3 != 0;
-    // low-precision-class TRSMs as CRT-8 products with the inverse factor (FP32 TRSM there)
-    const bool ctrsm = crt && h->crt_trsm && A->R.oz32 && nb % 32 == 0;
-    if ((crt32 || ctrsm) && !crt_constants(8, nb, &crtc32)) FAIL(h, MP_ERR_ARG, "CRT-8 constants for nb=%d", nb);
-    int8_t* const oz32b = (crt32 || ctrsm) ? A->at<int8_t>(A->R.oz32) : nullptr;
-    // the 8-slice splitting engine: selected (8), or the fallback of the CRT engine when nb % 256 != 0
-    const int ozS = !crt && (h->ozaki == 8 || h->ozaki == 16) && ozaki_available() && nb % 128 == 0 ? 8 : 0;
-    const bool oz32 = ozS && h->ozaki32 && nb % 256 == 0;
-    int8_t* const ozb = A->at<int8_t>(A->R.oz);
-    uint8_t* const crt_scr = crt ? A->at<uint8_t>(A->R.crt) : nullptr;
-    int* const crt_flags = crt ? A->at<int>(A->R.crtflags) : nullptr;
+    if (E.crt && !crt_constants(CRT_NMAX, nb, &crtc)) FAIL(h, MP_ERR_ARG, "CRT constants for nb=%d", nb);
+    if (E.ctrsm && !crt_constants(8, nb, &crtc32)) FAIL(h, MP_ERR_ARG, "CRT-8 constants for nb=%d", nb);
+    int8_t* const ozs = E.crt ? A->at<int8_t>(RG.oz) : nullptr;
+    int* const oze = E.crt ? A->at<int>(RG.ozexp) : nullptr;
+    int8_t* const o32s = E.ctrsm ? A->at<int8_t>(RG.oz32) : nullptr;
+    int* const e32 = E.ctrsm ? A->at<int>(RG.e32) : nullptr;
+    double* const wfac = E.ctrsm ? A->at<double>(RG.wfac) : nullptr;
+    const int64_t plane = (int64_t)slots;  // bytes between int8 residue planes
+    uint8_t* const crt_scr = E.crt ? A->at<uint8_t>(RG.crt) : nullptr;
+    int* const crt_flags = E.crt ? A->at<int>(RG.crtflags) : nullptr;
     // one tile-scheduler counter per CRT launch of this call (zeroed by potrf_run)
-    int* const crt_ctr = crt ? A->at<int>(A->R.crtctr) : nullptr;
+    int* const crt_ctr = E.crt ? A->at<int>(RG.crtctr) : nullptr;
     size_t ctr_next = 0;
     auto next_ctr = [&]() -> int* {  // two ints per launch
         if (ctr_next + 2 > crt_counters(nt)) return nullptr;
         ctr_next += 2;
         return crt_ctr + ctr_next - 2;
     };
-    int* const ozeb = A->at<int>(A->R.ozexp);
     auto K = [&](int m, int k) { return km[(size_t)m * nt + k]; };
     auto C = [&](int m, int k) { return cm[(size_t)m * nt + k]; };
     const double fnb = (double)nb;
@@ -781,11 +880,11 @@ static mp_status plan_potrf(mp_handle* h, mp_matrix* A, const uint8_t* km, const
     auto cur_push = [&](Op o) { cur->push_back(std::move(o)); };
     // ---- multi-rank exchange helpers; unused on one rank
     const bool dist = h->nranks > 1;
-    const bool la = h->lookahead != 0;  // also multi-rank: exchange waits run on the panel stream
+    const bool la = h->cfg.lookahead != 0;  // also multi-rank: exchange waits run on the panel stream
     // persistent CRT grids: the update leaves reserve_pairs CTA pairs to the panel stream (lookahead)
     int nsm = 148;
     cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, h->device);
-    const int upd_pairs = la ? std::max(1, nsm / 2 - h->reserve_pairs) : 0;
+    const int upd_pairs = la ? std::max(1, nsm / 2 - h->cfg.reserve_pairs) : 0;
     const int pan_pairs = 0;  // panel-stream CRT launches: any free SM (dynamic tiles, high priority)
     const int R = h->nranks, me = h->rank;
     Comm& X = A->comm;
@@ -802,12 +901,15 @@ static mp_status plan_potrf(mp_handle* h, mp_matrix* A, const uint8_t* km, const
         if (mp_exchange_plan(nt, h->P, h->Q, me, cm, xs.data(), cnt, &cnt)) FAIL(h, MP_ERR_ARG, "exchange plan failed");
         for (auto& x : xs) (x.dir == 0 ? xpub : xpull)[x.k].push_back(x);
     }
-    auto local_formats = [&](int k, int m, bool& n16, bool& n32) {  // operand formats of MY successors of L_mk
+    // the operand classes MY successors of L_mk run at: SYRK(m,k) on (m,m), GEMM(m,n,k), GEMM(n,m,k)
+    auto needs = [&](int k, int m, bool& n16, bool& n32, bool& n64) {
         n16 = n32 = false;
+        n64 = A->mine(m, m);
+        auto cls = [&](int p) { n16 |= p == MP_FP16, n32 |= p == MP_FP32, n64 |= p == MP_FP64; };
         for (int n = k + 1; n < m; ++n)
-            if (A->mine(m, n)) n16 |= K(m, n) == MP_FP16, n32 |= K(m, n) == MP_FP32;
+            if (A->mine(m, n)) cls(K(m, n));
         for (int n = m + 1; n < nt; ++n)
-            if (A->mine(n, m)) n16 |= K(n, m) == MP_FP16, n32 |= K(n, m) == MP_FP32;
+            if (A->mine(n, m)) cls(K(n, m));
     };
     auto push_wait = [&](std::vector<WaitItem>& w) {
         if (w.empty()) return;
@@ -816,9 +918,10 @@ static mp_status plan_potrf(mp_handle* h, mp_matrix* A, const uint8_t* km, const
         cur_push(Op{[=](cudaStream_t s) { return wait_flags_launch(dw, n, s); }, C_CONV, 0});
     };
 
-    // per step: panel(k) = POTRF + TRSM + conversion; next(k) = the update of column k+1 (what
-    // panel k+1 waits for); rest(k) = the rest of the trailing update
-    std::vector<std::vector<Op>> pan(nt), nxt(nt), rst(nt);
+    // per step: pan(k) = POTRF + TRSM + panel out (+ exchange); fmt(k) = the operand formats of
+    // panel k; nxt(k) = the update of column k+1 (what panel k+1 waits for); rst(k) = the rest of the
+    // trailing update
+    std::vector<std::vector<Op>> pan(nt), fmt(nt), nxt(nt), rst(nt);
     auto gemm = [&](std::vector<GemmJob>& jobs, int M, int N, int Kd, int lda, int ldb, int ldc, int lower,
                     double alpha, double beta, int round, bool cf32, int cls, double flops_per_job) {
         if (jobs.empty()) return;
@@ -837,9 +940,30 @@ static mp_status plan_potrf(mp_handle* h, mp_matrix* A, const uint8_t* km, const
         const int nj = (int)jobs.size();
         cur->push_back({[=](cudaStream_t s) { return dgemm_nt_launch(g, nj, round, cf32, s); }, cls, flops_per_job * nj});
     };
+    auto crt_args = [&](const CrtJob* dj, const int8_t* planes, const int* exps, int lower, const CrtConst& c,
+                        const void* cbase, uint64_t cr, int pairs, int store) {
+        CrtArgs a{};
+        a.jobs = dj;
+        a.planes = planes;
+        a.exps = exps;
+        a.plane_stride = plane;
+        a.nb = nb;
+        a.nt = nt;
+        a.lower = lower;
+        a.scratch = crt_scr;
+        a.slot_flags = crt_flags;
+        a.c = c;
+        a.cbase = cbase;
+        a.crows = cr;
+        a.max_pairs = pairs;
+        a.store = store;
+        a.counter = next_ctr();
+        a.phase_lock = h->cfg.crt_phase_lock;
+        return a;
+    };
 
     for (int k = 0; k < nt; ++k) {
-        const size_t set = la ? (size_t)(k & 1) : 0;
+        const size_t set = E.p64_double ? (size_t)(k & 1) : 0;
         const int sp = k & 1;  // send-slot parity (multi-rank)
         bool send_free_waited = false;
         auto wait_send_free = [&]() {  // every peer has pulled panel k-2 from slot set sp
@@ -850,20 +974,7 @@ static mp_status plan_potrf(mp_handle* h, mp_matrix* A, const uint8_t* km, const
             push_wait(w);
             send_free_waited = true;
         };
-        double* p64 = p64b + set * nt * nb2;
-        __half* p16 = p16b + set * nt * nb2;
-        float* phi = phib + set * nt * nb2;
-        float* plo = plob + set * nt * nb2;
-        int8_t* ozs = ozb + set * nt * nb2 * (crt ? CRT_NMAX : 8);
-        int* oze = ozeb + set * (size_t)nt * nb;
-        const int64_t ozplane = (int64_t)nt * nb2;
-        // 3xFP16 caches inside the TF32 hi/lo region of this set: hi at phi, lo at phi + nt nb^2
-        // halves, the row exponents at plo
-        auto s16item = [=](int m) {
-            __half* const h = (__half*)phi;
-            return Split16Item{p64 + (size_t)m * nb2, h + (size_t)m * nb2, h + (size_t)nt * nb2 + (size_t)m * nb2,
-                               (int*)plo + (size_t)m * nb};
-        };
+        double* p64 = p64b + set * slots;
         cur = &pan[k];
         // ---- 1. DPOTRF(k,k), FP64: two-level blocking — 128-column blocks
         //      (diagonal block Cholesky + inverse, block column as GEMM with the inverse, update
@@ -889,11 +1000,11 @@ static mp_status plan_potrf(mp_handle* h, mp_matrix* A, const uint8_t* km, const
                                    C_POTRF, (double)jb * jb * jb / 3.0});
                     const int rest = nb - jend;
                     if (rest <= 0) continue;
-                    double* X = Akk + (size_t)jend * nb + j0;
-                    std::vector<GemmJob> j1{GemmJob{X, wb, X}};
+                    double* Xb = Akk + (size_t)jend * nb + j0;
+                    std::vector<GemmJob> j1{GemmJob{Xb, wb, Xb}};
                     gemm(j1, rest, jb, jb, nb, IB, nb, 0, 1.0, 0.0, P64, false, C_POTRF, (double)rest * jb * jb);
                     if (Jend > jend) {
-                        std::vector<GemmJob> j2{GemmJob{X, X, Akk + (size_t)jend * nb + jend}};
+                        std::vector<GemmJob> j2{GemmJob{Xb, Xb, Akk + (size_t)jend * nb + jend}};
                         gemm(j2, rest, Jend - jend, jb, nb, nb, nb, 0, -1.0, 1.0, P64, false, C_POTRF,
                              2.0 * rest * (Jend - jend) * jb);
                     }
@@ -937,7 +1048,7 @@ static mp_status plan_potrf(mp_handle* h, mp_matrix* A, const uint8_t* km, const
                 const int o = pull_kk;
                 std::vector<WaitItem> w{WaitItem{pubflag(o, sp, k), ST(k)}};
                 push_wait(w);
-                std::vector<PullItem> pl{PullItem{sendslot(o, sp, k), pubflag(o, sp, k), ST(k), ltil, nullptr, nullptr, nullptr, pc, 0}};
+                std::vector<PullItem> pl{PullItem{sendslot(o, sp, k), pubflag(o, sp, k), ST(k), ltil, pc, 0}};
                 PullItem* dp = ar.push(pl);
                 cur_push(Op{[=](cudaStream_t s) { return pull_launch(dp, 1, (int64_t)nb2, s); }, C_CONV, 0});
             }
@@ -945,35 +1056,11 @@ static mp_status plan_potrf(mp_handle* h, mp_matrix* A, const uint8_t* km, const
                 cur->push_back({[=](cudaStream_t s) { return trtri_blocks_launch(ltil, nb, wb2, s); }, C_TRSM, 0});
         }
         // ---- 3. panel in
-        std::vector<PanelTile> pin, pout;
-        std::vector<Split16Item> s16out;  // 3xFP16 operands derived after panel out
-        for (int m = k + 1; m < nt; ++m) {
-            if (!A->mine(m, k)) continue;
-            PanelTile t{};
-            t.store = A->tile(m, k);
-            t.p64 = p64 + (size_t)m * nb2;
-            t.store_prec = A->st(m, k);
-            t.comm_prec = C(m, k);
-            pin.push_back(t);
-            // which operand formats do the successors of L_mk (row m, column m) on this GPU need?
-            bool need16 = false, need32 = false;
-            local_formats(k, m, need16, need32);
-            if (use_tc) {
-                if (need16) t.p16 = p16 + (size_t)m * nb2;
-                if (need32 && !oz32 && !crt32) {
-                    if (f16x3) {
-                        s16out.push_back(s16item(m));
-                    } else {
-                        t.hi = phi + (size_t)m * nb2;
-                        t.lo = plo + (size_t)m * nb2;
-                    }
-                }
-            }
-            pout.push_back(t);
-        }
+        std::vector<PanelTile> pin;
+        for (int m = k + 1; m < nt; ++m)
+            if (A->mine(m, k)) pin.push_back(PanelTile{A->tile(m, k), p64 + (size_t)m * nb2, A->st(m, k), C(m, k)});
         if (!pin.empty()) {
             PanelTile* d_in = ar.push(pin);
-            PanelTile* d_out = ar.push(pout);
             const int np = (int)pin.size();
             cur->push_back({[=](cudaStream_t s) { return panel_in_launch(d_in, np, (int64_t)nb2, s); }, C_CONV, 0});
             // ---- 4. TRSM(m,k): L_mk = A_mk L~_kk^{-T}.  FP64-class tiles: FP64 arithmetic (
@@ -984,7 +1071,7 @@ static mp_status plan_potrf(mp_handle* h, mp_matrix* A, const uint8_t* km, const
             std::vector<int> lo;      // low-precision-class tiles (ctrsm)
             for (auto& t : pin) {
                 const int m = (int)((t.p64 - p64) / (ptrdiff_t)nb2);
-                if (ctrsm && K(m, k) != MP_FP64) lo.push_back(m);
+                if (E.ctrsm && K(m, k) != MP_FP64) lo.push_back(m);
                 else dm.push_back(t.p64);
             }
             double* const islot = p64 + (size_t)k * nb2;  // panel slot k is free in panel k
@@ -1011,38 +1098,31 @@ static mp_status plan_potrf(mp_handle* h, mp_matrix* A, const uint8_t* km, const
                 }
             }
             // ---- 4b. FP32/FP16-class TRSM as the FP32-class product L_mk = A_mk W^T with the inverse
-            //      factor W = L~_kk^-1 (its FP64 substitution above, transposed into the L~ buffer, which
-            //      the substitution no longer reads): both operands as 8 CRT residue planes (b = 25 bits
-            //      per row), one CRT-8 launch over the column with an FP64 C (store mode) into the panel
-            //      slots, where the conversions of step 5 pick the tiles up as before.
+            //      factor W = L~_kk^-1 (its FP64 substitution above, transposed): both operands as 8 CRT
+            //      residue planes (b = 25 bits per row), one CRT-8 launch over the column with an FP64 C
+            //      (store mode) into the panel slots, where panel out (step 5) picks the tiles up.
             if (!lo.empty()) {
-                int8_t* const o32s = oz32b + set * nt * nb2 * 8;
-                double* const W = ltil;
-                cur->push_back({[=](cudaStream_t s) { return transpose_launch(islot, W, nb, s); }, C_TRSM, 0});
-                std::vector<CrtSplitItem> sp{CrtSplitItem{W, o32s + (size_t)k * nb2, oze + (size_t)k * nb, ozplane}};
-                std::vector<OzJob> tj;
+                cur->push_back({[=](cudaStream_t s) { return transpose_launch(islot, wfac, nb, s); }, C_TRSM, 0});
+                std::vector<CrtSplitItem> spl{CrtSplitItem{wfac, o32s + (size_t)k * nb2, e32 + (size_t)k * nb, plane}};
+                std::vector<CrtJob> tj;
                 for (int m : lo) {
-                    sp.push_back(CrtSplitItem{p64 + (size_t)m * nb2, o32s + (size_t)m * nb2, oze + (size_t)m * nb, ozplane});
-                    tj.push_back(OzJob{m, k, p64 + (size_t)m * nb2});
+                    spl.push_back(CrtSplitItem{p64 + (size_t)m * nb2, o32s + (size_t)m * nb2, e32 + (size_t)m * nb, plane});
+                    tj.push_back(CrtJob{m, k, p64 + (size_t)m * nb2});
                 }
-                CrtSplitItem* dsp = ar.push(sp);
-                const int nsp = (int)sp.size();
+                CrtSplitItem* dsp = ar.push(spl);
+                const int nsp = (int)spl.size();
                 cur->push_back({[=](cudaStream_t s) { return crt_split_launch(dsp, nsp, nb, crtc32, s); }, C_TRSM, 0});
-                OzJob* dj = ar.push(tj);
+                CrtJob* dj = ar.push(tj);
                 const int nj = (int)tj.size();
-                CrtArgs ca{dj, o32s, oze, ozplane, nb, nt, 0, crt_scr, crt_flags, crtc32, p64b, (uint64_t)2 * nt * nb,
-                           pan_pairs, 0, 1, next_ctr()};
+                const CrtArgs ca = crt_args(dj, o32s, e32, 0, crtc32, p64b, (uint64_t)RG.p64_sets * nt * nb, pan_pairs, 1);
                 cur->push_back({[=](cudaStream_t s) { return crt_gemm_launch(ca, nj, s); }, C_TRSM, 2.0 * fnb * fnb * fnb * nj});
             }
             fc.trsm += np * fnb * fnb * fnb;
-            // ---- 5. panel out (K2)
-            cur->push_back({[=](cudaStream_t s) { return panel_out_launch(d_out, np, (int64_t)nb2, s); }, C_CONV, 0});
-            if (!s16out.empty()) {
-                Split16Item* di = ar.push(s16out);
-                const int ns = (int)s16out.size();
-                cur->push_back({[=](cudaStream_t s) { return split16_launch(di, ns, nb, s); }, C_CONV, 0});
-            }
+            // ---- 5. panel out (K2): storage precision into the pool, comm precision in the panel slot
+            cur->push_back({[=](cudaStream_t s) { return panel_out_launch(d_in, np, (int64_t)nb2, s); }, C_CONV, 0});
         }
+        std::vector<char> have(nt, 0);  // panel slots holding L_mk on this GPU after step 5c
+        for (auto& t : pin) have[(t.p64 - p64) / (ptrdiff_t)nb2] = 1;
         if (dist) {
             // ---- 5b. publish my L_mk (comm precision) for remote successors
             std::vector<PackItem> packs;
@@ -1064,29 +1144,17 @@ static mp_status plan_potrf(mp_handle* h, mp_matrix* A, const uint8_t* km, const
                     cur_push(Op{[=](cudaStream_t s) { return set_flag_launch(fp, v, s); }, C_CONV, 0});
                 }
             }
-            // ---- 5c. pull the remote L_mk my tiles need: peer payload -> FP64 panel slot + caches
+            // ---- 5c. pull the remote L_mk my tiles need: peer payload -> FP64 panel slot
             std::vector<WaitItem> waits;
             std::vector<PullItem> pulls;
-            std::vector<Split16Item> s16pull;
             for (auto& x : xpull[k]) {
                 const int m = x.m;
                 if (m == k) continue;
                 const int o = x.peer;
-                bool n16 = false, n32 = false;
-                local_formats(k, m, n16, n32);
-                PullItem it{sendslot(o, sp, m), pubflag(o, sp, m), ST(k), p64 + (size_t)m * nb2, nullptr, nullptr,
-                            nullptr, C(m, k), 0};
-                if (use_tc && n16) it.p16 = p16 + (size_t)m * nb2;
-                if (use_tc && n32 && !oz32 && !crt32) {
-                    if (f16x3) {
-                        s16pull.push_back(s16item(m));
-                    } else {
-                        it.hi = phi + (size_t)m * nb2;
-                        it.lo = plo + (size_t)m * nb2;
-                    }
-                }
+                PullItem it{sendslot(o, sp, m), pubflag(o, sp, m), ST(k), p64 + (size_t)m * nb2, C(m, k), 0};
                 waits.push_back(WaitItem{it.flag, it.target});
                 pulls.push_back(it);
+                have[m] = 1;
             }
             push_wait(waits);
             if (!pulls.empty()) {
@@ -1094,168 +1162,127 @@ static mp_status plan_potrf(mp_handle* h, mp_matrix* A, const uint8_t* km, const
                 const int npl = (int)pulls.size();
                 cur_push(Op{[=](cudaStream_t s) { return pull_launch(dp, npl, (int64_t)nb2, s); }, C_CONV, 0});
             }
-            if (!s16pull.empty()) {
-                Split16Item* di = ar.push(s16pull);
-                const int ns = (int)s16pull.size();
-                cur_push(Op{[=](cudaStream_t s) { return split16_launch(di, ns, nb, s); }, C_CONV, 0});
-            }
             uint64_t* df = doneflag(me, sp);
             const uint64_t dv = ST(k);
             cur_push(Op{[=](cudaStream_t s) { return set_flag_launch(df, dv, s); }, C_CONV, 0});
         }
-        // ---- 5d. Ozaki: split every panel tile this GPU's FP64-class successors read into int8 slices
-        if (crt) {  // CRT engine: residue planes of every panel tile this GPU's FP64-class successors read
-            std::vector<CrtSplitItem> sp;
+        // ---- 5e. operand formats of panel k for this GPU's successors (single-buffered: they run on
+        //      the update stream after update k-1 released the caches)
+        cur = &fmt[k];
+        {
+            std::vector<Split16Item> s16;
+            std::vector<Tf32Item> t32s;
+            std::vector<CrtSplitItem> c16;
             for (int m = k + 1; m < nt; ++m) {
-                bool need = A->mine(m, m);
-                for (int n = k + 1; n < m && !need; ++n) need |= A->mine(m, n) && K(m, n) == MP_FP64;
-                for (int n = m + 1; n < nt && !need; ++n) need |= A->mine(n, m) && K(n, m) == MP_FP64;
-                if (need)
-                    sp.push_back(CrtSplitItem{p64 + (size_t)m * nb2, ozs + (size_t)m * nb2, oze + (size_t)m * nb, ozplane});
+                if (!have[m]) continue;
+                bool n16, n32, n64;
+                needs(k, m, n16, n32, n64);
+                const double* src = p64 + (size_t)m * nb2;
+                const bool lo3 = n32 && E.f32 == MP_F32_3XFP16;
+                if (E.h16 && (lo3 || (n16 && E.tc16)))
+                    s16.push_back(Split16Item{src, h16hi + (size_t)m * nb2, lo3 ? h16lo + (size_t)m * nb2 : nullptr,
+                                              e16 + (size_t)m * nb});
+                if (n32 && E.f32 == MP_F32_3XTF32) t32s.push_back(Tf32Item{src, phi + (size_t)m * nb2, plo + (size_t)m * nb2});
+                if (n64 && E.crt) c16.push_back(CrtSplitItem{src, ozs + (size_t)m * nb2, oze + (size_t)m * nb, plane});
             }
-            if (!sp.empty()) {
-                CrtSplitItem* dsp = ar.push(sp);
-                const int nsp = (int)sp.size();
+            if (!s16.empty()) {
+                Split16Item* di = ar.push(s16);
+                const int ns = (int)s16.size();
+                cur_push(Op{[=](cudaStream_t s) { return split16_launch(di, ns, nb, s); }, C_CONV, 0});
+            }
+            if (!t32s.empty()) {
+                Tf32Item* di = ar.push(t32s);
+                const int ns = (int)t32s.size();
+                cur_push(Op{[=](cudaStream_t s) { return tf32_split_launch(di, ns, (int64_t)nb2, s); }, C_CONV, 0});
+            }
+            if (!c16.empty()) {
+                CrtSplitItem* dsp = ar.push(c16);
+                const int nsp = (int)c16.size();
                 cur_push(Op{[=](cudaStream_t s) { return crt_split_launch(dsp, nsp, nb, crtc, s); }, C_CONV, 0});
-            }
-        }
-        if (crt32) {  // CRT-8 residue planes of every panel tile this GPU's FP32-class GEMMs read
-            std::vector<CrtSplitItem> sp;
-            int8_t* const o32s = oz32b + set * nt * nb2 * 8;
-            for (int m = k + 1; m < nt; ++m) {
-                bool need = false;
-                for (int n = k + 1; n < m && !need; ++n) need |= A->mine(m, n) && K(m, n) == MP_FP32;
-                for (int n = m + 1; n < nt && !need; ++n) need |= A->mine(n, m) && K(n, m) == MP_FP32;
-                // the row exponents are the same function of the panel tile as the 16-modulus split's
-                if (need)
-                    sp.push_back(CrtSplitItem{p64 + (size_t)m * nb2, o32s + (size_t)m * nb2, oze + (size_t)m * nb, ozplane});
-            }
-            if (!sp.empty()) {
-                CrtSplitItem* dsp = ar.push(sp);
-                const int nsp = (int)sp.size();
-                cur_push(Op{[=](cudaStream_t s) { return crt_split_launch(dsp, nsp, nb, crtc32, s); }, C_CONV, 0});
-            }
-        }
-        if (ozS) {
-            std::vector<OzSplitItem> sp;
-            for (int m = k + 1; m < nt; ++m) {
-                bool need = A->mine(m, m);
-                auto int8_class = [&](int p) { return p == MP_FP64 || (oz32 && p == MP_FP32); };
-                for (int n = k + 1; n < m && !need; ++n) need |= A->mine(m, n) && int8_class(K(m, n));
-                for (int n = m + 1; n < nt && !need; ++n) need |= A->mine(n, m) && int8_class(K(n, m));
-                if (need)
-                    sp.push_back(OzSplitItem{p64 + (size_t)m * nb2, ozs + (size_t)m * nb2, oze + (size_t)m * nb, ozplane});
-            }
-            if (!sp.empty()) {
-                OzSplitItem* dsp = ar.push(sp);
-                const int nsp = (int)sp.size();
-                cur_push(Op{[=](cudaStream_t s) { return ozaki_split_launch(dsp, nsp, nb, ozS, s); }, C_CONV, 0});
             }
         }
         // ---- 6. trailing update: SYRK + GEMM grouped by kernel(m,n); the tiles of
         //      column k+1 (next) are emitted separately so panel k+1 can start as soon as they are done
         for (int part = 0; part < 2; ++part) {
-        cur = part == 0 ? &nxt[k] : &rst[k];
-        std::vector<GemmJob> syrk, g64, g32, g16;
-        std::vector<TcJob> t32, t16;
-        std::vector<OzJob> o32, c32;
-        for (int m = k + 1; m < nt; ++m) {
-            if (A->mine(m, m) && ((m == k + 1) == (part == 0))) {
-                syrk.push_back(GemmJob{p64 + (size_t)m * nb2, p64 + (size_t)m * nb2, A->tile(m, m)});
-                fc.upd[MP_FP64] += fnb * fnb * fnb;
+            cur = part == 0 ? &nxt[k] : &rst[k];
+            std::vector<GemmJob> syrk, g64, g32, g16;
+            std::vector<CrtJob> csyrk, c64;
+            std::vector<TcJob> t32, t16;
+            for (int m = k + 1; m < nt; ++m) {
+                if (A->mine(m, m) && ((m == k + 1) == (part == 0))) {
+                    if (E.crt) csyrk.push_back(CrtJob{m, m, A->tile(m, m)});
+                    else syrk.push_back(GemmJob{p64 + (size_t)m * nb2, p64 + (size_t)m * nb2, A->tile(m, m)});
+                    fc.upd[MP_FP64] += fnb * fnb * fnb;
+                }
+                for (int n = k + 1; n < m; ++n) {
+                    if (!A->mine(m, n) || ((n == k + 1) != (part == 0))) continue;
+                    const int p = K(m, n);
+                    fc.upd[p] += 2.0 * fnb * fnb * fnb;
+                    if (p == MP_FP64) {
+                        if (E.crt) c64.push_back(CrtJob{m, n, A->tile(m, n)});
+                        else g64.push_back(GemmJob{p64 + (size_t)m * nb2, p64 + (size_t)n * nb2, A->tile(m, n)});
+                    } else if (p == MP_FP32 ? E.f32 != MP_F32_DMMA : E.tc16) {
+                        (p == MP_FP32 ? t32 : t16).push_back(TcJob{m, n, (float*)A->tile(m, n)});
+                    } else {
+                        (p == MP_FP32 ? g32 : g16).push_back(GemmJob{p64 + (size_t)m * nb2, p64 + (size_t)n * nb2, A->tile(m, n)});
+                    }
+                }
             }
-            for (int n = k + 1; n < m; ++n) {
-                if (!A->mine(m, n) || ((n == k + 1) != (part == 0))) continue;
-                const int p = K(m, n);
-                fc.upd[p] += 2.0 * fnb * fnb * fnb;
-                if (p == MP_FP64) {
-                    g64.push_back(GemmJob{p64 + (size_t)m * nb2, p64 + (size_t)n * nb2, A->tile(m, n)});
-                } else if (oz32 && p == MP_FP32) {
-                    o32.push_back(OzJob{m, n, A->tile(m, n)});
-                } else if (crt32 && p == MP_FP32) {
-                    c32.push_back(OzJob{m, n, A->tile(m, n)});
-                } else if (use_tc) {
-                    (p == MP_FP32 ? t32 : t16).push_back(TcJob{m, n, (float*)A->tile(m, n)});
+            const double f3 = fnb * fnb * fnb;
+            for (int lower = 1; lower >= 0; --lower) {  // FP64 class on INT8 tensor cores (CRT)
+                std::vector<CrtJob>& cj = lower ? csyrk : c64;
+                if (cj.empty()) continue;
+                CrtJob* dj = ar.push(cj);
+                const int nj = (int)cj.size();
+                // upd_pairs of the SM/2 CTA pairs: SMs stay free for the panel stream's POTRF/TRSM (lookahead)
+                const CrtArgs ca = crt_args(dj, ozs, oze, lower, crtc, cpool64, crows64, upd_pairs, 0);
+                cur_push(Op{[=](cudaStream_t s) { return crt_gemm_launch(ca, nj, s); }, C_UPD64, (lower ? f3 : 2 * f3) * nj});
+            }
+            gemm(syrk, nb, nb, nb, nb, nb, nb, 1, -1.0, 1.0, P64, false, C_UPD64, f3);
+            gemm(g64, nb, nb, nb, nb, nb, nb, 0, -1.0, 1.0, P64, false, C_UPD64, 2 * f3);
+            gemm(g32, nb, nb, nb, nb, nb, nb, 0, -1.0, 1.0, P32, true, C_UPD32, 2 * f3);
+            gemm(g16, nb, nb, nb, nb, nb, nb, 0, -1.0, 1.0, P16, true, C_UPD16, 2 * f3);
+            if (!t32.empty()) {
+                TcJob* dj = ar.push(t32);
+                const int nj = (int)t32.size();
+                TcArgs ta{};
+                ta.jobs = dj;
+                ta.nb = nb;
+                ta.nt = nt;
+                ta.cbase = cpool;
+                ta.crows = crows;
+                if (E.f32 == MP_F32_3XFP16) {
+                    ta.h16hi = h16hi;
+                    ta.h16lo = h16lo;
+                    ta.e16 = e16;
+                    ta.persistent = h->cfg.f16x3_persistent;
+                    ta.pairs = upd_pairs;  // lookahead: leave SMs to the panel stream (0: all)
+                    cur->push_back({[=](cudaStream_t s) { return tc_gemm_f16x3_launch(ta, nj, s); }, C_UPD32, 2 * f3 * nj});
                 } else {
-                    (p == MP_FP32 ? g32 : g16).push_back(GemmJob{p64 + (size_t)m * nb2, p64 + (size_t)n * nb2, A->tile(m, n)});
+                    ta.hi = phi;
+                    ta.lo = plo;
+                    cur->push_back({[=](cudaStream_t s) { return tc_gemm_tf32x3_launch(ta, nj, s); }, C_UPD32, 2 * f3 * nj});
                 }
             }
-        }
-        const double f3 = fnb * fnb * fnb;
-        if (ozS || crt) {  // FP64 class on INT8 tensor cores
-            for (int lower = 1; lower >= 0; --lower) {
-                std::vector<OzJob> oj;
-                for (auto& g : (lower ? syrk : g64)) {
-                    const int mm = (int)(((const double*)g.A - p64) / (ptrdiff_t)nb2);
-                    const int nn = (int)(((const double*)g.B - p64) / (ptrdiff_t)nb2);
-                    oj.push_back(OzJob{mm, nn, (double*)g.C});
-                }
-                if (oj.empty()) continue;
-                OzJob* dj = ar.push(oj);
-                const int nj = (int)oj.size();
-                if (crt) {
-                    // upd_pairs of the SM/2 CTA pairs: SMs stay free for the panel stream's POTRF/TRSM (lookahead)
-                    CrtArgs ca{dj, ozs, oze, ozplane, nb, nt, lower, crt_scr, crt_flags, crtc, cpool64, crows64, upd_pairs, 0, 0,
-                               next_ctr()};
-                    cur_push(Op{[=](cudaStream_t s) { return crt_gemm_launch(ca, nj, s); }, C_UPD64,
-                                (lower ? f3 : 2 * f3) * nj});
-                } else {
-                    OzArgs oa{dj, ozs, oze, ozplane, nb, nt, ozS, lower, 0};
-                    cur_push(Op{[=](cudaStream_t s) { return ozaki_gemm_launch(oa, nj, s); }, C_UPD64,
-                                (lower ? f3 : 2 * f3) * nj});
-                }
+            if (!t16.empty()) {
+                TcJob* dj = ar.push(t16);
+                const int nj = (int)t16.size();
+                TcArgs ta{};
+                ta.jobs = dj;
+                ta.nb = nb;
+                ta.nt = nt;
+                ta.h16hi = h16hi;
+                ta.e16 = e16;
+                ta.cbase = cpool;
+                ta.crows = crows;
+                cur->push_back({[=](cudaStream_t s) { return tc_gemm_f16_launch(ta, nj, s); }, C_UPD16, 2 * f3 * nj});
             }
-            syrk.clear();
-            g64.clear();
-        }
-        gemm(syrk, nb, nb, nb, nb, nb, nb, 1, -1.0, 1.0, P64, false, C_UPD64, f3);
-        gemm(g64, nb, nb, nb, nb, nb, nb, 0, -1.0, 1.0, P64, false, C_UPD64, 2 * f3);
-        gemm(g32, nb, nb, nb, nb, nb, nb, 0, -1.0, 1.0, P32, true, C_UPD32, 2 * f3);
-        gemm(g16, nb, nb, nb, nb, nb, nb, 0, -1.0, 1.0, P16, true, C_UPD16, 2 * f3);
-        if (!o32.empty()) {  // FP32 class on INT8 tensor cores: 4 slices, FP32 C tiles
-            OzJob* dj = ar.push(o32);
-            const int nj = (int)o32.size();
-            OzArgs oa{dj, ozs, oze, ozplane, nb, nt, 4, 0, 1};
-            cur_push(Op{[=](cudaStream_t s) { return ozaki_gemm_launch(oa, nj, s); }, C_UPD32, 2 * f3 * nj});
-        }
-        if (!c32.empty()) {  // FP32 class as 8 INT8 GEMMs (CRT-8), FP32 C
-            OzJob* dj = ar.push(c32);
-            const int nj = (int)c32.size();
-            int8_t* const o32s = oz32b + set * nt * nb2 * 8;
-            CrtArgs ca{dj, o32s, oze, ozplane, nb, nt, 0, crt_scr, crt_flags, crtc32, cpool, crows, upd_pairs, 1, 0, next_ctr()};
-            cur_push(Op{[=](cudaStream_t s) { return crt_gemm_launch(ca, nj, s); }, C_UPD32, 2 * f3 * nj});
-        }
-        if (!t32.empty()) {
-            TcJob* dj = ar.push(t32);
-            const int nj = (int)t32.size();
-            TcArgs ta{dj, phi, plo, nb, nt};
-            ta.cbase = cpool;
-            ta.crows = crows;
-            if (f16x3) {
-                ta.h16hi = (const __half*)phi;
-                ta.h16lo = (const __half*)phi + (size_t)nt * nb2;
-                ta.e16 = (const int*)plo;
-                ta.pairs = upd_pairs;  // lookahead: leave SMs to the panel stream (0: all)
-                cur->push_back({[=](cudaStream_t s) { return tc_gemm_f16x3_launch(ta, nj, s); }, C_UPD32, 2 * f3 * nj});
-            } else {
-                cur->push_back({[=](cudaStream_t s) { return tc_gemm_tf32x3_launch(ta, nj, s); }, C_UPD32, 2 * f3 * nj});
-            }
-        }
-        if (!t16.empty()) {
-            TcJob* dj = ar.push(t16);
-            const int nj = (int)t16.size();
-            TcArgs ta{dj, nullptr, nullptr, nb, nt};
-            ta.p16 = p16;
-            ta.cbase = cpool;
-            ta.crows = crows;
-            cur->push_back({[=](cudaStream_t s) { return tc_gemm_f16_launch(ta, nj, s); }, C_UPD16, 2 * f3 * nj});
-        }
         }  // part
     }
     // ---- assemble the schedule
     if (!la) {
         for (int k = 0; k < nt; ++k)
-            for (auto* v : {&pan[k], &nxt[k], &rst[k]})
+            for (auto* v : {&pan[k], &fmt[k], &nxt[k], &rst[k]})
                 for (auto& o : *v) ops.push_back(std::move(o));
         return MP_OK;
     }
@@ -1272,6 +1299,7 @@ static mp_status plan_potrf(mp_handle* h, mp_matrix* A, const uint8_t* km, const
     ops.push_back(op_record(1, 1));
     for (int k = 0; k + 1 < nt; ++k) {
         ops.push_back(op_wait(0, 1 + 2 * k));
+        on(fmt[k], 0);  // panel k's operand formats: the caches were released by update k-1
         on(nxt[k], 0);
         ops.push_back(op_record(0, 2 + 2 * k));
         ops.push_back(op_wait(1, 2 + 2 * k));
@@ -1551,13 +1579,9 @@ mp_status mp_gp_sample(mp_handle* h, const mp_matrix* Lc, const double* d_e, dou
         const double* yk = ye + (size_t)k * nb;
         ops.push_back({[=](cudaStream_t s) { return gemv_sub_launch(dg, ng, yk, nb, s); }, C_SOLVE, 0});
     }
+    // r = -(L e): negated into d_z on the device
+    ops.push_back({[=](cudaStream_t s) { return scale_vec_launch(d_z, r, n, -1.0, s); }, C_SOLVE, 0});
     if (mp_status st = run_plan(h, A, ar, ops)) return st;
-    // r = -(L e): copy out negated
-    std::vector<double> tmp(n);
-    CK(h, cudaMemcpyAsync(tmp.data(), r, (size_t)n * 8, cudaMemcpyDeviceToHost, h->stream));
-    CK(h, cudaStreamSynchronize(h->stream));
-    for (auto& v : tmp) v = -v;
-    CK(h, cudaMemcpyAsync(d_z, tmp.data(), (size_t)n * 8, cudaMemcpyHostToDevice, h->stream));
     CK(h, cudaStreamSynchronize(h->stream));
     return MP_OK;
 }
@@ -1581,7 +1605,7 @@ mp_status mp_eval(mp_handle* h, mp_matrix* A, const double* x, const double* y, 
                   const double theta[3], double u_req, const double* eps, mp_comm_policy policy, mp_map_mode mode,
                   const uint8_t* user_kernel_prec, mp_eval_report* rep) {
     if (!h || !A || !x || !y || !z || !rep) return MP_ERR_ARG;
-    if (!A->bound) FAIL(h, MP_ERR_STATE, "bind a worst-case workspace (mp_matrix_bytes with NULL) first");
+    if (!A->bound) FAIL(h, MP_ERR_STATE, "bind or attach a workspace first (mp_matrix_bind / mp_matrix_attach)");
     if (mp_status s = check_theta(h, theta, A->cov)) return s;
     memset(rep, 0, sizeof *rep);
     const int nt = A->nt;
@@ -1633,6 +1657,11 @@ mp_status mp_eval(mp_handle* h, mp_matrix* A, const double* x, const double* y, 
             return MP_ERR_ARG;
     }
     if (st) FAIL(h, st, "precision map failed");
+    {  // the workspace this map needs (tiles in storage precision + the map-independent regions)
+        const size_t need = layout(A, sm.data()).total;
+        rep->workspace_bytes = need;
+        if (need > wsb) FAIL(h, MP_ERR_NOMEM, "workspace %zu bytes < %zu needed by this evaluation's map", wsb, need);
+    }
     if (mp_status b = mp_matrix_bind(A, sm.data(), ws, wsb)) return b;
     if (mp_status g = mp_matern_gen(h, A, dx, dy, theta, sm.data(), nullptr)) return g;
     CK(h, cudaEventRecord(ev[2], h->stream));

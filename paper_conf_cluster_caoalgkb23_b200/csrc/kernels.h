@@ -69,24 +69,28 @@ cudaError_t bessel_k_launch(double nu, const double* x, double* out, int n, cuda
 struct PanelTile {
     void* store;      // the tile in the pool (storage precision)
     double* p64;      // FP64 panel slot
-    __half* p16;      // FP16 copy (or null)
-    float* hi;        // TF32 hi (or null)
-    float* lo;        // TF32 lo (or null)
     int store_prec;   // P64 / P32
     int comm_prec;    // precision the tile is sent at (P64 / P32 / P16)
 };
-// 3xFP16 FP32-class operands of one FP64 panel tile (split16_kernel, convert.cu)
+struct Tf32Item {     // 3xTF32 operands of one panel tile (FP32 class with MP_F32_3XTF32)
+    const double* src;
+    float* hi;
+    float* lo;
+};
+// Row-scaled FP16 operands of one FP64 panel tile (split16_kernel, convert.cu)
 struct Split16Item {
     const double* src;  // FP64 panel slot (nb x nb)
-    __half* hi;         // row-scaled FP16 hi / lo (nb x nb)
+    __half* hi;         // row-scaled FP16 hi / lo (nb x nb); lo may be null (FP16 class only)
     __half* lo;
     int* exps;          // [nb]: 2^exps undoes row i's scale
 };
 cudaError_t split16_launch(const Split16Item* items, int n, int nb, cudaStream_t s);
 // p64 = (double) store
 cudaError_t panel_in_launch(const PanelTile* t, int ntiles, int64_t elems, cudaStream_t s);
-// store = round(p64, store_prec); p64 = round(p64, comm_prec); p16/hi/lo = conversions of p64
+// store = round(p64, store_prec); p64 = round(p64, comm_prec)
 cudaError_t panel_out_launch(const PanelTile* t, int ntiles, int64_t elems, cudaStream_t s);
+// hi/lo = 3xTF32 split of fp32(src)
+cudaError_t tf32_split_launch(const Tf32Item* t, int ntiles, int64_t elems, cudaStream_t s);
 // dst = round(src, prec) elementwise on FP64 arrays
 cudaError_t round_copy_launch(const double* src, double* dst, int64_t elems, int prec, cudaStream_t s);
 // zero the strictly upper triangle of an nb x nb row-major tile
@@ -112,6 +116,8 @@ cudaError_t gemv_sub_launch(const GemvTile* t, int ntiles, const double* y, int 
 // per diagonal tile k: out[k] = sum_{i < nreal_k} log L_kk[i][i]
 cudaError_t logdiag_launch(const double* const* diag_tiles, const int* nreal, int ntiles, int nb,
                            double* out, cudaStream_t s);
+// dst[i] = a * src[i]
+cudaError_t scale_vec_launch(double* dst, const double* src, int64_t n, double a, cudaStream_t s);
 // out[b] = sum of squares of v[b*chunk .. min(n, (b+1)*chunk))
 cudaError_t sumsq_chunks_launch(const double* v, int64_t n, int chunk, double* out, cudaStream_t s);
 

@@ -5,6 +5,8 @@
 // bit-reproducible run to run.
 #include <math.h>
 
+#include <algorithm>
+
 #include "common.cuh"
 #include "kernels.h"
 
@@ -184,6 +186,17 @@ cudaError_t logdiag_launch(const double* const* diag_tiles, const int* nreal, in
                            cudaStream_t s) {
     if (ntiles <= 0) return cudaSuccess;
     logdiag_kernel<<<ntiles, 256, 0, s>>>(diag_tiles, nreal, nb, out);
+    return cudaGetLastError();
+}
+
+__global__ void scale_vec_kernel(double* dst, const double* src, int64_t n, double a) {
+    const int64_t stride = (int64_t)gridDim.x * blockDim.x;
+    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += stride) dst[i] = a * src[i];
+}
+
+cudaError_t scale_vec_launch(double* dst, const double* src, int64_t n, double a, cudaStream_t s) {
+    if (n <= 0) return cudaSuccess;
+    scale_vec_kernel<<<(unsigned)std::min<int64_t>((n + 255) / 256, 1184), 256, 0, s>>>(dst, src, n, a);
     return cudaGetLastError();
 }
 

@@ -13,7 +13,9 @@
 //   warps 4-..       epilogue: tcgen05.ld 32x32b (warp w reads TMEM lanes 32(w%4)..+31 = its rows),
 //                    -acc staged in shared memory (128-byte swizzle) and reduced into C with
 //                    cp.reduce.async.bulk.tensor .add (one add per element: RN(C - acc)).
-// KIND 0 (FP16 class, "FP16_32"): kind::f16, BK = 64, 96 KB of stages so two CTAs share an SM.
+// KIND 0 (FP16 class, "FP16_32"): kind::f16, BK = 64, 96 KB of stages so two CTAs share an SM;
+//   the operands are the row-scaled FP16 hi planes of the 3xFP16 split and the epilogue multiplies
+//   by 2^(eA_i + eB_j) (exact), so tiny FP16-class entries keep 11 bits relative to their row.
 // KIND 1 (FP32 class, 3xTF32, reading C13): kind::tf32, BK = 32, stages of {A_hi, A_lo, B_hi, B_lo},
 //   8 epilogue warps; per k-step three MMAs lo.hi + hi.lo + hi.hi; K is split in chunks of 64
 //   accumulated in two ping-pong TMEM accumulators and summed by the epilogue in FP32.
@@ -47,7 +49,7 @@ struct __align__(64) TcParams {
     CUtensorMap a, b, a_lo, b_lo, c;
     const TcJob* jobs;
     const float* cbase;
-    const int* exps;  // KIND 2: per panel-cache row, 2^exps undoes the operand scale
+    const int* exps;  // per panel-cache row, 2^exps undoes the operand's power-of-two row scale
     int nb, tiles_n, tiles_per_job;
     int total;        // persistent kernel: pair tiles of the launch
 };
@@ -364,6 +366,8 @@ __global__ void __launch_bounds__(TcThreads<KIND>::N, TcCfg<KIND, CL>::MIN_BLOCK
         const uint32_t tl = ((uint32_t)(q * 32) << 16) + (uint32_t)(half * COLS);
         const uint32_t stg = smem_u32(smem) + (uint32_t)(warp - 4) * 8192u;  // two 4 KB boxes per warp
         if (KIND == 0) {
+            const float ra = __int_as_float((p.exps[rowA + q * 32 + lane] + 127) << 23);
+            const int4* eb = (const int4*)(p.exps + jb.n * p.nb + ccol0);
             mbar_wait(smem_u32(&done_bar), 0);
             tc_fence_after();
 #pragma unroll 1
@@ -378,6 +382,7 @@ __global__ void __launch_bounds__(TcThreads<KIND>::N, TcCfg<KIND, CL>::MIN_BLOCK
                 float v[32];
 #pragma unroll
                 for (int i = 0; i < 32; ++i) v[i] = __uint_as_float(r[i]);
+                scale_group(v, ra, eb + g * 8);  // undo the operands' power-of-two row scales
                 stage_box_neg(buf, lane, v);
                 if (lane == 0) tma_reduce_add(&p.c, buf, ccol0 + g * 32, crow0);
             }
@@ -639,19 +644,11 @@ static int tc_sm_count() {
     }
     return n;
 }
-// MPGEO_TC16X3_PERSIST=1: the persistent 3xFP16 kernel (opt-in).  Measured at C3 (profiles/r01,
+// The persistent 3xFP16 kernel (opt-in, mp_config::f16x3_persistent).  Measured at C3 (profiles/r01,
 // s4_persist_*.json): the FP32-class update drops from 1.88 to 1.27-1.35 s, but the evaluation does
 // not gain (183.6-186.5 vs 187.1 Tflop/s): the GPU runs at its power cap, so the denser kernel
 // lowers the clock for the CRT and FP16 launches, and with reserved pairs the panel stream gets
-// fewer SMs (conversions 0.41 -> 0.85 s).  Default: one CTA pair per output tile.
-static bool tc16x3_persistent() {
-    static const int v = [] {
-        const char* e = getenv("MPGEO_TC16X3_PERSIST");
-        return e ? atoi(e) : 0;
-    }();
-    return v != 0;
-}
-
+// fewer SMs.  Default: one CTA pair per output tile.
 template <int KIND, int CL>
 static cudaError_t launch(const TcArgs& a, int njobs, cudaStream_t s) {
     using Cfg = TcCfg<KIND, CL>;
@@ -669,8 +666,10 @@ static cudaError_t launch(const TcArgs& a, int njobs, cudaStream_t s) {
     constexpr uint32_t BROWS = Cfg::BN / CL;
     bool ok;
     if (KIND == 0) {
-        ok = make_map(&p.a, a.p16, CU_TENSOR_MAP_DATA_TYPE_FLOAT16, 2, rows, a.nb, Cfg::BK, TC_BM) &&
-             make_map(&p.b, a.p16, CU_TENSOR_MAP_DATA_TYPE_FLOAT16, 2, rows, a.nb, Cfg::BK, BROWS);
+        ok = a.h16hi && a.e16 &&
+             make_map(&p.a, a.h16hi, CU_TENSOR_MAP_DATA_TYPE_FLOAT16, 2, rows, a.nb, Cfg::BK, TC_BM) &&
+             make_map(&p.b, a.h16hi, CU_TENSOR_MAP_DATA_TYPE_FLOAT16, 2, rows, a.nb, Cfg::BK, BROWS);
+        p.exps = a.e16;
     } else if (KIND == 2) {
         ok = a.h16hi && a.h16lo && a.e16 &&
              make_map(&p.a, a.h16hi, CU_TENSOR_MAP_DATA_TYPE_FLOAT16, 2, rows, a.nb, Cfg::BK, TC_BM) &&
@@ -696,7 +695,7 @@ static cudaError_t launch(const TcArgs& a, int njobs, cudaStream_t s) {
     if (grid > 0x7fffffffLL) return cudaErrorInvalidConfiguration;
     void (*kern)(TcParams) = tc_gemm_kernel<KIND, CL>;
     int smem_bytes = Cfg::SMEM;
-    if (KIND == 2 && CL == 2 && tc16x3_persistent()) {
+    if (KIND == 2 && CL == 2 && a.persistent) {
         static bool pattr = false;
         if (!pattr) {
             cudaError_t e = cudaFuncSetAttribute(tc_f16x3_persistent_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, P16_SMEM);
@@ -704,11 +703,7 @@ static cudaError_t launch(const TcArgs& a, int njobs, cudaStream_t s) {
             pattr = true;
         }
         p.total = (int)(grid / CL);
-        static const int env_pairs = [] {  // MPGEO_TC16X3_PAIRS: override of the pair count
-            const char* e = getenv("MPGEO_TC16X3_PAIRS");
-            return e ? atoi(e) : 0;
-        }();
-        int pairs = env_pairs > 0 ? env_pairs : a.pairs > 0 ? a.pairs : tc_sm_count() / 2;
+        int pairs = a.pairs > 0 ? a.pairs : tc_sm_count() / 2;
         if (pairs > p.total) pairs = p.total;
         grid = (long long)pairs * CL;
         kern = tc_f16x3_persistent_kernel;
@@ -729,21 +724,9 @@ static cudaError_t launch(const TcArgs& a, int njobs, cudaStream_t s) {
     return cudaLaunchKernelEx(&cfg, kern, p);
 }
 
-// CTAs per MMA: MPGEO_TC_CLUSTER (3xTF32) and MPGEO_TC16_CLUSTER (FP16); default 2 = CTA pairs (faster
-// than single-CTA for both kinds, profiles/r01/README.md)
-static int env_cluster(const char* name, int dflt) {
-    const char* e = getenv(name);
-    return e ? (atoi(e) == 2 ? 2 : 1) : dflt;
-}
-
-cudaError_t tc_gemm_f16_launch(const TcArgs& a, int njobs, cudaStream_t s) {
-    static const int cl = env_cluster("MPGEO_TC16_CLUSTER", 2);
-    return cl == 2 ? launch<0, 2>(a, njobs, s) : launch<0, 1>(a, njobs, s);
-}
+// CTA pairs (cta_group::2) for every kind: faster than single CTAs for both (profiles/r01/README.md)
+cudaError_t tc_gemm_f16_launch(const TcArgs& a, int njobs, cudaStream_t s) { return launch<0, 2>(a, njobs, s); }
 cudaError_t tc_gemm_f16x3_launch(const TcArgs& a, int njobs, cudaStream_t s) { return launch<2, 2>(a, njobs, s); }
-cudaError_t tc_gemm_tf32x3_launch(const TcArgs& a, int njobs, cudaStream_t s) {
-    static const int cl = env_cluster("MPGEO_TC_CLUSTER", 2);
-    return cl == 2 ? launch<1, 2>(a, njobs, s) : launch<1, 1>(a, njobs, s);
-}
+cudaError_t tc_gemm_tf32x3_launch(const TcArgs& a, int njobs, cudaStream_t s) { return launch<1, 2>(a, njobs, s); }
 
 }  // namespace mpgeo

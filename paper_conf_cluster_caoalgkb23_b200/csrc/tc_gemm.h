@@ -1,6 +1,8 @@
 // K6 / K7 — tcgen05 tensor-core GEMMs for the trailing update of FP32-class and FP16-class tiles
 // (GEMM(m,n,k) at kernel(m,n)):   C_mn (FP32 tile) -= L_mk L_nk^T
-//   FP16 class  (the paper's FP16_32): FP16 operands, FP32 accumulation in TMEM (kind::f16);
+//   FP16 class  (the paper's FP16_32): FP16 operands, FP32 accumulation in TMEM (kind::f16); the
+//                operands are the row-scaled FP16 hi planes of the 3xFP16 split (x = 2^e hi up to
+//                FP16 rounding), so FP16-class entries far below 2^-14 do not underflow;
 //   FP32 class : 3xTF32 — hi = rna_tf32(a), lo = rna_tf32(a - hi), C -= hi.hi + hi.lo + lo.hi with
 //                an FP32 TMEM accumulator (kind::tf32), reading C13 in DESIGN.md.
 // Operands are the consumer-side conversions of the panel (K2), stored as [nt*nb][nb] row-major
@@ -20,13 +22,14 @@ struct TcArgs {
     const float* hi;      // TF32 hi panel cache, [nt * nb][nb]
     const float* lo;      // TF32 lo panel cache
     int nb, nt;
-    const __half* p16;    // FP16 panel cache, [nt * nb][nb]
-    // 3xFP16 FP32-class operands (tc_gemm_f16x3_launch): row-scaled FP16 hi / lo panel caches
-    // [nt * nb][nb] and the per-row exponents e (x = 2^e (hi + lo) up to the split error)
+    // row-scaled FP16 hi / lo panel caches [nt * nb][nb] (split16_kernel) and the per-row exponents e
+    // (x = 2^e (hi + lo) up to the split error): hi + lo for the 3xFP16 FP32 class, hi alone for the
+    // FP16 class
     const __half* h16hi = nullptr;
     const __half* h16lo = nullptr;
     const int* e16 = nullptr;
-    int pairs = 0;  // persistent 3xFP16 kernel: CTA pairs to use (0: all SMs / 2)
+    int persistent = 0;  // 3xFP16: persistent CTA-pair kernel (mp_config::f16x3_persistent)
+    int pairs = 0;       // persistent 3xFP16 kernel: CTA pairs to use (0: all SMs / 2)
     // every TcJob::C lies in [cbase, cbase + crows * nb) at a whole row offset (the epilogue
     // reduces into C through one TMA tensor map over this range)
     const float* cbase;

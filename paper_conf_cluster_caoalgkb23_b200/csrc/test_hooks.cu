@@ -3,11 +3,11 @@
 #include <math.h>
 #include <stdio.h>
 #include <stdlib.h>
+#include <algorithm>
 #include <vector>
 
 #include "kernels.h"
 #include "tc_gemm.h"
-#include "ozaki.h"
 #include "crt.h"
 
 using namespace mpgeo;
@@ -46,6 +46,7 @@ mp_status mp_test_dgemm(const double* d_A, const double* d_B, void* d_C, int M, 
 mp_status mp_test_tc_gemm(int kind, const void* d_panel, const void* d_panel_lo, float* d_C, int nb, int nt, int m,
                           int n) {
     if (!tc_gemm_available()) return MP_ERR_UNSUPPORTED;
+    if (kind != 1) return MP_ERR_ARG;  // 3xTF32 only; the FP16 kinds take an FP64 panel (mp_test_tc_gemm_split)
     TcJob j{m, n, d_C};
     TcJob* dj = nullptr;
     if (cudaMalloc(&dj, sizeof j) != cudaSuccess) return MP_ERR_CUDA;
@@ -56,22 +57,18 @@ mp_status mp_test_tc_gemm(int kind, const void* d_panel, const void* d_panel_lo,
     a.nt = nt;
     a.cbase = d_C;
     a.crows = (uint64_t)nb;
-    cudaError_t e;
-    if (kind == 1) {
-        a.hi = (const float*)d_panel;
-        a.lo = (const float*)d_panel_lo;
-        e = tc_gemm_tf32x3_launch(a, 1, 0);
-    } else {
-        a.p16 = (const __half*)d_panel;
-        e = tc_gemm_f16_launch(a, 1, 0);
-    }
+    a.hi = (const float*)d_panel;
+    a.lo = (const float*)d_panel_lo;
+    cudaError_t e = tc_gemm_tf32x3_launch(a, 1, 0);
     cudaError_t e2 = cudaDeviceSynchronize();
     cudaFree(dj);
     return (e == cudaSuccess && e2 == cudaSuccess) ? MP_OK : MP_ERR_CUDA;
 }
 
-mp_status mp_test_tc_gemm_f16x3(const double* d_panel, float* d_C, int nb, int nt, int m, int n) {
+mp_status mp_test_tc_gemm_split(int kind, const double* d_panel, float* d_C, int nb, int nt, int m, int n,
+                                int persistent) {
     if (!tc_gemm_available()) return MP_ERR_UNSUPPORTED;
+    if (kind != 0 && kind != 2) return MP_ERR_ARG;
     const size_t elems = (size_t)nt * nb * nb;
     __half *hi = nullptr, *lo = nullptr;
     int* ex = nullptr;
@@ -85,8 +82,9 @@ mp_status mp_test_tc_gemm_f16x3(const double* d_panel, float* d_C, int nb, int n
     if (e == cudaSuccess) e = cudaMalloc(&dj, sizeof j);
     if (e == cudaSuccess) e = cudaMalloc(&di, nt * sizeof(Split16Item));
     if (e == cudaSuccess) {
-        for (int t = 0; t < nt; ++t)
-            items.push_back({d_panel + (size_t)t * nb * nb, hi + (size_t)t * nb * nb, lo + (size_t)t * nb * nb, ex + (size_t)t * nb});
+        for (int t = 0; t < nt; ++t)  // the FP16 class derives hi only (lo stays untouched)
+            items.push_back({d_panel + (size_t)t * nb * nb, hi + (size_t)t * nb * nb,
+                             kind == 2 ? lo + (size_t)t * nb * nb : nullptr, ex + (size_t)t * nb});
         cudaMemcpy(dj, &j, sizeof j, cudaMemcpyHostToDevice);
         cudaMemcpy(di, items.data(), nt * sizeof(Split16Item), cudaMemcpyHostToDevice);
         e = split16_launch(di, nt, nb, 0);
@@ -101,7 +99,8 @@ mp_status mp_test_tc_gemm_f16x3(const double* d_panel, float* d_C, int nb, int n
         a.e16 = ex;
         a.cbase = d_C;
         a.crows = (uint64_t)nb;
-        e = tc_gemm_f16x3_launch(a, 1, 0);
+        a.persistent = persistent;
+        e = kind == 2 ? tc_gemm_f16x3_launch(a, 1, 0) : tc_gemm_f16_launch(a, 1, 0);
     }
     cudaError_t e2 = cudaDeviceSynchronize();
     cudaFree(hi);
@@ -114,42 +113,9 @@ mp_status mp_test_tc_gemm_f16x3(const double* d_panel, float* d_C, int nb, int n
 
 int mp_tc_available(void) { return tc_gemm_available() ? 1 : 0; }
 
-mp_status mp_test_ozaki_gemm(const double* d_panel, double* d_C, int nb, int nt, int m, int n, int S, int lower) {
-    if (!ozaki_available()) return MP_ERR_UNSUPPORTED;
-    const int64_t plane = (int64_t)nt * nb * nb;
-    int8_t* sl = nullptr;
-    int* ex = nullptr;
-    OzSplitItem* it = nullptr;
-    OzJob* dj = nullptr;
-    if (cudaMalloc(&sl, plane * 8) || cudaMalloc(&ex, sizeof(int) * nt * nb) ||
-        cudaMalloc(&it, sizeof(OzSplitItem) * nt) || cudaMalloc(&dj, sizeof(OzJob)))
-        return MP_ERR_CUDA;
-    std::vector<OzSplitItem> h(nt);
-    for (int t = 0; t < nt; ++t)
-        h[t] = OzSplitItem{d_panel + (size_t)t * nb * nb, sl + (size_t)t * nb * nb, ex + (size_t)t * nb, plane};
-    cudaMemcpy(it, h.data(), sizeof(OzSplitItem) * nt, cudaMemcpyHostToDevice);
-    OzJob j{m, n, d_C};
-    cudaMemcpy(dj, &j, sizeof j, cudaMemcpyHostToDevice);
-    cudaError_t e = ozaki_split_launch(it, nt, nb, 8, 0);  // the cache always holds 8 planes
-    OzArgs a{dj, sl, ex, plane, nb, nt, S, lower, S == 4 ? 1 : 0};  // S = 4: FP32 class, C is float
-    if (e == cudaSuccess) e = ozaki_gemm_launch(a, 1, 0);
-    cudaError_t e2 = cudaDeviceSynchronize();
-    cudaFree(sl);
-    cudaFree(ex);
-    cudaFree(it);
-    cudaFree(dj);
-    return (e == cudaSuccess && e2 == cudaSuccess) ? MP_OK : MP_ERR_CUDA;
-}
-
-mp_status mp_test_crt_gemm(const double* d_panel, void* d_C, int nb, int nt, int m, int n, int nmod, int lower) {
-    // nmod = 8: the FP32-class update instantiation (FP32 C)
-    return mp_test_crt_gemm_ex(d_panel, d_C, nb, nt, m, n, nmod, lower, nmod == 8, 0);
-}
-
-mp_status mp_test_crt_gemm_ex(const double* d_panel, void* d_C, int nb, int nt, int m, int n, int nmod, int lower,
-                              int c_f32, int store) {
+mp_status mp_test_crt_gemm(const double* d_panel, double* d_C, int nb, int nt, int m, int n, int nmod, int lower,
+                           int store) {
     if (!crt_available()) return MP_ERR_UNSUPPORTED;
-    const int f32 = c_f32;
     CrtConst c;
     if (!crt_constants(nmod, nb, &c)) return MP_ERR_ARG;
     const int64_t plane = (int64_t)nt * nb * nb;
@@ -157,11 +123,11 @@ mp_status mp_test_crt_gemm_ex(const double* d_panel, void* d_C, int nb, int nt, 
     int8_t* pl = nullptr;
     int* ex = nullptr;
     CrtSplitItem* it = nullptr;
-    OzJob* dj = nullptr;
+    CrtJob* dj = nullptr;
     uint8_t* scr = nullptr;
     int* flags = nullptr;
     if (cudaMalloc(&pl, plane * nmod) || cudaMalloc(&ex, sizeof(int) * nt * nb) ||
-        cudaMalloc(&it, sizeof(CrtSplitItem) * nt) || cudaMalloc(&dj, sizeof(OzJob)) ||
+        cudaMalloc(&it, sizeof(CrtSplitItem) * nt) || cudaMalloc(&dj, sizeof(CrtJob)) ||
         cudaMalloc(&scr, (size_t)slots * CRT_SLOT_BYTES) || cudaMalloc(&flags, sizeof(int) * (slots + 2)))
         return MP_ERR_CUDA;
     cudaMemset(flags, 0, sizeof(int) * (slots + 2));  // slot flags + the tile counter and phase
@@ -169,22 +135,26 @@ mp_status mp_test_crt_gemm_ex(const double* d_panel, void* d_C, int nb, int nt, 
     for (int t = 0; t < nt; ++t)
         h[t] = CrtSplitItem{d_panel + (size_t)t * nb * nb, pl + (size_t)t * nb * nb, ex + (size_t)t * nb, plane};
     cudaMemcpy(it, h.data(), sizeof(CrtSplitItem) * nt, cudaMemcpyHostToDevice);
-    OzJob j{m, n, d_C};
+    CrtJob j{m, n, d_C};
     cudaMemcpy(dj, &j, sizeof j, cudaMemcpyHostToDevice);
     cudaError_t e = crt_split_launch(it, nt, nb, c, 0);
-    CrtArgs a{dj, pl, ex, plane, nb, nt, lower, scr, flags, c, d_C, (uint64_t)nb, 0, f32, store, flags + slots};
+    CrtArgs a{};
+    a.jobs = dj;
+    a.planes = pl;
+    a.exps = ex;
+    a.plane_stride = plane;
+    a.nb = nb;
+    a.nt = nt;
+    a.lower = lower;
+    a.scratch = scr;
+    a.slot_flags = flags;
+    a.c = c;
+    a.cbase = d_C;
+    a.crows = (uint64_t)nb;
+    a.store = store;
+    a.counter = flags + slots;
     if (e == cudaSuccess) e = crt_gemm_launch(a, 1, 0);
     cudaError_t e2 = cudaDeviceSynchronize();
-    if (const char* path = getenv("MPGEO_CRT_DUMP")) {  // debugging aid: planes, exponents, 8 scratch slots
-        std::vector<char> buf((size_t)plane * nmod + sizeof(int) * nt * nb + 8 * CRT_SLOT_BYTES);
-        cudaMemcpy(buf.data(), pl, (size_t)plane * nmod, cudaMemcpyDeviceToHost);
-        cudaMemcpy(buf.data() + plane * nmod, ex, sizeof(int) * nt * nb, cudaMemcpyDeviceToHost);
-        cudaMemcpy(buf.data() + plane * nmod + sizeof(int) * nt * nb, scr, 8 * CRT_SLOT_BYTES, cudaMemcpyDeviceToHost);
-        if (FILE* f = fopen(path, "wb")) {
-            fwrite(buf.data(), 1, buf.size(), f);
-            fclose(f);
-        }
-    }
     cudaFree(pl);
     cudaFree(ex);
     cudaFree(it);
@@ -195,27 +165,26 @@ mp_status mp_test_crt_gemm_ex(const double* d_panel, void* d_C, int nb, int nt, 
     return (e == cudaSuccess && e2 == cudaSuccess) ? MP_OK : MP_ERR_CUDA;
 }
 
-/* Isolated timing of the FP64-class engines on a batched trailing-update-like launch: a random FP64
- * panel of nt tiles, njobs tile-GEMMs C_j -= P_{m_j} P_{n_j}^T (distinct C tiles), engine 8 (8-slice
- * splitting) or 16 (CRT, nmod moduli).  ms[0] = split of the nt panel tiles, ms[1] = one GEMM launch
- * (mean over reps after one warm-up). */
-mp_status mp_bench_fp64_engine(int engine, int nb, int nt, int njobs, int nmod, int reps, float* ms) {
+/* Isolated timing of the CRT FP64-class engine on a batched trailing-update-like launch: a
+ * deterministic FP64 panel of nt tiles, njobs tile-GEMMs C_j -= P_{m_j} P_{n_j}^T (distinct C tiles)
+ * with nmod moduli.  ms[0] = split of the nt panel tiles, ms[1] = one GEMM launch (mean over reps
+ * after one warm-up). */
+mp_status mp_bench_fp64_engine(int nb, int nt, int njobs, int nmod, int reps, float* ms) {
     const int64_t plane = (int64_t)nt * nb * nb;
-    const int np = engine == 16 ? nmod : 8;
     double *P = nullptr, *Cb = nullptr;
     int8_t* pl = nullptr;
     int* ex = nullptr;
-    void* it = nullptr;
-    OzJob* dj = nullptr;
+    CrtSplitItem* it = nullptr;
+    CrtJob* dj = nullptr;
     uint8_t* scr = nullptr;
     int* flags = nullptr;
     const int slots = crt_scratch_slots();
-    if (cudaMalloc(&P, plane * 8) || cudaMalloc(&Cb, (size_t)njobs * nb * nb * 8) || cudaMalloc(&pl, plane * np) ||
-        cudaMalloc(&ex, sizeof(int) * nt * nb) || cudaMalloc(&it, 64 * nt) || cudaMalloc(&dj, sizeof(OzJob) * njobs) ||
-        cudaMalloc(&scr, (size_t)slots * CRT_SLOT_BYTES) || cudaMalloc(&flags, sizeof(int) * (slots + 2 * (1 + reps))))
+    if (cudaMalloc(&P, plane * 8) || cudaMalloc(&Cb, (size_t)njobs * nb * nb * 8) || cudaMalloc(&pl, plane * nmod) ||
+        cudaMalloc(&ex, sizeof(int) * nt * nb) || cudaMalloc(&it, sizeof(CrtSplitItem) * nt) ||
+        cudaMalloc(&dj, sizeof(CrtJob) * njobs) || cudaMalloc(&scr, (size_t)slots * CRT_SLOT_BYTES) ||
+        cudaMalloc(&flags, sizeof(int) * (slots + 2 * (1 + reps))))
         return MP_ERR_CUDA;
     cudaMemset(flags, 0, sizeof(int) * (slots + 2 * (1 + reps)));  // slot flags + counter pair per launch
-    cudaMemset(P, 0, plane * 8);
     cudaMemset(Cb, 0, (size_t)njobs * nb * nb * 8);
     {   // deterministic non-trivial panel: x = sin(i * 0.37 + j * 0.11) scaled per row
         std::vector<double> h((size_t)nb * nb);
@@ -225,49 +194,40 @@ mp_status mp_bench_fp64_engine(int engine, int nb, int nt, int njobs, int nmod, 
             cudaMemcpy(P + (size_t)t * nb * nb, h.data(), h.size() * 8, cudaMemcpyHostToDevice);
         }
     }
-    std::vector<OzJob> jobs(njobs);
-    const bool same = getenv("MPGEO_BENCH_SAMEJOB") != nullptr;  // every job reads panel tiles (0, 1)
-    for (int j = 0; j < njobs; ++j)
-        jobs[j] = same ? OzJob{0, 1, Cb + (size_t)j * nb * nb} : OzJob{j % nt, (j / nt + j + 1) % nt, Cb + (size_t)j * nb * nb};
-    cudaMemcpy(dj, jobs.data(), sizeof(OzJob) * njobs, cudaMemcpyHostToDevice);
+    std::vector<CrtJob> jobs(njobs);
+    for (int j = 0; j < njobs; ++j) jobs[j] = CrtJob{j % nt, (j / nt + j + 1) % nt, Cb + (size_t)j * nb * nb};
+    cudaMemcpy(dj, jobs.data(), sizeof(CrtJob) * njobs, cudaMemcpyHostToDevice);
     CrtConst c;
-    if (engine == 16 && !crt_constants(nmod, nb, &c)) return MP_ERR_ARG;
-    if (engine == 16) {
-        std::vector<CrtSplitItem> hs(nt);
-        for (int t = 0; t < nt; ++t)
-            hs[t] = CrtSplitItem{P + (size_t)t * nb * nb, pl + (size_t)t * nb * nb, ex + (size_t)t * nb, plane};
-        cudaMemcpy(it, hs.data(), sizeof(CrtSplitItem) * nt, cudaMemcpyHostToDevice);
-    } else {
-        std::vector<OzSplitItem> hs(nt);
-        for (int t = 0; t < nt; ++t)
-            hs[t] = OzSplitItem{P + (size_t)t * nb * nb, pl + (size_t)t * nb * nb, ex + (size_t)t * nb, plane};
-        cudaMemcpy(it, hs.data(), sizeof(OzSplitItem) * nt, cudaMemcpyHostToDevice);
-    }
-    auto split = [&]() {
-        return engine == 16 ? crt_split_launch((const CrtSplitItem*)it, nt, nb, c, 0)
-                            : ozaki_split_launch((const OzSplitItem*)it, nt, nb, 8, 0);
-    };
+    if (!crt_constants(nmod, nb, &c)) return MP_ERR_ARG;
+    std::vector<CrtSplitItem> hs(nt);
+    for (int t = 0; t < nt; ++t) hs[t] = CrtSplitItem{P + (size_t)t * nb * nb, pl + (size_t)t * nb * nb, ex + (size_t)t * nb, plane};
+    cudaMemcpy(it, hs.data(), sizeof(CrtSplitItem) * nt, cudaMemcpyHostToDevice);
     int launch_no = 0;
     auto gemm = [&]() {
-        if (engine == 16) {
-            int* const ctr = flags + slots + 2 * std::min(launch_no++, reps);
-            // nmod = 8: the FP32-class instantiation (FP32 C tiles, 2 nb^2 floats apart)
-            CrtArgs a{dj, pl, ex, plane, nb, nt, 0, scr, flags, c, Cb, (uint64_t)njobs * nb * (nmod == 8 ? 2 : 1), 0,
-                      nmod == 8, 0, ctr};
-            return crt_gemm_launch(a, njobs, 0);
-        }
-        OzArgs a{dj, pl, ex, plane, nb, nt, 8, 0, 0};
-        return ozaki_gemm_launch(a, njobs, 0);
+        CrtArgs a{};
+        a.jobs = dj;
+        a.planes = pl;
+        a.exps = ex;
+        a.plane_stride = plane;
+        a.nb = nb;
+        a.nt = nt;
+        a.scratch = scr;
+        a.slot_flags = flags;
+        a.c = c;
+        a.cbase = Cb;
+        a.crows = (uint64_t)njobs * nb;
+        a.counter = flags + slots + 2 * std::min(launch_no++, reps);
+        return crt_gemm_launch(a, njobs, 0);
     };
     cudaEvent_t e0, e1, e2;
     cudaEventCreate(&e0);
     cudaEventCreate(&e1);
     cudaEventCreate(&e2);
-    cudaError_t e = split();
+    cudaError_t e = crt_split_launch(it, nt, nb, c, 0);
     if (e == cudaSuccess) e = gemm();
     cudaDeviceSynchronize();
     cudaEventRecord(e0, 0);
-    for (int r = 0; r < reps && e == cudaSuccess; ++r) e = split();
+    for (int r = 0; r < reps && e == cudaSuccess; ++r) e = crt_split_launch(it, nt, nb, c, 0);
     cudaEventRecord(e1, 0);
     for (int r = 0; r < reps && e == cudaSuccess; ++r) e = gemm();
     cudaEventRecord(e2, 0);

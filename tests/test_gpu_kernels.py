@@ -87,19 +87,30 @@ def tf32_rna(a32: np.ndarray) -> np.ndarray:
     return b.view(np.float32)
 
 
-def test_tc_gemm_f16(lib):
+@pytest.mark.parametrize("scale", [0.1, 4e-8])
+def test_tc_gemm_f16_class_row_scaled(lib, scale):
+    """FP16 class (P:113 FP16_32): operands are the row-scaled FP16 hi planes, so the
+    product keeps FP16 accuracy (11 bits per operand relative to its row, FP32 accumulation) even for
+    tiles whose entries lie below FP16's smallest normal (scale 4e-8: the C3 FP16-class magnitude,
+    where a plain FP16 conversion underflows to 0-2 bits).  Bound: |err| <= (2^-10 + K 2^-23) |A||B|^T
+    entrywise, against the exact product of the FP32-rounded operands."""
     assert lib.mp_tc_available() == 1
     nb, nt = 512, 3
     rng = np.random.default_rng(3)
-    P = (rng.standard_normal((nt * nb, nb)) * 0.1).astype(np.float16)
-    Cm = rng.standard_normal((nb, nb)).astype(np.float32)
+    P = rng.standard_normal((nt * nb, nb)) * scale * np.exp2(-rng.integers(0, 8, size=(nt * nb, 1)))
+    Cm = (rng.standard_normal((nb, nb)) * scale * scale).astype(np.float32)
     dP, dC = dev(P), dev(Cm)
-    assert lib.mp_test_tc_gemm(2, C.c_void_p(dP.data_ptr()), None, C.c_void_p(dC.data_ptr()), nb, nt, 2, 0) == 0
+    assert lib.mp_test_tc_gemm_split(0, C.c_void_p(dP.data_ptr()), C.c_void_p(dC.data_ptr()), nb, nt, 2, 0, 0) == 0
     got = dC.cpu().numpy().astype(np.float64)
-    Pd = P.astype(np.float64)
-    ref = Cm.astype(np.float64) - Pd[2 * nb:3 * nb] @ Pd[0:nb].T
-    err = np.max(np.abs(got - ref))
-    assert err <= 1e-5 * np.max(np.abs(ref)), err
+    A32 = P.astype(np.float32).astype(np.float64)
+    A, B = A32[2 * nb:3 * nb], A32[0:nb]
+    ref = Cm.astype(np.float64) - A @ B.T
+    bound = (2.0**-10 + nb * 2.0**-23) * (np.abs(A) @ np.abs(B).T) + 2.0**-23 * np.abs(ref)
+    assert np.all(np.abs(got - ref) <= bound), np.max(np.abs(got - ref) / bound)
+    if scale < 1e-4:  # a plain (unscaled) FP16 conversion would lose the product entirely
+        plain = A.astype(np.float16).astype(np.float64) @ B.astype(np.float16).astype(np.float64).T
+        assert np.linalg.norm(plain - A @ B.T) > 0.1 * np.linalg.norm(A @ B.T)
+        assert np.linalg.norm(got - ref) < 1e-2 * np.linalg.norm(A @ B.T)
 
 
 def test_tc_gemm_tf32x3_matches_sgemm_accuracy(lib):
@@ -125,19 +136,23 @@ def test_tc_gemm_tf32x3_matches_sgemm_accuracy(lib):
     assert err_tc < err_1x / 50  # far better than a single TF32 product
 
 
-@pytest.mark.parametrize("spread", [0, 30])
-def test_tc_gemm_f16x3_matches_sgemm_accuracy(lib, spread):
+@pytest.mark.parametrize("nb,spread,colspread,persistent", [(512, 0, 0, 0), (512, 30, 0, 0), (2048, 0, 0, 0),
+                                                              (2048, 30, 30, 0), (2048, 30, 30, 1)])
+def test_tc_gemm_f16x3_matches_sgemm_accuracy(lib, nb, spread, colspread, persistent):
     """Reading C13c pin: 3xFP16 (row-scaled FP16 hi/lo split, kind::f16) error vs the exact product of
-    the FP32-rounded operands <= 2x the SGEMM error on the same inputs, also when row magnitudes
-    spread over 2^-spread .. 1 (the per-row power-of-two scales keep every row inside FP16 range);
-    a zero row gives a zero row of the product."""
-    nb, nt = 512, 2
-    rng = np.random.default_rng(5)
+    the FP32-rounded operands <= 2x the SGEMM error on the same inputs — at the bench tile size
+    nb = 2048 (16 TMEM chunks of K = 128), with row magnitudes spread over 2^-spread .. 1 and, within
+    each row, entries spread over 2^-colspread .. 1 (the large within-row range of Cholesky panel rows;
+    ADVICE r01), also with the persistent kernel; a zero row gives a zero row of the product."""
+    nt = 2
+    rng = np.random.default_rng(5 + nb + spread)
     P = rng.standard_normal((nt * nb, nb)) * np.exp2(-rng.integers(0, spread + 1, size=(nt * nb, 1)))
+    P *= np.exp2(-rng.uniform(0, colspread, size=(1, nb)))
     P[nb + 3] = 0.0
     Cm = np.zeros((nb, nb), np.float32)
     dP, dC = dev(P), dev(Cm)
-    assert lib.mp_test_tc_gemm_f16x3(C.c_void_p(dP.data_ptr()), C.c_void_p(dC.data_ptr()), nb, nt, 1, 0) == 0
+    assert lib.mp_test_tc_gemm_split(2, C.c_void_p(dP.data_ptr()), C.c_void_p(dC.data_ptr()), nb, nt, 1, 0,
+                                     persistent) == 0
     got = -dC.cpu().numpy().astype(np.float64)
     A32 = P.astype(np.float32)
     Ad = A32.astype(np.float64)
@@ -148,76 +163,27 @@ def test_tc_gemm_f16x3_matches_sgemm_accuracy(lib, spread):
     ok = rn > 0
     err_tc = np.max(np.linalg.norm(got - exact, axis=1)[ok] / rn[ok])
     err_sg = np.max(np.linalg.norm(sgemm - exact, axis=1)[ok] / rn[ok])
-    print(f"3xFP16 spread={spread}: row-wise error {err_tc:.3e}, SGEMM {err_sg:.3e}")
+    print(f"3xFP16 nb={nb} spread={spread}/{colspread} persistent={persistent}: row-wise error {err_tc:.3e}, "
+          f"SGEMM {err_sg:.3e}")
     assert err_tc <= 2 * err_sg + 1e-9, (err_tc, err_sg)
     assert np.all(got[3] == 0.0)
     single = (A32[nb:].astype(np.float16).astype(np.float64) @ A32[:nb].astype(np.float16).astype(np.float64).T)
-    if spread == 0:
+    if spread == 0 and colspread == 0:
         assert err_tc < np.max(np.linalg.norm(single - exact, axis=1)[ok] / rn[ok]) / 50
-
-
-@pytest.mark.parametrize("S", [8])
-def test_ozaki_int8_fp64_gemm(lib, S):
-    """FP64 GEMM emulated with int8 slices on tcgen05 kind::i8 vs the exact FP64 product: for S = 8
-    the error stays within a few units of an FP64 GEMM's (|err| <= 8 K u max|a| max|b|)."""
-    nb, nt = 512, 3
-    rng = np.random.default_rng(S)
-    P = rng.standard_normal((nt * nb, nb)) * np.exp(rng.uniform(-3, 3, (nt * nb, 1)))  # row scales vary
-    Cm = rng.standard_normal((nb, nb))
-    dP, dC = dev(P), dev(Cm)
-    assert lib.mp_test_ozaki_gemm(C.c_void_p(dP.data_ptr()), C.c_void_p(dC.data_ptr()), nb, nt, 2, 0, S, 0) == 0
-    got = dC.cpu().numpy()
-    A, B = P[2 * nb:], P[:nb]
-    ref = Cm - A @ B.T
-    scale = np.abs(A).max(axis=1)[:, None] * np.abs(B).max(axis=1)[None, :]
-    err = np.max(np.abs(got - ref) / scale)
-    bound = 8 * nb * 2.0**-53
-    assert err <= bound, (S, err, bound)
-    # lower-only (SYRK) variant leaves strictly-upper 128x64 blocks untouched
-    dC2 = dev(Cm)
-    assert lib.mp_test_ozaki_gemm(C.c_void_p(dP.data_ptr()), C.c_void_p(dC2.data_ptr()), nb, nt, 1, 1, S, 1) == 0
-    got2 = dC2.cpu().numpy()
-    ref2 = Cm - P[nb:2 * nb] @ P[nb:2 * nb].T
-    for bi in range(nb // 128):
-        for bj in range(nb // 64):
-            blk = (slice(bi * 128, (bi + 1) * 128), slice(bj * 64, (bj + 1) * 64))
-            if bj * 64 > bi * 128 + 127:
-                assert np.array_equal(got2[blk], Cm[blk])
-            else:
-                assert np.max(np.abs(got2[blk] - ref2[blk])) <= 1e-9
-
-
-def test_ozaki_int8_fp32_class_gemm(lib):
-    """FP32 class on INT8 tensor cores (first 4 slices = 28 bits, reading C13b): error vs the exact
-    product of the FP32 operands within 2x an SGEMM's on the same inputs (the C13 pin)."""
-    nb, nt = 512, 2
-    rng = np.random.default_rng(11)
-    A32 = (rng.standard_normal((nt * nb, nb)) * np.exp(rng.uniform(-2, 2, (nt * nb, 1)))).astype(np.float32)
-    Cm = np.zeros((nb, nb), np.float32)
-    dP, dC = dev(A32.astype(np.float64)), dev(Cm)
-    assert lib.mp_test_ozaki_gemm(C.c_void_p(dP.data_ptr()), C.c_void_p(dC.data_ptr()), nb, nt, 1, 0, 4, 0) == 0
-    got = -dC.cpu().numpy().astype(np.float64)
-    Ad = A32.astype(np.float64)
-    exact = Ad[nb:] @ Ad[:nb].T
-    sgemm = (A32[nb:] @ A32[:nb].T).astype(np.float64)
-    err = np.linalg.norm(got - exact) / np.linalg.norm(exact)
-    err_sg = np.linalg.norm(sgemm - exact) / np.linalg.norm(exact)
-    assert err <= 2 * err_sg, (err, err_sg)
 
 
 @pytest.mark.parametrize("nb,nt,m,n,nmod", [(512, 3, 2, 0, 16), (4096, 2, 1, 0, 16), (2048, 3, 1, 2, 16)])
 def test_crt_int8_fp64_gemm(lib, nb, nt, m, n, nmod):
     """FP64 GEMM by CRT modular emulation on tcgen05 kind::i8 vs the exact FP64 product: with 16
     moduli the operands keep b = 56 bits (rounded) per row, so |err| <= K 2^-(b+1) max|a_i| max|b_j|
-    + the final FP64 rounding — within the FP64-GEMM bound 8 K u max|a| max|b| used for the splitting
-    engine.  nb = 4096 gives 256 pair tiles for 74 persistent CTA pairs (several tiles per pair, both
+    + the final FP64 rounding — within the FP64-GEMM-level bound 8 K u max|a| max|b|.  nb = 4096 gives 256 pair tiles for 74 persistent CTA pairs (several tiles per pair, both
     accumulator parities, scratch-slot reuse).  Rows of very different scale and an all-zero row."""
     rng = np.random.default_rng(nb + nmod)
     P = rng.standard_normal((nt * nb, nb)) * np.exp(rng.uniform(-3, 3, (nt * nb, 1)))
     P[m * nb + 5] = 0.0
     Cm = rng.standard_normal((nb, nb))
     dP, dC = dev(P), dev(Cm)
-    assert lib.mp_test_crt_gemm(C.c_void_p(dP.data_ptr()), C.c_void_p(dC.data_ptr()), nb, nt, m, n, nmod, 0) == 0
+    assert lib.mp_test_crt_gemm(C.c_void_p(dP.data_ptr()), C.c_void_p(dC.data_ptr()), nb, nt, m, n, nmod, 0, 0) == 0
     got = dC.cpu().numpy()
     A, B = P[m * nb:(m + 1) * nb], P[n * nb:(n + 1) * nb]
     ref = Cm - A @ B.T
@@ -230,32 +196,6 @@ def test_crt_int8_fp64_gemm(lib, nb, nt, m, n, nmod):
     assert np.array_equal(got[5], Cm[5])  # zero row of A: C row untouched
 
 
-@pytest.mark.parametrize("nb,nt,m,n", [(512, 2, 1, 0), (2048, 3, 2, 1), (4096, 2, 0, 1)])
-def test_crt8_fp32_class_gemm(lib, nb, nt, m, n):
-    """FP32 class as CRT-8 (8 moduli, b = 25 operand bits per row at K = 2048, FP32 C reduce-added by
-    the TMA unit): error vs the exact product of the FP32 operands within 2x an SGEMM's on the same
-    inputs (the C13 pin), rows of very different scale; plus the same pin against the FP32 C update."""
-    rng = np.random.default_rng(nb + 8)
-    A32 = (rng.standard_normal((nt * nb, nb)) * np.exp(rng.uniform(-2, 2, (nt * nb, 1)))).astype(np.float32)
-    Cm = (rng.standard_normal((nb, nb)) * 0.01).astype(np.float32)
-    dP, dC = dev(A32.astype(np.float64)), dev(Cm)
-    assert lib.mp_test_crt_gemm(C.c_void_p(dP.data_ptr()), C.c_void_p(dC.data_ptr()), nb, nt, m, n, 8, 0) == 0
-    got = dC.cpu().numpy().astype(np.float64)
-    Ad = A32.astype(np.float64)
-    A, B = Ad[m * nb:(m + 1) * nb], Ad[n * nb:(n + 1) * nb]
-    exact = Cm.astype(np.float64) - A @ B.T
-    sgemm = (Cm - A32[m * nb:(m + 1) * nb] @ A32[n * nb:(n + 1) * nb].T).astype(np.float64)
-    err = np.linalg.norm(got - exact) / np.linalg.norm(exact)
-    err_sg = np.linalg.norm(sgemm - exact) / np.linalg.norm(exact)
-    assert err <= 2 * err_sg, (err, err_sg)
-    # entrywise: the operand rounding is 2^-26 of the row / column max
-    ma = np.abs(A).max(axis=1)[:, None]
-    mb = np.abs(B).max(axis=1)[None, :]
-    # two FP32 roundings: the converted product and the reduce-add
-    ent = np.abs(got - exact) - 2.0**-23 * (np.abs(exact) + np.abs(A @ B.T))
-    assert np.all(ent <= 2 * nb * 2.0**-26 * ma * mb), np.max(ent / (ma * mb))
-
-
 @pytest.mark.parametrize("nmod", [8, 16])
 def test_crt_store_mode_fp64_c(lib, nmod):
     """Store mode (C = P_m P_n^T, the TRSM product X = A_mk W^T with W = L_kk^-1): CRT-8 (the FP32-class
@@ -266,8 +206,7 @@ def test_crt_store_mode_fp64_c(lib, nmod):
     P[n * nb:(n + 1) * nb] = np.tril(P[n * nb:(n + 1) * nb])  # a triangular B operand, like the inverse factor
     Cm = np.full((nb, nb), np.nan)
     dP, dC = dev(P), dev(Cm)
-    assert lib.mp_test_crt_gemm_ex(C.c_void_p(dP.data_ptr()), C.c_void_p(dC.data_ptr()), nb, nt, m, n, nmod, 0, 0,
-                                   1) == 0
+    assert lib.mp_test_crt_gemm(C.c_void_p(dP.data_ptr()), C.c_void_p(dC.data_ptr()), nb, nt, m, n, nmod, 0, 1) == 0
     got = dC.cpu().numpy()
     A, B = P[m * nb:(m + 1) * nb], P[n * nb:(n + 1) * nb]
     ref = A @ B.T
@@ -287,7 +226,7 @@ def test_crt_int8_syrk_lower(lib):
     P = rng.standard_normal((nt * nb, nb))
     Cm = rng.standard_normal((nb, nb))
     dP, dC = dev(P), dev(Cm)
-    assert lib.mp_test_crt_gemm(C.c_void_p(dP.data_ptr()), C.c_void_p(dC.data_ptr()), nb, nt, 1, 1, 16, 1) == 0
+    assert lib.mp_test_crt_gemm(C.c_void_p(dP.data_ptr()), C.c_void_p(dC.data_ptr()), nb, nt, 1, 1, 16, 1, 0) == 0
     got = dC.cpu().numpy()
     A = P[nb:]
     ref = Cm - A @ A.T

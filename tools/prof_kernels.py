@@ -33,29 +33,14 @@ def main(which):
         print("dgemm TF/s", 5 * 2 * M * N * K / (s.elapsed_time(e) / 1e3) / 1e12)
     if which in ("tc", "all"):
         nb, nt = 2048, 4
-        P16 = (torch.randn(nt * nb, nb, device="cuda") * 0.1).half()
+        P = torch.randn(nt * nb, nb, dtype=torch.float64, device="cuda") * 0.1
         Cf = torch.zeros(nb, nb, device="cuda")
         hi = torch.randn(nt * nb, nb, device="cuda")
         lo = torch.randn(nt * nb, nb, device="cuda") * 1e-4
         for _ in range(3):
-            assert lib.mp_test_tc_gemm(2, p(P16), None, p(Cf), nb, nt, 1, 0) == 0
+            assert lib.mp_test_tc_gemm_split(0, p(P), p(Cf), nb, nt, 1, 0, 0) == 0
+            assert lib.mp_test_tc_gemm_split(2, p(P), p(Cf), nb, nt, 1, 0, 0) == 0
             assert lib.mp_test_tc_gemm(1, p(hi), p(lo), p(Cf), nb, nt, 1, 0) == 0
-    if which in ("ozaki", "all"):
-        nb, nt = 2048, 4
-        P = torch.randn(nt * nb, nb, dtype=torch.float64, device="cuda")
-        Cm = torch.zeros(nb, nb, dtype=torch.float64, device="cuda")
-        C32 = torch.zeros(nb, nb, dtype=torch.float32, device="cuda")
-        for _ in range(3):
-            assert lib.mp_test_ozaki_gemm(p(P), p(Cm), nb, nt, 2, 1, 8, 0) == 0
-            assert lib.mp_test_ozaki_gemm(p(P), p(C32), nb, nt, 2, 1, 4, 0) == 0
-        for S, Cx in ((8, Cm), (4, C32)):
-            s, e = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-            s.record()
-            for _ in range(5):
-                lib.mp_test_ozaki_gemm(p(P), p(Cx), nb, nt, 2, 1, S, 0)
-            e.record()
-            torch.cuda.synchronize()
-            print(f"ozaki S={S}: {s.elapsed_time(e) / 5:.3f} ms per call (incl. split of {nt} tiles + malloc)")
     if which in ("tf32err", "all"):
         from tests.test_gpu_kernels import tf32_rna
         for K in (64, 256, 1024, 2048):
