@@ -42,7 +42,9 @@ def test_config3_sampled_generation_and_norms(ev):
     okm, osm, ocm = precision_maps(s, 1e-9)
     low = np.tril(np.ones((nt, nt), bool))
     assert np.array_equal(km[low], okm[low]) and np.array_equal(cm[low], ocm[low])
-    # sampled covariance entries after the storage-precision write
+    # sampled covariance entries after the storage-precision write (workspace sized for this map)
+    if M.bytes_for(sm) > M.nbytes:
+        M.attach(M.bytes_for(sm))
     M.bind(sm)
     M.matern_gen(to_dev(x), to_dev(y), theta, sm)
     rng = np.random.default_rng(5)

@@ -20,7 +20,8 @@ def main():
     z = synth.normal_vector(n, seed=1)
     dx, dy, dz = (torch.from_numpy(v).cuda() for v in (x, y, z))
     ev = mp.Evaluator(n, nb)
-    mode = {"adaptive": mp.MP_MAP_ADAPTIVE, "fp64": mp.MP_MAP_FP64, "band": mp.MP_MAP_BAND}[cfg["map"]]
+    mode = {"adaptive": mp.MP_MAP_ADAPTIVE, "fp64": mp.MP_MAP_FP64, "band": mp.MP_MAP_BAND,
+            "extreme": mp.MP_MAP_EXTREME}[cfg["map"]]
     for _ in range(warm + 1):
         r = ev.eval(dx, dy, dz, cfg["theta"], u_req=1e-9, mode=mode)
     torch.cuda.synchronize()
