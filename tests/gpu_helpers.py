@@ -109,13 +109,17 @@ def mp_backward_check(A, Lhat, L, km, sm, cm, nt, nb, lowp_trsm=True, scaled_fp1
 
 
 def loglik_perturbation_bound(A_dense, z, dA_fro):
-    """First-order bound on |l(A + dA) - l(A)|: 1/2 (||A^-1||_F + ||A^-1 z||^2) ||dA||_F, doubled for the
-    second-order terms (valid while ||A^-1||_2 ||dA|| << 1)."""
+    """Bound on |l(A + dA) - l(A)| given ||dA||_F, valid whenever rho = ||A^-1||_2 ||dA||_F < 1:
+    |log det(A + dA) - log det A| = |sum_i log(1 + mu_i)| <= sum |mu_i| / (1 - rho) <= ||A^-1||_F ||dA||_F / (1 - rho)
+    (mu_i the eigenvalues of A^-1/2 dA A^-1/2) and |z^T (A + dA)^-1 z - z^T A^-1 z| <= ||A^-1 z||^2 ||dA|| / (1 - rho),
+    so |dl| <= 1/2 (||A^-1||_F + ||A^-1 z||^2) ||dA||_F / (1 - rho).  Returns (bound, rho)."""
     import scipy.linalg
     c = scipy.linalg.cho_factor(A_dense, lower=True)
     Ainv = scipy.linalg.cho_solve(c, np.eye(A_dense.shape[0]))
     w = scipy.linalg.cho_solve(c, z)
-    return (np.linalg.norm(Ainv) + float(w @ w)) * dA_fro, float(np.linalg.norm(Ainv, 2))
+    rho = float(np.linalg.norm(Ainv, 2)) * dA_fro
+    bound = 0.5 * (np.linalg.norm(Ainv) + float(w @ w)) * dA_fro / (1.0 - rho) if rho < 1 else float("inf")
+    return bound, rho
 
 
 def residual_tiles(A, L, nt):

@@ -16,12 +16,12 @@ for what in "$@"; do
         > gpurun_out/ncu_launches_c5_summary.md 2>&1 ;;
     crt)
       timeout 1500 ncu --set full --clock-control none --import-source on --kernel-name-base demangled \
-        -k 'regex:crt_gemm_kernel<\(int\)16' -s 21 -c 1 -o gpurun_out/ncu_crt16_c5 -f \
+        -k 'regex:crt_gemm_kernel<\(int\)16' -s 23 -c 1 -o gpurun_out/ncu_crt16_c5 -f \
         python tools/one_eval.py c5 0 > gpurun_out/ncu_crt16_c5.log 2>&1
       python tools/ncu_summary.py gpurun_out/ncu_crt16_c5.ncu-rep > gpurun_out/ncu_crt16_c5_summary.txt 2>&1 ;;
     f16x3)
       timeout 1500 ncu --set full --clock-control none --import-source on --kernel-name-base demangled \
-        -k 'regex:tc_gemm_kernel<\(int\)2' -s 10 -c 1 -o gpurun_out/ncu_f16x3_c5 -f \
+        -k 'regex:tc_gemm_kernel<\(int\)2' -s 11 -c 1 -o gpurun_out/ncu_f16x3_c5 -f \
         python tools/one_eval.py c5 0 > gpurun_out/ncu_f16x3_c5.log 2>&1
       python tools/ncu_summary.py gpurun_out/ncu_f16x3_c5.ncu-rep > gpurun_out/ncu_f16x3_c5_summary.txt 2>&1 ;;
     membound)
