@@ -1,0 +1,31 @@
+#!/bin/bash
+# Batch of bench.py lines for the DESIGN.md studies (one gpurun session).  Each line: name + bench args.
+# Output: gpurun_out/study_<name>.json (+ .err).  Usage: tools/study.sh <set>
+cd "$(dirname "$0")/.."
+mkdir -p gpurun_out
+run() {
+  local name=$1; shift
+  timeout 1500 python bench.py --no-cpu-baseline --no-e2e --steps 2 --warmup 3 "$@" \
+    > gpurun_out/study_$name.json 2> gpurun_out/study_$name.err
+  echo "$name rc=$? $(python -c "import json,sys; d=json.load(open('gpurun_out/study_$name.json')); print(round(d['value'],1), 'Tflop/s', round(d['ms_per_step']/1e3,2), 's', round(d['joules_per_eval'] or 0), 'J', d['loglik'], d['tiles_fp64_fp32_fp16'], 'stc', d['stc_tiles'])" 2>/dev/null)"
+}
+case $1 in
+  conv_c5)
+    run c5_auto --config c5 --policy auto
+    run c5_ttc --config c5 --policy ttc
+    run c5_ext_auto --config c5 --map extreme --policy auto
+    run c5_ext_ttc --config c5 --map extreme --policy ttc ;;
+  c2)
+    for m in adaptive band fp64 extreme; do run c2_${m}_auto --config c2 --map $m --policy auto; done
+    run c2_extreme_ttc --config c2 --map extreme --policy ttc
+    run c2_fp64_dmma --config c2 --map fp64 --engine fp64_engine=1
+    run c2b01_band --config c2 --map band --theta 1,0.1,0.5
+    run c2b01_fp64 --config c2 --map fp64 --theta 1,0.1,0.5
+    run c2b01_adaptive --config c2 --map adaptive --theta 1,0.1,0.5 ;;
+  c3)
+    run c3_adaptive --config c3
+    run c3_fp64_crt --config c3 --map fp64
+    run c3_fp64_dmma --config c3 --map fp64 --engine fp64_engine=1
+    run c3_adaptive_dmma --config c3 --engine fp64_engine=1
+    run c3_nolook --config c3 --engine lookahead=0 ;;
+esac
