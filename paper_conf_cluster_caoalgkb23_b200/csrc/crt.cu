@@ -330,13 +330,12 @@ __device__ __forceinline__ void tile_coords(const CrtParams& p, int t, int& job,
     }
 }
 
-// scratch byte offset of the 16-byte run (modulus pair j, column half h, 32-column chunk c, 8-column
-// group e, CTA row r) holding 8 combined residues R (uint16): a warp's 32 rows of one run are 512
-// contiguous bytes (coalesced stores and loads)
-__device__ __forceinline__ uint32_t scr_off(int j, int h, int c, int e, int r) {
-    return ((uint32_t)(((j * 2 + h) * 4 + c) * 4 + e) * 128u + (uint32_t)r) * 16u;
+// scratch byte offset of the 16-byte run (block b of column half h, CTA row r) holding 8 combined
+// residues R (uint16) of one moduli pair and one 8-column group: a warp's 32 rows of one block are
+// 512 contiguous bytes (coalesced stores and loads)
+__device__ __forceinline__ uint32_t scr_off(int b, int h, int r) {
+    return ((uint32_t)(h * CRT_SCR_BLOCKS + b) * 128u + (uint32_t)r) * 16u;
 }
-constexpr uint32_t SCR_J_STRIDE = 2 * 4 * 4 * 128 * 16;  // bytes between moduli pairs
 
 __device__ __forceinline__ void tmem_ld32_nowait(uint32_t taddr, uint32_t (&r)[32]) {
     asm volatile(
@@ -381,6 +380,10 @@ __global__ void __launch_bounds__(THREADS, 1) crt_gemm_kernel(const __grid_const
     // publishes them in a ring in both CTAs (late-starting pairs simply claim fewer tiles)
     __shared__ int tile_ring[RING];
     __shared__ __align__(8) uint64_t ring_full[RING], ring_empty[RING];
+    // per epilogue warp: scratch block of (moduli pair j, group gi) for the two tiles in flight, and
+    // the 16 blocks the last reconstruction step freed (the next residue step's destinations)
+    __shared__ uint8_t scr_tab[EPI_WARPS][2][CRT_NMAX / 2 * 16];
+    __shared__ uint8_t scr_free[EPI_WARPS][16];
 
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     const uint32_t crank = cluster_rank();
@@ -512,10 +515,12 @@ __global__ void __launch_bounds__(THREADS, 1) crt_gemm_kernel(const __grid_const
         }
     } else if (warp >= 4) {
         // ---------------- epilogue.  Per tile T: for each moduli pair j, reduce modulus a (residues
-        // kept as bytes), reduce modulus b and store the combined residues R_j of T into scratch half
-        // T&1, then reconstruct two of the 16 eight-column groups of tile T-1 (from half (T-1)&1) and
-        // reduce-add them into C — so the reconstruction fills the epilogue's slack while the tensor
-        // core works on T (a tile's reconstruction is ~7x one modulus' MMA time).
+        // kept as bytes), reduce modulus b and store the combined residues R_j of T into 16 scratch
+        // blocks (one per 8-column group), then reconstruct 16/NP of the 16 eight-column groups of
+        // tile T-1 and reduce-add them into C — so the reconstruction fills the epilogue's slack while
+        // the tensor core works on T.  The 16 blocks each reconstruction step frees are the next
+        // residue step's destinations (scr_tab / scr_free): one tile of scratch + 16 spare blocks per
+        // CTA (576 KB) instead of two tiles, so the scratch in flight stays within L2.
         const int q = (warp - 4) & 3, h = (warp - 4) >> 2;
         const int r = q * 32 + lane;  // CTA row = TMEM lane
         uint8_t* const scr0 = p.scratch + (size_t)slot_sh * CRT_SLOT_BYTES;
@@ -527,15 +532,24 @@ __global__ void __launch_bounds__(THREADS, 1) crt_gemm_kernel(const __grid_const
         uint32_t nred = 0;    // C reduce-adds issued by this warp (staging-buffer parity)
         // the previous tile, whose reconstruction is pending
         bool pv = false;
-        int pv_crow0 = 0, pv_ccol0 = 0, pv_half = 0;
+        int pv_crow0 = 0, pv_ccol0 = 0, pv_tab = 0;
         double pv_rs = 0.0;
         const int* pv_ecol = nullptr;
+        const int ew = warp - 4;
+        if (lane < 16) scr_free[ew][lane] = (uint8_t)(NP * 16 + lane);  // the spare blocks
+        __syncwarp();
 
         // reconstruct groups gi (8 columns each) of the pending tile: X = sum_j R_j w_j - q M, scaled
         auto load_group = [&](int gi, uint4 (&w)[NP]) {
-            const uint8_t* src = scr0 + (size_t)pv_half * CRT_HALF_BYTES + scr_off(0, h, gi >> 2, gi & 3, r);
 #pragma unroll
-            for (int jj = 0; jj < NP; ++jj) w[jj] = __ldcs((const uint4*)(src + (size_t)jj * SCR_J_STRIDE));  // last use
+            for (int jj = 0; jj < NP; ++jj)  // last use of each block
+                w[jj] = __ldcs((const uint4*)(scr0 + scr_off(scr_tab[ew][pv_tab][jj * 16 + gi], h, r)));
+        };
+        // after reconstructing groups [g0, g0 + 16/NP) of the pending tile their 16 blocks are free
+        auto free_groups = [&](int g0) {
+            __syncwarp();
+            if (lane < 16) scr_free[ew][lane] = scr_tab[ew][pv_tab][(lane % NP) * 16 + g0 + lane / NP];
+            __syncwarp();
         };
         // L2 prefetch of groups [g0, g1) of the pending tile (all 128 rows of this column half: one
         // 2 KB bulk prefetch per moduli pair and group, issued by one warp of the half)
@@ -543,7 +557,7 @@ __global__ void __launch_bounds__(THREADS, 1) crt_gemm_kernel(const __grid_const
             if (q == 0 && lane == 0)
                 for (int gi = g0; gi < g1; ++gi)
                     for (int jj = 0; jj < NP; ++jj) {
-                        const uint8_t* src = scr0 + (size_t)pv_half * CRT_HALF_BYTES + scr_off(jj, h, gi >> 2, gi & 3, 0);
+                        const uint8_t* src = scr0 + scr_off(scr_tab[ew][pv_tab][jj * 16 + gi], h, 0);
                         asm volatile("cp.async.bulk.prefetch.L2.global [%0], 2048;" ::"l"(src) : "memory");
                     }
         };
@@ -613,10 +627,14 @@ __global__ void __launch_bounds__(THREADS, 1) crt_gemm_kernel(const __grid_const
             tile &= (1 << 28) - 1;
             int job, bi, bj;
             tile_coords(p, tile, job, bi, bj);
-            uint8_t* const scr = scr0 + (size_t)(it_tile & 1) * CRT_HALF_BYTES;
+            const int ct = it_tile & 1;  // this tile's block table
             for (int jj = 0; jj < NP; ++jj) {
                 const int j = (j0 + jj) & (NP - 1);  // moduli pair (phase-rotated order)
                 if (pv) prefetch_groups((jj * 16) / NP, ((jj + 1) * 16) / NP);
+                // this pair's 16 destination blocks: those the last reconstruction step freed (the
+                // first tile of the CTA takes the blocks in order)
+                if (lane < 16) scr_tab[ew][ct][j * 16 + lane] = pv ? scr_free[ew][lane] : (uint8_t)(j * 16 + lane);
+                __syncwarp();
                 // ---- first modulus a of pair j: canonical residues r_a kept as bytes (32 registers)
                 uint32_t ra[4][8];
                 {
@@ -684,7 +702,8 @@ __global__ void __launch_bounds__(THREADS, 1) crt_gemm_kernel(const __grid_const
                         }
 #pragma unroll
                         for (int e = 0; e < 4; ++e)
-                            *(uint4*)(scr + scr_off(j, h, c, e, r)) = make_uint4(pk[4 * e], pk[4 * e + 1], pk[4 * e + 2], pk[4 * e + 3]);
+                            *(uint4*)(scr0 + scr_off(scr_tab[ew][ct][j * 16 + c * 4 + e], h, r)) =
+                                make_uint4(pk[4 * e], pk[4 * e + 1], pk[4 * e + 2], pk[4 * e + 3]);
                         if (c < 3) tmem_wait(vn);
                     }
                     fence_before();
@@ -705,6 +724,7 @@ __global__ void __launch_bounds__(THREADS, 1) crt_gemm_kernel(const __grid_const
                         if (gi + 1 < g1) recon(gi + 1, wb);
                         if (gi + 2 < g1) load_group(gi + 2, wa);
                     }
+                    free_groups(g0);
                     PROF_ADD(pw_recon);
                 }
             }
@@ -712,7 +732,7 @@ __global__ void __launch_bounds__(THREADS, 1) crt_gemm_kernel(const __grid_const
             const CrtJob jb = p.jobs[job];
             const int grow = bi * 256 + (int)crank * BM + r;  // row inside the tile
             pv = true;
-            pv_half = it_tile & 1;
+            pv_tab = ct;
             pv_rs = ldexp(1.0, p.exps[jb.m * p.nb + grow] - p.c.bits);
             pv_ecol = p.exps + (size_t)jb.n * p.nb + bj * BN + h * 128;
             pv_crow0 = (int)(((const char*)jb.C - (const char*)p.cbase) / ((size_t)p.nb * 8)) + bi * 256 +

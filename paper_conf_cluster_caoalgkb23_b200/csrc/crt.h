@@ -54,10 +54,13 @@ struct CrtArgs {
     int* counter = nullptr;  // 2 device ints of this launch, zero at launch: tile counter, modulus phase
     int phase_lock = 1;    // 1: each tile starts at the modulus pair the other CTAs are on
 };
-// one CTA's 128 x 256 combined residues (N/2 x 2 bytes each) for two tiles (the epilogue reconstructs
-// tile T-1 while it reduces tile T)
-constexpr size_t CRT_HALF_BYTES = (size_t)CRT_NMAX * 128 * 256;
-constexpr size_t CRT_SLOT_BYTES = 2 * CRT_HALF_BYTES;
+// One CTA's residue staging: per 128-column half, 2 KB blocks (128 rows x one 8-column group of one
+// moduli pair, uint16 residues); a tile needs N/2 x 16 blocks per half and the epilogue recycles the
+// blocks tile T-1's reconstruction frees for tile T's residues, so one tile + 16 spare blocks suffice
+// (the block permutation is tracked per warp in shared memory, crt.cu)
+constexpr int CRT_SCR_BLOCK = 128 * 16;
+constexpr int CRT_SCR_BLOCKS = CRT_NMAX / 2 * 16 + 16;  // per column half
+constexpr size_t CRT_SLOT_BYTES = (size_t)2 * CRT_SCR_BLOCKS * CRT_SCR_BLOCK;
 int crt_scratch_slots();                                         // 2 x SM count
 bool crt_available();
 cudaError_t crt_split_launch(const CrtSplitItem* items, int n, int nb, const CrtConst& c, cudaStream_t s);
