@@ -173,7 +173,7 @@ constexpr int BK = 128;             // int8 elements per 128-byte swizzled row
 constexpr int A_BYTES = BM * BK;    // 16 KB
 constexpr int B_BYTES = (BN / 2) * BK;  // 16 KB: each CTA loads half of B
 constexpr int STAGE_BYTES = A_BYTES + B_BYTES;
-constexpr int STAGES = 6;
+constexpr int STAGES = 5;  // 5 x 32 KB: with the C staging (32 KB) and the scratch-block tables the CTA fits in 227 KB
 constexpr int RING = 4;  // tile-index ring depth (dynamic scheduler)
 // C update staging: per epilogue warp two 32 x 8 FP64 boxes (2 KB, 64-byte swizzle) reduced into C
 // by the TMA unit (cp.reduce.async.bulk.tensor .add on the FP64 C map)
