@@ -72,7 +72,7 @@ bool crt_constants(int nmod, int K, CrtConst* c) {
         const unsigned p = (unsigned)kModuli[t];
         c->p[t] = (int)p;
         c->invp[t] = 1.0 / (double)p;
-        c->mq[t] = (int)(((1ull << 32) + p / 2) / p);
+        c->bm[t] = (unsigned)(((1ull << 38) + p - 1) / p);
     }
     // paired moduli m_j = p_2j p_2j+1 (< 2^16): the epilogue combines the two residues exactly,
     // R = r_a + a ((r_b - r_a) a^-1 mod b), and reconstructs from nmod/2 residues R_j in [0, m_j).
@@ -358,11 +358,15 @@ __device__ __forceinline__ void tmem_wait(uint32_t (&r)[32]) {
 __device__ __forceinline__ double exp2i(int e) {
     return (e >= -1022 && e <= 1023) ? __hiloint2double((e + 1023) << 20, 0) : ldexp(1.0, e);
 }
-// canonical residue of a (|a| < 2^27) modulo p in [0, p): q = round(a/p) +- 1 by a multiply-high
-__device__ __forceinline__ int mod_canon(int a, int p, int mq) {
-    const int q = (int)(((long long)a * mq + 0x80000000LL) >> 32);
-    int r = a - q * p;  // in [-p/2 - 1, p/2 + 1]
-    return r < 0 ? r + p : r;
+// canonical residue of a modulo p in [0, p), |a| <= 2^27 (the INT32 accumulator bound K 2^14 for
+// K <= 8192; |(r_b - r_a) ia| < 2^16): exact Barrett reduction.  a' = a + p 2^20 is a multiple-of-p
+// shift of a in [0, 2^29); with m = ceil(2^38/p), floor(a' m / 2^38) = floor(a'/p) because the excess
+// a' (m - 2^38/p) / 2^38 < 2^-9 < 1/p.  One IMAD.HI + shift + IMAD, no correction step
+// (tools/dbg/epi_rate.cu measures it against the previous rounded-quotient form).
+__device__ __forceinline__ int mod_canon(int a, int p, unsigned bm) {
+    const unsigned ap = (unsigned)(a + (p << 20));
+    const unsigned q = __umulhi(ap, bm) >> 6;
+    return (int)(ap - q * (unsigned)p);
 }
 
 }  // namespace
@@ -644,7 +648,8 @@ __global__ void __launch_bounds__(THREADS, 1) crt_gemm_kernel(const __grid_const
                     PROF_ADD(pw_accfull); }
                     PROF_T0();
                     fence_after();
-                    const int pa = p.c.p[2 * j], mqa = p.c.mq[2 * j];
+                    const int pa = p.c.p[2 * j];
+                    const unsigned mqa = p.c.bm[2 * j];
                     uint32_t v0[32], v1[32];
                     tmem_ld32_nowait(tmem + tl + buf * (uint32_t)BN, v0);
                     tmem_wait(v0);
@@ -677,7 +682,8 @@ __global__ void __launch_bounds__(THREADS, 1) crt_gemm_kernel(const __grid_const
                     PROF_ADD(pw_accfull); }
                     PROF_T0();
                     fence_after();
-                    const int pa = p.c.p[2 * j], pb = p.c.p[2 * j + 1], mqb = p.c.mq[2 * j + 1], ia = p.c.ia[j];
+                    const int pa = p.c.p[2 * j], pb = p.c.p[2 * j + 1], ia = p.c.ia[j];
+                    const unsigned mqb = p.c.bm[2 * j + 1];
                     uint32_t v0[32], v1[32];
                     tmem_ld32_nowait(tmem + tl + buf * (uint32_t)BN, v0);
                     tmem_wait(v0);

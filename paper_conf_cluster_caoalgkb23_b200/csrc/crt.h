@@ -15,7 +15,7 @@ struct CrtConst {
     int nmod;                  // number of moduli N (even, <= 16)
     int bits;                  // operand integers: x' = rint(x 2^(bits - e_row)), |x'| <= 2^bits
     int p[CRT_NMAX];           // pairwise coprime moduli <= 256
-    int mq[CRT_NMAX];          // round(2^32 / p): q = (a * mq + 2^31) >> 32 ~ round(a / p) for |a| < 2^27
+    unsigned bm[CRT_NMAX];     // ceil(2^38 / p): exact Barrett floor((a + p 2^20) / p) for |a| <= 2^27 (crt.cu)
     double invp[CRT_NMAX];     // 1/p (FP64, for the operand residues)
     int ia[CRT_NMAX / 2];      // p_2j^-1 mod p_2j+1
     int mpair[CRT_NMAX / 2];   // m_j = p_2j p_2j+1

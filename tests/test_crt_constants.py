@@ -105,3 +105,23 @@ def test_crt_epilogue_model_exact_to_final_rounding():
         worst = max(worst, float(abs(Fraction(got) - X)) / (K * 4.0**bits))
     # relative to the operand scale K 2^(2b): at most the final rounding, far below an FP64 GEMM's K u = 2^-42
     assert worst <= 2.0**-52
+
+
+def test_exact_barrett_reduction_of_the_epilogue():
+    """crt.cu mod_canon: r = a' - floor(a' m / 2^38) p with a' = a + p 2^20 and m = ceil(2^38 / p) equals
+    a mod p for every |a| <= 2^27 (the INT32 accumulator bound at K <= 8192) and every modulus of the
+    engine (dense samples + both ends of the range, exact integer arithmetic)."""
+    import numpy as np
+    moduli = [256, 255, 253, 251, 247, 241, 239, 233, 229, 227, 223, 217, 211, 199, 197, 193]
+    rng = np.random.default_rng(0)
+    lim = 1 << 27
+    a = np.concatenate([np.arange(-lim, -lim + 50000), np.arange(-50000, 50000), np.arange(lim - 50000, lim + 1),
+                        rng.integers(-lim, lim + 1, 500000)]).astype(np.int64)
+    for p in moduli:
+        m = ((1 << 38) + p - 1) // p
+        assert m < (1 << 32)
+        ap = (a + (p << 20)).astype(np.uint64)
+        assert int(ap.max()) < (1 << 29)
+        q = ((ap * np.uint64(m)) >> np.uint64(32)) >> np.uint64(6)  # __umulhi(a', m) >> 6
+        r = (ap - q * np.uint64(p)).astype(np.int64)
+        assert np.array_equal(r, np.mod(a, p)), p
