@@ -28,4 +28,10 @@ case $1 in
     run c3_fp64_dmma --config c3 --map fp64 --engine fp64_engine=1
     run c3_adaptive_dmma --config c3 --engine fp64_engine=1
     run c3_nolook --config c3 --engine lookahead=0 ;;
+  sens)
+    run c3_ureq1e-8 --config c3 --u-req 1e-8
+    run c3_nu1 --config c3 --theta 1,0.03,1.0
+    run c3_nu1_fp64 --config c3 --theta 1,0.03,1.0 --map fp64
+    run c5_ureq1e-8 --config c5 --u-req 1e-8
+    run c5_nu1 --config c5 --theta 1,0.03,1.0 ;;
 esac
