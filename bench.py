@@ -54,7 +54,7 @@ FP64_ENGINES = {0: "crt-int8 (16 moduli, Ozaki scheme II; per-row normwise bound
                 1: "dmma-fp64 (native)"}
 FP32_ENGINES = {0: "tcgen05 3xFP16 (row-scaled 11+11-bit split; per-row normwise bound)",
                 1: "tcgen05 3xTF32", 2: "dmma (FP32-rounded operands, FP32 C)"}
-DTYPE = {(0, 0, 1): "mixed f64(crt16-int8)/f32(3xf16)/f16(row-scaled)"}
+DTYPE = {(0, 0, 1): "mixed f64(crt16-int8)/f32(3xf16)/f16(row-scaled)"}  # + "/fp16-storage" with fp16_storage
 
 
 def ncu_traffic():
@@ -424,6 +424,8 @@ def main():
     dt = DTYPE.get((eng["fp64"], eng["fp32"], eng["fp16_tensor"]),
                    f"mixed f64({'crt16-int8' if crt else 'dmma'})/f32({['3xf16', '3xtf32', 'dmma'][eng['fp32']]})/"
                    f"f16({'row-scaled' if eng['fp16_tensor'] else 'dmma'})")
+    if h.config().get("fp16_storage"):
+        dt += " fp16-storage"
     if cfg["map"] == "fp64":
         dt = "f64 (" + ("crt16-int8 emulation" if crt else "dmma") + ")"
     out = {

@@ -33,7 +33,8 @@
  *    are ignored on input and set to 255 (maps) / 0 (norms) on output.
  *  - Precision codes: MP_FP64 = 0, MP_FP32 = 1, MP_FP16 = 2 (smaller = higher).
  *    MP_FP16 is the paper's FP16_32 class: FP16 operands, FP32 accumulation,
- *    FP32 storage.
+ *    FP32 storage; a storage map may hold MP_FP16 only with
+ *    mp_config::fp16_storage (tiles stored as fp16(x 2^t), t from the pass-1 tile norms).
  *  - Multi-GPU: one process (and one handle) per GPU, P x Q process grid with
  *    P <= Q, 2D block-cyclic tile ownership
  *    owner(m, k) = (m mod P) * Q + (k mod Q).  Results returned to the host
@@ -135,6 +136,9 @@ typedef struct {
                              correlation; 0: K_nu evaluated per entry */
     int f16x3_persistent; /* 1: persistent-CTA 3xFP16 kernel; 0 (default): one CTA pair per output tile */
     int crt_phase_lock;   /* 1 (default): CRT tiles start at the modulus pair the other CTAs are on */
+    int fp16_storage;     /* 1: FP16 storage class: mp_eval stores FP16-class tiles in FP16 (one
+                             power-of-two exponent per tile from its norm; 2 B instead of the paper's FP32)
+                             and sends them in FP16; needs the tcgen05 FP16 engine.  0 (default): P:152 */
 } mp_config;
 
 /* Fill *cfg with the defaults above. */

@@ -39,7 +39,7 @@ class Config(C.Structure):
     """mp_config (include/mpgeo.h): engines and schedule switches of a handle."""
     _fields_ = [("fp64_engine", C.c_int), ("fp32_engine", C.c_int), ("fp16_tensor", C.c_int), ("lookahead", C.c_int),
                 ("reserve_pairs", C.c_int), ("lowp_trsm_product", C.c_int), ("matern_table", C.c_int),
-                ("f16x3_persistent", C.c_int), ("crt_phase_lock", C.c_int)]
+                ("f16x3_persistent", C.c_int), ("crt_phase_lock", C.c_int), ("fp16_storage", C.c_int)]
 
     def as_dict(self):
         return {name: getattr(self, name) for name, _ in self._fields_}

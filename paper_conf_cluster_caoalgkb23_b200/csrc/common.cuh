@@ -26,6 +26,14 @@ __device__ __forceinline__ double round_to(double v, int prec) {
     return v;
 }
 
+// FP16 storage class (mp_config::fp16_storage): an FP16-class tile is stored as
+// fp16(x 2^t) with one power-of-two exponent t per tile (chosen from the tile norm so the stored values
+// stay far inside the FP16 range, engine.cu), read back as fp16 2^-t: 11 significant bits per entry
+// without FP16's underflow.  2^t is built from its exponent bits (|t| <= 1000).
+__device__ __forceinline__ double pow2d(int t) { return __hiloint2double((t + 1023) << 20, 0); }
+__device__ __forceinline__ __half store16(double v, int t) { return __double2half(v * pow2d(t)); }
+__device__ __forceinline__ double load16(__half h, int t) { return (double)__half2float(h) * pow2d(-t); }
+
 // Warp / block reductions (fixed order => deterministic).
 __device__ __forceinline__ double warp_sum(double v) {
 #pragma unroll

@@ -30,6 +30,9 @@ __global__ void __launch_bounds__(CV_T) panel_in_kernel(const PanelTile* tiles, 
         double2 v;
         if (t.store_prec == P64) {
             v = *(const double2*)((const double*)t.store + i);
+        } else if (t.store_prec == P16) {
+            const __half2 h = *(const __half2*)((const __half*)t.store + i);
+            v = make_double2(load16(__low2half(h), t.scale), load16(__high2half(h), t.scale));
         } else {
             const float2 f = *(const float2*)((const float*)t.store + i);
             v = make_double2((double)f.x, (double)f.y);
@@ -45,6 +48,11 @@ __global__ void __launch_bounds__(CV_T) panel_out_kernel(const PanelTile* tiles,
         const double2 v = *(const double2*)(t.p64 + i);
         if (t.store_prec == P64) {
             *(double2*)((double*)t.store + i) = v;
+        } else if (t.store_prec == P16) {  // FP16 storage class: the successors receive the stored values
+            const __half h0 = store16(v.x, t.scale), h1 = store16(v.y, t.scale);
+            *(__half2*)((__half*)t.store + i) = __halves2half2(h0, h1);
+            *(double2*)(t.p64 + i) = make_double2(load16(h0, t.scale), load16(h1, t.scale));
+            continue;
         } else {
             *(float2*)((float*)t.store + i) = make_float2(__double2float_rn(v.x), __double2float_rn(v.y));
         }

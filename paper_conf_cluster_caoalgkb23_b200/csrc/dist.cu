@@ -55,8 +55,8 @@ __global__ void __launch_bounds__(256) pack_kernel(const PackItem* items, int64_
             *(float4*)((float*)it.dst + i) =
                 make_float4(__double2float_rn(a.x), __double2float_rn(a.y), __double2float_rn(b.x), __double2float_rn(b.y));
         } else {
-            __half2 h[2] = {__halves2half2(__double2half(a.x), __double2half(a.y)),
-                            __halves2half2(__double2half(b.x), __double2half(b.y))};
+            __half2 h[2] = {__halves2half2(store16(a.x, it.scale), store16(a.y, it.scale)),
+                            __halves2half2(store16(b.x, it.scale), store16(b.y, it.scale))};
             *(uint2*)((__half*)it.dst + i) = *(const uint2*)h;
         }
     }
@@ -82,8 +82,8 @@ __global__ void __launch_bounds__(256) pull_kernel(const PullItem* items, int64_
         } else {
             const uint2 u = *(const uint2*)((const __half*)it.src + i);
             const __half2 h0 = *(const __half2*)&u.x, h1 = *(const __half2*)&u.y;
-            a = make_double2(__low2float(h0), __high2float(h0));
-            b = make_double2(__low2float(h1), __high2float(h1));
+            a = make_double2(load16(__low2half(h0), it.scale), load16(__high2half(h0), it.scale));
+            b = make_double2(load16(__low2half(h1), it.scale), load16(__high2half(h1), it.scale));
         }
         *(double2*)(it.p64 + i) = a;
         *(double2*)(it.p64 + i + 2) = b;

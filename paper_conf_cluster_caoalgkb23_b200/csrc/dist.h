@@ -15,7 +15,7 @@ struct PackItem {
     const double* src;  // FP64 values already rounded to `prec`
     void* dst;          // own send slot
     int prec;
-    int pad;
+    int scale;          // P16 payload: fp16(x 2^scale) (0 = the plain FP16 of STC; the FP16 storage class's exponent)
 };
 struct PullItem {
     const void* src;       // peer payload (comm precision)
@@ -23,7 +23,7 @@ struct PullItem {
     uint64_t target;
     double* p64;           // local FP64 panel slot (the operand formats are derived from it later)
     int prec;
-    int pad;
+    int scale;             // P16 payload exponent (see PackItem)
 };
 constexpr int MAX_PEERS = 8;
 struct GatherItem {

@@ -74,6 +74,7 @@ struct Engines {
     int f32 = MP_F32_DMMA;   // FP32 class engine (mp_fp32_engine)
     bool ctrsm = false;      // FP32/FP16-class TRSM as the CRT-8 product with the inverse factor
     bool h16 = false;        // row-scaled FP16 hi (+ lo) caches exist
+    bool s16 = false;        // FP16 storage class for FP16-class tiles (mp_config::fp16_storage)
     bool p64_double = false; // the update reads the FP64 panel buffer (a DMMA class): two panel sets
 };
 static Engines engines_for(const mp_handle* h, int nb) {
@@ -85,6 +86,7 @@ static Engines engines_for(const mp_handle* h, int nb) {
                                                                                                 : MP_F32_DMMA;
     e.ctrsm = e.crt && h->cfg.lowp_trsm_product != 0;
     e.h16 = e.tc16 || e.f32 == MP_F32_3XFP16;
+    e.s16 = h->cfg.fp16_storage != 0;
     e.p64_double = h->cfg.lookahead != 0 && (!e.crt || !e.tc16 || e.f32 == MP_F32_DMMA);
     return e;
 }
@@ -121,6 +123,9 @@ struct mp_matrix {
     bool bound = false, generated = false, factored = false;
     int cov = MP_COV_MATERN;
     std::vector<uint8_t> storage, kmap, cmap;
+    std::vector<double> sqn;      // tile sums of squares of the last generation pass 1 (NT*NT, all-gathered)
+    std::vector<int> tscale;      // FP16 storage class: per-tile exponent t (stored value fp16(x 2^t))
+    int ts(int m, int k) const { return tscale.empty() ? 0 : tscale[(size_t)m * nt + k]; }
     Regions R;
     int owner(int m, int k) const { return (m % h->P) * h->Q + (k % h->Q); }
     bool mine(int m, int k) const { return h->nranks == 1 || owner(m, k) == h->rank; }
@@ -234,7 +239,7 @@ static Regions layout(const mp_matrix* A, const uint8_t* storage) {
             for (int m = k; m < nt; ++m)
                 if (A->mine(m, k)) {
                     const uint8_t p = storage ? storage[(size_t)m * nt + k] : (uint8_t)MP_FP64;
-                    R.tile_off[(size_t)m * nt + k] = take(nb2 * (p == MP_FP64 ? 8 : 4));
+                    R.tile_off[(size_t)m * nt + k] = take(nb2 * (p == MP_FP64 ? 8 : p == MP_FP32 ? 4 : 2));
                 }
     R.total = align_up(off, 256);
     return R;
@@ -334,6 +339,7 @@ void mp_config_default(mp_config* c) {
     c->matern_table = 1;
     c->f16x3_persistent = 0;
     c->crt_phase_lock = 1;
+    c->fp16_storage = 0;
 }
 
 mp_status mp_get_unique_id(uint8_t id[128]) {
@@ -599,7 +605,7 @@ mp_status mp_matrix_bind(mp_matrix* A, const uint8_t* storage_prec, void* d_work
         for (int k = 0; k < nt; ++k)
             for (int m = k; m < nt; ++m) {
                 const uint8_t p = storage_prec[(size_t)m * nt + k];
-                if (p != MP_FP64 && p != MP_FP32) FAIL(h, MP_ERR_ARG, "storage map entry (%d,%d)=%d", m, k, p);
+                if (p > MP_FP16) FAIL(h, MP_ERR_ARG, "storage map entry (%d,%d)=%d", m, k, p);
                 if (m == k && p != MP_FP64) FAIL(h, MP_ERR_ARG, "diagonal tiles are stored in FP64 (P:117)");
             }
     Regions R = layout(A, storage_prec);
@@ -611,6 +617,17 @@ mp_status mp_matrix_bind(mp_matrix* A, const uint8_t* storage_prec, void* d_work
     for (int k = 0; k < nt; ++k)
         for (int m = k; m < nt; ++m)
             A->storage[(size_t)m * nt + k] = storage_prec ? storage_prec[(size_t)m * nt + k] : (uint8_t)MP_FP64;
+    // FP16 storage class: per-tile exponent t with ||A_mk||_F 2^t <= 2^10, from the norms of the last
+    // generation pass 1 (every entry is below the tile's Frobenius norm, so the stored values stay 2^6 below
+    // the FP16 maximum, leaving headroom for the trailing updates; without norms t = 0)
+    A->tscale.assign((size_t)nt * nt, 0);
+    for (int k = 0; k < nt; ++k)
+        for (int m = k + 1; m < nt; ++m) {
+            const size_t i = (size_t)m * nt + k;
+            if (A->storage[i] != MP_FP16 || A->sqn.size() != (size_t)nt * nt || !(A->sqn[i] > 0)) continue;
+            const int e = (int)std::floor(std::log2(std::sqrt(A->sqn[i])));
+            A->tscale[i] = std::max(-900, std::min(900, 10 - e - 1));
+        }
     A->bound = true;
     A->generated = A->factored = false;
     return MP_OK;
@@ -648,6 +665,12 @@ mp_status mp_matrix_get_tile(mp_handle* h, const mp_matrix* A, int m, int k, dou
     if (A->st(m, k) == MP_FP64) {
         CK(h, cudaMemcpyAsync(h_tile, A->tile(m, k), nb2 * 8, cudaMemcpyDeviceToHost, h->stream));
         CK(h, cudaStreamSynchronize(h->stream));
+    } else if (A->st(m, k) == MP_FP16) {
+        std::vector<__half> tmp(nb2);
+        CK(h, cudaMemcpyAsync(tmp.data(), A->tile(m, k), nb2 * 2, cudaMemcpyDeviceToHost, h->stream));
+        CK(h, cudaStreamSynchronize(h->stream));
+        const double sc = std::ldexp(1.0, -A->ts(m, k));
+        for (size_t i = 0; i < nb2; ++i) h_tile[i] = (double)__half2float(tmp[i]) * sc;
     } else {
         std::vector<float> tmp(nb2);
         CK(h, cudaMemcpyAsync(tmp.data(), A->tile(m, k), nb2 * 4, cudaMemcpyDeviceToHost, h->stream));
@@ -664,6 +687,12 @@ mp_status mp_matrix_set_tile(mp_handle* h, mp_matrix* A, int m, int k, const dou
     const size_t nb2 = A->nb2();
     if (A->st(m, k) == MP_FP64) {
         CK(h, cudaMemcpyAsync(A->tile(m, k), h_tile, nb2 * 8, cudaMemcpyHostToDevice, h->stream));
+        CK(h, cudaStreamSynchronize(h->stream));
+    } else if (A->st(m, k) == MP_FP16) {
+        std::vector<__half> tmp(nb2);
+        const double sc = std::ldexp(1.0, A->ts(m, k));
+        for (size_t i = 0; i < nb2; ++i) tmp[i] = __float2half((float)(h_tile[i] * sc));
+        CK(h, cudaMemcpyAsync(A->tile(m, k), tmp.data(), nb2 * 2, cudaMemcpyHostToDevice, h->stream));
         CK(h, cudaStreamSynchronize(h->stream));
     } else {
         std::vector<float> tmp(nb2);
@@ -788,6 +817,7 @@ mp_status mp_matern_gen(mp_handle* h, mp_matrix* A, const double* d_x, const dou
         CK(h, cudaStreamSynchronize(h->stream));
         for (size_t i = 0; i < (size_t)nt * nt; ++i) tile_sqnorm[i] = 0.0;
         for (int i = 0; i < ntl; ++i) tile_sqnorm[(size_t)tl[i].m * nt + tl[i].k] = v[i];
+        A->sqn.clear();
         if (h->nranks > 1) {
             // all-gather over peer memory: every tile has exactly one owner, so the merge is exact
             Comm& X = A->comm;
@@ -805,6 +835,7 @@ mp_status mp_matern_gen(mp_handle* h, mp_matrix* A, const double* d_x, const dou
             }
             if (mp_status st = dist_barrier(h, A, stamp + 1)) return st;
         }
+        A->sqn.assign(tile_sqnorm, tile_sqnorm + (size_t)nt * nt);  // the FP16 storage class's tile exponents
         return MP_OK;
     }
     if (!A->bound) FAIL(h, MP_ERR_STATE, "matrix not bound");
@@ -815,7 +846,7 @@ mp_status mp_matern_gen(mp_handle* h, mp_matrix* A, const double* d_x, const dou
     std::vector<GenTile> tl;
     for (int k = 0; k < nt; ++k)
         for (int m = k; m < nt; ++m)
-            if (A->mine(m, k)) tl.push_back(GenTile{m, k, A->st(m, k), 0, A->tile(m, k)});
+            if (A->mine(m, k)) tl.push_back(GenTile{m, k, A->st(m, k), A->ts(m, k), A->tile(m, k)});
     Arena ar;
     ar.dev_base = A->ws + A->R.ctrl;
     GenTile* d_tl = ar.push(tl);
@@ -875,6 +906,12 @@ static mp_status plan_potrf(mp_handle* h, mp_matrix* A, const uint8_t* km, const
     };
     auto K = [&](int m, int k) { return km[(size_t)m * nt + k]; };
     auto C = [&](int m, int k) { return cm[(size_t)m * nt + k]; };
+    auto xscale = [&](int m, int k) { return A->ts(m, k); };  // FP16 storage class payloads carry the tile exponent
+    if (E.s16 && !E.tc16)
+        for (int k = 0; k < nt; ++k)
+            for (int m = k + 1; m < nt; ++m)
+                if (A->st(m, k) == MP_FP16)
+                    FAIL(h, MP_ERR_UNSUPPORTED, "FP16 storage class needs the tcgen05 FP16 engine (nb %% 256 == 0)");
     const double fnb = (double)nb;
     std::vector<Op>* cur = nullptr;
     auto cur_push = [&](Op o) { cur->push_back(std::move(o)); };
@@ -1058,7 +1095,8 @@ static mp_status plan_potrf(mp_handle* h, mp_matrix* A, const uint8_t* km, const
         // ---- 3. panel in
         std::vector<PanelTile> pin;
         for (int m = k + 1; m < nt; ++m)
-            if (A->mine(m, k)) pin.push_back(PanelTile{A->tile(m, k), p64 + (size_t)m * nb2, A->st(m, k), C(m, k)});
+            if (A->mine(m, k))
+                pin.push_back(PanelTile{A->tile(m, k), p64 + (size_t)m * nb2, A->st(m, k), C(m, k), A->ts(m, k), 0});
         if (!pin.empty()) {
             PanelTile* d_in = ar.push(pin);
             const int np = (int)pin.size();
@@ -1130,7 +1168,7 @@ static mp_status plan_potrf(mp_handle* h, mp_matrix* A, const uint8_t* km, const
             for (auto& x : xpub[k]) {
                 const int m = x.m;
                 if (m == k) continue;
-                packs.push_back(PackItem{p64 + (size_t)m * nb2, sendslot(me, sp, m), C(m, k), 0});
+                packs.push_back(PackItem{p64 + (size_t)m * nb2, sendslot(me, sp, m), C(m, k), A->st(m, k) == MP_FP16 ? xscale(m, k) : 0});
                 flags.push_back(WaitItem{pubflag(me, sp, m), ST(k)});
             }
             if (!packs.empty()) {
@@ -1151,7 +1189,8 @@ static mp_status plan_potrf(mp_handle* h, mp_matrix* A, const uint8_t* km, const
                 const int m = x.m;
                 if (m == k) continue;
                 const int o = x.peer;
-                PullItem it{sendslot(o, sp, m), pubflag(o, sp, m), ST(k), p64 + (size_t)m * nb2, C(m, k), 0};
+                PullItem it{sendslot(o, sp, m), pubflag(o, sp, m), ST(k), p64 + (size_t)m * nb2, C(m, k),
+                            A->st(m, k) == MP_FP16 ? xscale(m, k) : 0};
                 waits.push_back(WaitItem{it.flag, it.target});
                 pulls.push_back(it);
                 have[m] = 1;
@@ -1222,7 +1261,7 @@ static mp_status plan_potrf(mp_handle* h, mp_matrix* A, const uint8_t* km, const
                         if (E.crt) c64.push_back(CrtJob{m, n, A->tile(m, n)});
                         else g64.push_back(GemmJob{p64 + (size_t)m * nb2, p64 + (size_t)n * nb2, A->tile(m, n)});
                     } else if (p == MP_FP32 ? E.f32 != MP_F32_DMMA : E.tc16) {
-                        (p == MP_FP32 ? t32 : t16).push_back(TcJob{m, n, (float*)A->tile(m, n)});
+                        (p == MP_FP32 ? t32 : t16).push_back(TcJob{m, n, A->tile(m, n), A->ts(m, n), 0});
                     } else {
                         (p == MP_FP32 ? g32 : g16).push_back(GemmJob{p64 + (size_t)m * nb2, p64 + (size_t)n * nb2, A->tile(m, n)});
                     }
@@ -1275,6 +1314,10 @@ static mp_status plan_potrf(mp_handle* h, mp_matrix* A, const uint8_t* km, const
                 ta.e16 = e16;
                 ta.cbase = cpool;
                 ta.crows = crows;
+                if (E.s16) {  // FP16 storage class: FP16 C tiles (FP16 view of the pool)
+                    ta.c16 = 1;
+                    ta.crows = (RG.total - RG.pool) / ((size_t)nb * 2);
+                }
                 cur->push_back({[=](cudaStream_t s) { return tc_gemm_f16_launch(ta, nj, s); }, C_UPD16, 2 * f3 * nj});
             }
         }  // part
@@ -1323,7 +1366,8 @@ static mp_status potrf_run(mp_handle* h, mp_matrix* A, const uint8_t* km, const 
             const size_t i = (size_t)m * nt + k;
             if (km[i] > MP_FP16 || cm[i] > MP_FP16 || (m == k && km[i] != MP_FP64))
                 FAIL(h, MP_ERR_ARG, "bad map entry at (%d,%d)", m, k);
-            if (m > k && A->st(m, k) != (km[i] == MP_FP64 ? MP_FP64 : MP_FP32))
+            if (m > k && A->st(m, k) != (km[i] == MP_FP64 ? MP_FP64 : MP_FP32) &&
+                !(A->st(m, k) == MP_FP16 && km[i] == MP_FP16 && h->cfg.fp16_storage))
                 FAIL(h, MP_ERR_ARG, "kernel map inconsistent with the bound storage map at (%d,%d)", m, k);
             if (m > k && cm[i] < A->st(m, k)) FAIL(h, MP_ERR_ARG, "comm precision above storage at (%d,%d)", m, k);
         }
@@ -1433,7 +1477,7 @@ static mp_status loglik_dist(mp_handle* h, mp_matrix* A, const double* d_z, doub
         if (myq == k % Q) {
             std::vector<GemvTile> gv;
             for (int m = k + 1; m < nt; ++m)
-                if (A->mine(m, k)) gv.push_back(GemvTile{A->tile(m, k), A->st(m, k), 0, racc + (size_t)m * nb});
+                if (A->mine(m, k)) gv.push_back(GemvTile{A->tile(m, k), A->st(m, k), A->ts(m, k), racc + (size_t)m * nb});
             if (!gv.empty()) {
                 if (o != me) wait_op({WaitItem{yflag(o, k), ST(k)}});
                 GemvTile* dg = ar.push(gv);
@@ -1529,7 +1573,7 @@ mp_status mp_loglik(mp_handle* h, const mp_matrix* Lc, const double* d_z, double
         op.nlaunch = 2 * ceil_div(nb, POTRF_IB) - 1;
         ops.push_back(std::move(op));
         std::vector<GemvTile> gv;
-        for (int m = k + 1; m < nt; ++m) gv.push_back(GemvTile{A->tile(m, k), A->st(m, k), 0, r + (size_t)m * nb});
+        for (int m = k + 1; m < nt; ++m) gv.push_back(GemvTile{A->tile(m, k), A->st(m, k), A->ts(m, k), r + (size_t)m * nb});
         if (!gv.empty()) {
             GemvTile* dg = ar.push(gv);
             const int ng = (int)gv.size();
@@ -1573,7 +1617,7 @@ mp_status mp_gp_sample(mp_handle* h, const mp_matrix* Lc, const double* d_e, dou
     // the GEMV kernel accumulates r_m -= L_mk e_k, i.e. r = -L e; the sign is flipped on the way out
     for (int k = 0; k < nt; ++k) {
         std::vector<GemvTile> gv;
-        for (int m = k; m < nt; ++m) gv.push_back(GemvTile{A->tile(m, k), A->st(m, k), 0, r + (size_t)m * nb});
+        for (int m = k; m < nt; ++m) gv.push_back(GemvTile{A->tile(m, k), A->st(m, k), A->ts(m, k), r + (size_t)m * nb});
         GemvTile* dg = ar.push(gv);
         const int ng = (int)gv.size();
         const double* yk = ye + (size_t)k * nb;
@@ -1657,6 +1701,12 @@ mp_status mp_eval(mp_handle* h, mp_matrix* A, const double* x, const double* y, 
             return MP_ERR_ARG;
     }
     if (st) FAIL(h, st, "precision map failed");
+    if (h->cfg.fp16_storage)  // FP16 storage class: FP16-class tiles stored in FP16, and
+        for (int k = 0; k < nt; ++k)  // they travel in FP16 (Alg. 2 caps comm at storage)
+            for (int m = k + 1; m < nt; ++m) {
+                const size_t i = (size_t)m * nt + k;
+                if (km[i] == MP_FP16) sm[i] = cm[i] = MP_FP16;
+            }
     {  // the workspace this map needs (tiles in storage precision + the map-independent regions)
         const size_t need = layout(A, sm.data()).total;
         rep->workspace_bytes = need;

@@ -33,8 +33,8 @@ cudaError_t trtri_batch_launch(const double* const* Ls, int ntiles, int nb, doub
 // ---- K1: Matérn generation (matern.cu)
 struct GenTile {
     int m, k;     // tile coordinates
-    int prec;     // storage precision of the destination (P64 / P32); unused in pass 1
-    int pad;
+    int prec;     // storage precision of the destination (P64 / P32 / P16); unused in pass 1
+    int scale;    // P16 storage: the tile's exponent t (stored value fp16(x 2^t))
     void* dst;    // nb x nb row-major destination (pass 2)
 };
 struct MaternArgs {
@@ -69,8 +69,10 @@ cudaError_t bessel_k_launch(double nu, const double* x, double* out, int n, cuda
 struct PanelTile {
     void* store;      // the tile in the pool (storage precision)
     double* p64;      // FP64 panel slot
-    int store_prec;   // P64 / P32
+    int store_prec;   // P64 / P32 / P16 (FP16 storage class, scaled by 2^scale)
     int comm_prec;    // precision the tile is sent at (P64 / P32 / P16)
+    int scale;        // P16 storage: the tile's exponent
+    int pad;
 };
 struct Tf32Item {     // 3xTF32 operands of one panel tile (FP32 class with MP_F32_3XTF32)
     const double* src;
@@ -108,7 +110,7 @@ cudaError_t trsv_blocked_launch(const double* L, int nb, const double* Wk, doubl
 struct GemvTile {
     const void* L;    // tile (m, k), storage precision, nb x nb
     int prec;
-    int pad;
+    int scale;        // P16 storage: the tile's exponent
     double* r;        // r_m (nb), updated r_m -= L y
 };
 // r_m -= L_mk y_k for a batch of tiles sharing y

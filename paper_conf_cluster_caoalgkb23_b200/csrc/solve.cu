@@ -74,6 +74,13 @@ __global__ void __launch_bounds__(GV_T) gemv_sub_kernel(const GemvTile* tiles, c
                 s = fma(v.x, ys[c], s);
                 s = fma(v.y, ys[c + 1], s);
             }
+        } else if (t.prec == P16) {
+            const __half* row = (const __half*)t.L + (size_t)i * nb;
+            for (int c = 2 * lane; c < nb; c += 64) {
+                const __half2 v = *(const __half2*)(row + c);
+                s = fma(load16(__low2half(v), t.scale), ys[c], s);
+                s = fma(load16(__high2half(v), t.scale), ys[c + 1], s);
+            }
         } else {
             const float* row = (const float*)t.L + (size_t)i * nb;
             for (int c = 2 * lane; c < nb; c += 64) {

@@ -48,10 +48,11 @@ struct TcThreads {
 struct __align__(64) TcParams {
     CUtensorMap a, b, a_lo, b_lo, c;
     const TcJob* jobs;
-    const float* cbase;
+    const char* cbase;
     const int* exps;  // per panel-cache row, 2^exps undoes the operand's power-of-two row scale
     int nb, tiles_n, tiles_per_job;
     int total;        // persistent kernel: pair tiles of the launch
+    int c16;          // KIND 0: FP16 C tiles (FP16 storage class)
 };
 
 // CL = CTAs per MMA: 1 (tcgen05.mma.cta_group::1, M = 128) or 2 (a CTA pair on one TPC,
@@ -228,6 +229,24 @@ __device__ __forceinline__ void scale_group(float* v, float ra, const int4* eb) 
         v[4 * i + 3] = (v[4 * i + 3] * ra) * __int_as_float((e4.w + 127) << 23);
     }
 }
+// FP16 C (FP16 storage class): -v 2^cscale as FP16 into a 32 x 32 box with 64-byte rows (64-byte swizzle:
+// 16-byte chunk j of row r at chunk j ^ ((r >> 1) & 3)); v already carries the operands' row scales
+__device__ __forceinline__ void stage_box_neg16(uint32_t buf, int lane, const float* v, float cs) {
+#pragma unroll
+    for (int j = 0; j < 4; ++j) {
+        uint32_t w[4];
+#pragma unroll
+        for (int i = 0; i < 4; ++i) {
+            const __half2 h = __floats2half2_rn(-v[8 * j + 2 * i] * cs, -v[8 * j + 2 * i + 1] * cs);
+            w[i] = *(const uint32_t*)&h;
+        }
+        const uint32_t a = buf + (uint32_t)lane * 64u + ((uint32_t)(j ^ ((lane >> 1) & 3)) << 4);
+        asm volatile("st.shared.v4.b32 [%0], {%1, %2, %3, %4};" ::"r"(a), "r"(w[0]), "r"(w[1]), "r"(w[2]), "r"(w[3])
+                     : "memory");
+    }
+    asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+    __syncwarp();
+}
 __device__ __forceinline__ void tma_reduce_add(const CUtensorMap* map, uint32_t buf, int c0, int c1) {
     asm volatile("cp.reduce.async.bulk.tensor.2d.global.shared::cta.add.tile.bulk_group [%0, {%2, %3}], [%1];" ::"l"(
                      (uint64_t)map),
@@ -361,7 +380,8 @@ __global__ void __launch_bounds__(TcThreads<KIND>::N, TcCfg<KIND, CL>::MIN_BLOCK
         constexpr int COLS = Cfg::BN / (EPI_WARPS / 4);
         const int q = (warp - 4) & 3;
         const int half = (warp - 4) >> 2;
-        const int crow0 = (int)((jb.C - p.cbase) / p.nb) + bi * Cfg::BM + (int)crank * TC_BM + q * 32;
+        const int crow0 = (int)(((const char*)jb.C - p.cbase) / ((size_t)p.nb * (p.c16 ? 2 : 4))) + bi * Cfg::BM +
+                          (int)crank * TC_BM + q * 32;
         const int ccol0 = bj * Cfg::BN + half * COLS;
         const uint32_t tl = ((uint32_t)(q * 32) << 16) + (uint32_t)(half * COLS);
         const uint32_t stg = smem_u32(smem) + (uint32_t)(warp - 4) * 8192u;  // two 4 KB boxes per warp
@@ -383,7 +403,8 @@ __global__ void __launch_bounds__(TcThreads<KIND>::N, TcCfg<KIND, CL>::MIN_BLOCK
 #pragma unroll
                 for (int i = 0; i < 32; ++i) v[i] = __uint_as_float(r[i]);
                 scale_group(v, ra, eb + g * 8);  // undo the operands' power-of-two row scales
-                stage_box_neg(buf, lane, v);
+                if (p.c16) stage_box_neg16(buf, lane, v, __int_as_float((jb.cscale + 127) << 23));
+                else stage_box_neg(buf, lane, v);
                 if (lane == 0) tma_reduce_add(&p.c, buf, ccol0 + g * 32, crow0);
             }
         } else {
@@ -563,7 +584,7 @@ __global__ void __launch_bounds__((4 + P16_EPI) * 32, 1) tc_f16x3_persistent_ker
             coords(t, job, bi, bj);
             const TcJob jb = p.jobs[job];
             const int rowA = jb.m * p.nb + bi * Cfg::BM + (int)crank * TC_BM;
-            const int crow0 = (int)((jb.C - p.cbase) / p.nb) + bi * Cfg::BM + (int)crank * TC_BM + q * 32;
+            const int crow0 = (int)(((const char*)jb.C - p.cbase) / ((size_t)p.nb * 4)) + bi * Cfg::BM + (int)crank * TC_BM + q * 32;
             const int ccol0 = bj * Cfg::BN + half * COLS;
             float sum[COLS];
 #pragma unroll
@@ -620,7 +641,7 @@ static PFN_cuTensorMapEncodeTiled_v12000 encode_fn() {
 }
 
 static bool make_map(CUtensorMap* m, const void* base, CUtensorMapDataType dt, int esz, uint64_t rows, uint64_t cols,
-                     uint32_t box_cols, uint32_t box_rows) {
+                     uint32_t box_cols, uint32_t box_rows, CUtensorMapSwizzle sw = CU_TENSOR_MAP_SWIZZLE_128B) {
     auto fn = encode_fn();
     if (!fn) return false;
     cuuint64_t dims[2] = {cols, rows};
@@ -628,7 +649,7 @@ static bool make_map(CUtensorMap* m, const void* base, CUtensorMapDataType dt, i
     cuuint32_t box[2] = {box_cols, box_rows};
     cuuint32_t es[2] = {1, 1};
     return fn(m, dt, 2, const_cast<void*>(base), dims, strides, box, es, CU_TENSOR_MAP_INTERLEAVE_NONE,
-              CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+              sw, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
               CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
 }
 
@@ -683,11 +704,18 @@ static cudaError_t launch(const TcArgs& a, int njobs, cudaStream_t s) {
              make_map(&p.b, a.hi, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 4, rows, a.nb, Cfg::BK, BROWS) &&
              make_map(&p.b_lo, a.lo, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 4, rows, a.nb, Cfg::BK, BROWS);
     }
-    // C: FP32 rows of nb over [cbase, cbase + crows * nb), 32 x 32 boxes, 128-byte swizzle
-    ok = ok && a.cbase && make_map(&p.c, a.cbase, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 4, a.crows, a.nb, 32, 32);
+    // C: FP32 rows of nb over [cbase, cbase + crows * nb), 32 x 32 boxes, 128-byte swizzle; FP16 C (KIND 0
+    // with c16): 32 x 32 boxes of 64-byte rows, 64-byte swizzle
+    if (a.c16 && KIND != 0) return cudaErrorInvalidValue;
+    if (a.c16)
+        ok = ok && a.cbase && make_map(&p.c, a.cbase, CU_TENSOR_MAP_DATA_TYPE_FLOAT16, 2, a.crows, a.nb, 32, 32,
+                                       CU_TENSOR_MAP_SWIZZLE_64B);
+    else
+        ok = ok && a.cbase && make_map(&p.c, a.cbase, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 4, a.crows, a.nb, 32, 32);
     if (!ok) return cudaErrorInvalidValue;
     p.jobs = a.jobs;
-    p.cbase = a.cbase;
+    p.cbase = (const char*)a.cbase;
+    p.c16 = a.c16;
     p.nb = a.nb;
     p.tiles_n = a.nb / Cfg::BN;
     p.tiles_per_job = (a.nb / Cfg::BM) * p.tiles_n;

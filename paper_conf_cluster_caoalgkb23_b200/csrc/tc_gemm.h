@@ -14,8 +14,10 @@
 
 namespace mpgeo {
 struct TcJob {
-    int m, n;   // panel rows of the two operands (tiles (m,k) and (n,k) of the current panel)
-    float* C;   // FP32 nb x nb output tile (row-major)
+    int m, n;    // panel rows of the two operands (tiles (m,k) and (n,k) of the current panel)
+    void* C;     // nb x nb output tile (row-major): FP32, or FP16 with TcArgs::c16 (FP16 storage class)
+    int cscale;  // c16: the C tile's exponent (stored value fp16(x 2^cscale))
+    int pad;
 };
 struct TcArgs {
     const TcJob* jobs;
@@ -30,10 +32,11 @@ struct TcArgs {
     const int* e16 = nullptr;
     int persistent = 0;  // 3xFP16: persistent CTA-pair kernel (mp_config::f16x3_persistent)
     int pairs = 0;       // persistent 3xFP16 kernel: CTA pairs to use (0: all SMs / 2)
-    // every TcJob::C lies in [cbase, cbase + crows * nb) at a whole row offset (the epilogue
-    // reduces into C through one TMA tensor map over this range)
-    const float* cbase;
+    // every TcJob::C lies in [cbase, cbase + crows rows of nb elements) at a whole row offset (the
+    // epilogue reduces into C through one TMA tensor map over this range)
+    const void* cbase;
     uint64_t crows;
+    int c16 = 0;  // FP16-class GEMM only: C tiles are FP16 (reduce-added in FP16, scaled by 2^cscale)
 };
 bool tc_gemm_available();
 cudaError_t tc_gemm_tf32x3_launch(const TcArgs& a, int njobs, cudaStream_t s);

@@ -91,3 +91,26 @@ def test_precision_map_rejects_bad_input():
     bad[2, 2] = FP16  # diagonal must be FP64
     with pytest.raises(MpError):
         precision_map(None, kernel_prec=bad)
+
+
+def test_config_defaults_and_unique_id_on_cpu():
+    """mp_config_default fills the documented defaults (include/mpgeo.h); mp_get_unique_id gives 128
+    bytes with fresh randomness per call and this host's name (no GPU needed for either)."""
+    import socket
+    import paper_conf_cluster_caoalgkb23_b200 as mp
+    cfg = mp.default_config()
+    assert cfg == {"fp64_engine": mp.MP_F64_CRT16, "fp32_engine": mp.MP_F32_3XFP16, "fp16_tensor": 1, "lookahead": 1,
+                   "reserve_pairs": 6, "lowp_trsm_product": 1, "matern_table": 1, "f16x3_persistent": 0,
+                   "crt_phase_lock": 1, "fp16_storage": 0}
+    a, b = mp.unique_id(), mp.unique_id()
+    assert len(a) == len(b) == 128 and a != b and a[:32] != b[:32]
+    assert a[48:48 + len(socket.gethostname().encode()[:79])] == socket.gethostname().encode()[:79]
+
+
+def test_multirank_init_requires_the_communicator_id():
+    """nranks > 1 without the id of mp_get_unique_id is an argument error (checked before any CUDA call)."""
+    import ctypes as C
+    from paper_conf_cluster_caoalgkb23_b200._lib import lib, MP_ERR_ARG
+    h = C.c_void_p()
+    assert lib.mp_init(0, 0, 2, 1, 2, None, None, C.byref(h)) == MP_ERR_ARG
+    assert lib.mp_init(0, 0, 16, 4, 4, None, None, C.byref(h)) != 0  # more ranks than MAX_PEERS

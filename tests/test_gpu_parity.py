@@ -311,3 +311,35 @@ def test_gp_sample_matches_dense_factor(mp, handle):
     from oracle.tiles import dense_covariance
     ref = np.linalg.cholesky(dense_covariance(x, y, theta)) @ e
     assert np.max(np.abs(dz.cpu().numpy() - ref)) <= 1e-12 * np.max(np.abs(ref))
+
+
+def test_fp16_storage_class(mp):
+    """SURVEY §8(f)3 FP16 storage class (mp_config.fp16_storage): FP16-class tiles stored as fp16(x 2^t),
+    sent in FP16.  Maps: storage and comm FP16 exactly where the kernel map is FP16 (else the paper's
+    maps); l within the north-star 1e-5 of the FP64 oracle; the factor's backward error within the bound
+    of the maps (FP16 storage rounding included); smaller workspace than the P:152 FP32 storage."""
+    n, nb, u_req, theta = 10000, 512, 1e-9, (1.0, 0.03, 0.5)
+    x, y = synth.locations(n, 0)
+    z = synth.normal_vector(n, 1)
+    ref = oracle_loglik(x, y, z, theta, nb)
+    nt = num_tiles(n, nb)
+    okm, osm, ocm = precision_maps(tile_sqnorms(ref["tiles"], nt), u_req)
+    h16 = mp.Handle(0, config={"fp16_storage": 1})
+    ev16 = mp.Evaluator(n, nb, handle=h16)
+    r16 = ev16.eval(x, y, z, theta, u_req=u_req)
+    km, sm, cm = ev16.M.maps()
+    low = np.tril(np.ones((nt, nt), bool), -1)
+    assert np.array_equal(km[low], okm[low]) and r16.tiles[2] > 0
+    f16 = low & (okm == FP16)
+    assert np.all(sm[f16] == FP16) and np.all(cm[f16] == FP16)
+    assert np.array_equal(sm[low & ~f16], osm[low & ~f16]) and np.array_equal(cm[low & ~f16], ocm[low & ~f16])
+    err = abs(r16.loglik - ref["loglik"]) / abs(ref["loglik"])
+    assert err <= 1e-5, err
+    Lhat = {key: ev16.M.tile(*key)[: t.shape[0], : t.shape[1]] for key, t in ref["tiles"].items()}
+    worst, _ = mp_backward_check(ref["tiles"], Lhat, ref["factor"], km, sm, cm, nt, nb)
+    assert worst <= 1.0, worst
+    ev32 = mp.Evaluator(n, nb)
+    r32 = ev32.eval(x, y, z, theta, u_req=u_req)
+    assert r16.workspace_bytes < r32.workspace_bytes
+    print(f"FP16 storage: l rel. error {err:.2e} (FP32 storage {abs(r32.loglik - ref['loglik']) / abs(ref['loglik']):.2e}), "
+          f"workspace {r16.workspace_bytes / 1e9:.2f} vs {r32.workspace_bytes / 1e9:.2f} GB")
