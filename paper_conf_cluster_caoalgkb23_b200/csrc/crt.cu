@@ -183,10 +183,11 @@ constexpr int SMEM = STAGES * STAGE_BYTES + 8 * STG_WARP + 1024;
 constexpr int EPI_WARPS = 8;
 constexpr int THREADS = (4 + EPI_WARPS) * 32;
 constexpr uint32_t TMEM_COLS = 512;  // two 256-column accumulators
-#ifndef CRT_SCR_HINT
-#define CRT_SCR_HINT 1
+// L2 eviction priority of the operand loads (residue planes): 0 normal, 1 evict_last for A (the row
+// operand consecutive jobs share), 2 evict_last for A and B
+#ifndef CRT_L2HINT
+#define CRT_L2HINT 0
 #endif
-constexpr bool SCR_HINT = CRT_SCR_HINT;  // L2 evict_last policy on the residue scratch
 // instruction descriptor: D = S32 (2 << 4), A = B = signed int8 (1 << 7, 1 << 10), K-major,
 // N >> 3 at bit 17, M >> 4 at bit 24 (M = 256 for the pair)
 constexpr uint32_t IDESC = (2u << 4) | (1u << 7) | (1u << 10) | ((uint32_t)(BN >> 3) << 17) | ((uint32_t)(256 >> 4) << 24);
@@ -271,6 +272,14 @@ __device__ __forceinline__ void tma3d_pair(uint32_t dst, const CUtensorMap* map,
     asm volatile(
         "cp.async.bulk.tensor.3d.cta_group::2.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1, {%3, %4, %5}], [%2];" ::"r"(dst),
         "l"((uint64_t)map), "r"(bar), "r"(c0), "r"(c1), "r"(c2)
+        : "memory");
+}
+// the same with an L2 cache-policy hint (createpolicy)
+__device__ __forceinline__ void tma3d_pair_hint(uint32_t dst, const CUtensorMap* map, uint32_t bar, int c0, int c1, int c2,
+                                                uint64_t pol) {
+    asm volatile(
+        "cp.async.bulk.tensor.3d.cta_group::2.shared::cluster.global.mbarrier::complete_tx::bytes.L2::cache_hint [%0], [%1, {%3, %4, %5}], [%2], %6;" ::"r"(dst),
+        "l"((uint64_t)map), "r"(bar), "r"(c0), "r"(c1), "r"(c2), "l"(pol)
         : "memory");
 }
 __device__ __forceinline__ void fence_before() { asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory"); }
@@ -443,6 +452,8 @@ __global__ void __launch_bounds__(THREADS, 1) crt_gemm_kernel(const __grid_const
     if (warp == 0 && lane == 0) {
         // ---------------- TMA producer: per tile, per modulus, K in 128-byte blocks
         uint32_t it = 0;
+        uint64_t pol_last = 0;
+        if (CRT_L2HINT) asm volatile("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(pol_last));
         for (int i = 0;; ++i) {
             int tile;
             if (crank == 0) {  // claim the next pair tile and publish it to both CTAs
@@ -479,8 +490,10 @@ __global__ void __launch_bounds__(THREADS, 1) crt_gemm_kernel(const __grid_const
                     const uint32_t lb = su32(&full_bar[s]);
                     const uint32_t fb = cluster_addr(lb, 0);
                     if (crank == 0) mbar_expect_tx(lb, 2 * STAGE_BYTES);
-                    tma3d_pair(st, &p.a, fb, kb * BK, rowA, t);
-                    tma3d_pair(st + A_BYTES, &p.b, fb, kb * BK, rowB, t);
+                    if (CRT_L2HINT >= 1) tma3d_pair_hint(st, &p.a, fb, kb * BK, rowA, t, pol_last);
+                    else tma3d_pair(st, &p.a, fb, kb * BK, rowA, t);
+                    if (CRT_L2HINT >= 2) tma3d_pair_hint(st + A_BYTES, &p.b, fb, kb * BK, rowB, t, pol_last);
+                    else tma3d_pair(st + A_BYTES, &p.b, fb, kb * BK, rowB, t);
                 }
             }
         }
