@@ -144,3 +144,41 @@ def test_exchange_plan_consistent_over_gloo(world, P, Q):
                      if d == 1 and m > k) for name in maps}
     assert vol["extreme_auto"] * 2 == vol["extreme_ttc"]
     assert vol["random_auto"] <= vol["random_ttc"]
+
+
+def _uid_worker(rank, world, port, q):
+    import sys
+    sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    import torch.distributed as dist
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    try:
+        import paper_conf_cluster_caoalgkb23_b200 as mp
+        q.put((rank, mp.shared_unique_id(), None))
+    except Exception:  # pragma: no cover - reported to the parent
+        import traceback
+        q.put((rank, None, traceback.format_exc()))
+    finally:
+        dist.destroy_process_group()
+
+
+def test_communicator_id_is_shared_over_gloo():
+    """mp_get_unique_id on rank 0, broadcast over torch.distributed (gloo, world size 3): every rank
+    holds the same 128 bytes (the id each rank passes to mp_init_config and that mp_matrix_comm_connect
+    checks in the peers' exchange areas)."""
+    import torch.multiprocessing as tmp
+    ctx = tmp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_uid_worker, args=(r, 3, port, q)) for r in range(3)]
+    for p in procs:
+        p.start()
+    ids = {}
+    for _ in range(3):
+        r, uid, err = q.get(timeout=300)
+        assert err is None, err
+        ids[r] = uid
+    for p in procs:
+        p.join(timeout=60)
+    assert len(ids[0]) == 128 and ids[0] == ids[1] == ids[2]
