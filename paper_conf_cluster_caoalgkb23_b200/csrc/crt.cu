@@ -437,7 +437,7 @@ __global__ void __launch_bounds__(THREADS, 1) crt_gemm_kernel(const __grid_const
     fence_after();
     const uint32_t tmem = tmem_slot;
 #ifdef CRT_PROF
-    long long pw_accempty = 0, pw_full = 0, pw_accfull = 0, pw_resid = 0, pw_recon = 0;
+    long long pw_accempty = 0, pw_full = 0, pw_accfull = 0, pw_resid = 0, pw_recon = 0, pw_stgwait = 0, pw_ld = 0;
 #endif
 
     // ring slot i % RING: wait for the published tile index, then release the slot to the leader
@@ -580,6 +580,16 @@ __global__ void __launch_bounds__(THREADS, 1) crt_gemm_kernel(const __grid_const
         };
         auto recon = [&](int gi, const uint4 (&w)[NP]) {
             const int col0 = (gi >> 2) * 32 + (gi & 3) * 8;
+#ifdef CRT_PROF
+            {  // time until the scratch loads of this group have landed
+                PROF_T0();
+                uint32_t t = 0;
+#pragma unroll
+                for (int jj = 0; jj < NP; ++jj) t ^= w[jj].x ^ w[jj].w;
+                asm volatile("" ::"r"(t));
+                PROF_ADD(pw_ld);
+            }
+#endif
             double sh[8], sl[8];
 #pragma unroll
             for (int v = 0; v < 8; ++v) sh[v] = sl[v] = 0.0;
@@ -600,7 +610,9 @@ __global__ void __launch_bounds__(THREADS, 1) crt_gemm_kernel(const __grid_const
             // k ^ ((l >> 1) & 3)); one lane reduces the box into C through the TMA unit
             const uint32_t sb = stg_s + (nred & 1u) * (uint32_t)STG_BOX;
             if (nred >= 2) {
+                PROF_T0();
                 if (lane == 0) asm volatile("cp.async.bulk.wait_group.read 1;" ::: "memory");
+                PROF_ADD(pw_stgwait);
                 __syncwarp();
             }
             double o[8];
@@ -777,6 +789,9 @@ __global__ void __launch_bounds__(THREADS, 1) crt_gemm_kernel(const __grid_const
     if (blockIdx.x < 4 && (threadIdx.x == 32 || threadIdx.x == 128 || threadIdx.x == 288))
         printf("cta %d thr %d: accempty %lld full %lld | accfull %lld resid %lld recon %lld (cycles)\n", blockIdx.x,
                threadIdx.x, pw_accempty, pw_full, pw_accfull, pw_resid, pw_recon);
+    if (blockIdx.x < 2 && threadIdx.x == 128)
+        printf("cta %d thr %d: recon detail: staging-buffer waits %lld, first-use of the scratch loads %lld (cycles)\n",
+               blockIdx.x, threadIdx.x, pw_stgwait, pw_ld);
 #endif
     fence_before();
     __threadfence();
