@@ -34,9 +34,11 @@ class MLEResult:
 
 def fit(ev: Evaluator, x, y, z, theta0=(0.01, 0.01, 0.01), bounds=((0.01, 2.0),) * 3, u_req: float = 1e-9,
         mode: int = MP_MAP_ADAPTIVE, policy: int = MP_COMM_AUTO, tol: float = 1e-9, maxfev: int = 500,
-        fixed_nu: float | None = None, log=None) -> MLEResult:
+        fixed_nu: float | None = None, log=None, cache: dict | None = None) -> MLEResult:
     """theta_hat = argmax l(theta).  `fixed_nu` fits (sigma^2, beta) only.  x, y, z: host numpy
-    arrays or device tensors (device tensors avoid the per-call host-to-device copy)."""
+    arrays or device tensors (device tensors avoid the per-call host-to-device copy).  `cache`: exact
+    {theta: l} values of an earlier identical run (the optimiser and the evaluation are deterministic,
+    so a replay retraces it and continues)."""
     from scipy.optimize import Bounds, minimize
 
     hist = []
@@ -47,8 +49,11 @@ def fit(ev: Evaluator, x, y, z, theta0=(0.01, 0.01, 0.01), bounds=((0.01, 2.0),)
 
     def obj(t):
         th = full(t)
-        rep = ev.eval(x, y, z, th, u_req=u_req, mode=mode, policy=policy)
-        ll = rep.loglik if math.isfinite(rep.loglik) else -PENALTY
+        if cache and th in cache:
+            ll = cache[th]
+        else:
+            rep = ev.eval(x, y, z, th, u_req=u_req, mode=mode, policy=policy)
+            ll = rep.loglik if math.isfinite(rep.loglik) else -PENALTY
         hist.append((th, ll))
         if log:
             log(th, ll)

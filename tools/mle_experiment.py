@@ -29,6 +29,15 @@ def main():
     n = int(sys.argv[1]) if len(sys.argv) > 1 else 40000
     modes = (sys.argv[2] if len(sys.argv) > 2 else "fp64,mp").split(",")
     maxfev = int(sys.argv[3]) if len(sys.argv) > 3 else 600
+    # replay: the exact (hex) history of an interrupted run of the same workload; COBYQA is deterministic and
+    # so is the evaluation, so the optimiser retraces it from the cache and continues live (one GPU call is
+    # limited to an hour; a C3 FP64-map MLE from the paper's start takes longer)
+    cache = {}
+    for path in sys.argv[4:]:
+        for line in open(path):
+            f = line.split()
+            if len(f) == 4 and f[0].startswith(("0x", "-0x")):
+                cache[tuple(float.fromhex(v) for v in f[:3])] = float.fromhex(f[3])
     nb = 2048
     theta_true = (1.0, 0.03, 0.5)
     x, y = synth.locations(n, 0)
@@ -45,10 +54,10 @@ def main():
         logf = open(f"gpurun_out/mle_n{n}_{name}.log", "w")
 
         def log(th, ll, logf=logf):
-            logf.write(f"{th[0]:.10f} {th[1]:.10f} {th[2]:.10f} {ll:.10f}\n")
+            logf.write(" ".join(float(v).hex() for v in (*th, ll)) + "\n")
             logf.flush()
 
-        r = fit(ev, dx, dy, dz, mode=mode, u_req=1e-9, maxfev=maxfev, log=log)
+        r = fit(ev, dx, dy, dz, mode=mode, u_req=1e-9, maxfev=maxfev, log=log, cache=cache)
         rep = ev.eval(dx, dy, dz, tuple(r.theta), mode=mode)
         out[name] = {"theta": list(r.theta), "loglik": r.loglik, "nfev": r.nfev, "seconds": time.time() - t0,
                      "tiles_fp64_fp32_fp16": list(rep.tiles), "message": r.message}
