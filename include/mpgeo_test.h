@@ -37,6 +37,10 @@ mp_status mp_bench_fp64_engine(int nb, int nt, int njobs, int nmod, int reps, fl
  * nmod moduli, the split CRT weights w_j = H_j + L_j of the nmod/2 paired moduli m_j = p_2j p_2j+1
  * and M = Mhl[0] + Mhl[1] (host pointers). */
 mp_status mp_test_crt_constants(int nmod, int K, int* bits, int* moduli, double* H, double* L, double* Mhl);
+/* The CRT engine's element reconstruction (crt_recon_bits, the same host/device function the GEMM
+   epilogue runs), evaluated on the host: R = n x (nmod/2) combined pair residues (row-major), e0[n]
+   exponents, neg = 1 for -X; out[n] = FP64 results.  Pinned on CPU against big-integer CRT. */
+mp_status mp_test_crt_recon(int nmod, int K, const uint32_t* R, const int* e0, int n, int neg, double* out);
 /* 1 if the tcgen05 kernels are compiled in, else 0. */
 int mp_tc_available(void);
 /* Correctly rounded sum of n doubles (host; the S of the precision rule). */

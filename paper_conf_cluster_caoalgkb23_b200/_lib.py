@@ -115,6 +115,7 @@ def _load() -> C.CDLL:
         "mp_test_crt_gemm": (i32, [vp, vp, i32, i32, i32, i32, i32, i32, i32]),
         "mp_bench_fp64_engine": (i32, [i32, i32, i32, i32, i32, C.POINTER(C.c_float)]),
         "mp_test_crt_constants": (i32, [i32, i32, C.POINTER(i32), C.POINTER(i32), dp, dp, dp]),
+        "mp_test_crt_recon": (i32, [i32, i32, C.POINTER(C.c_uint32), C.POINTER(i32), i32, i32, dp]),
     }
     for name, (res, args) in sig.items():
         f = getattr(lib, name)

@@ -59,14 +59,18 @@ static double u128_to_double(unsigned __int128 v) {  // correctly rounded enough
 }
 
 bool crt_constants(int nmod, int K, CrtConst* c) {
-    if (nmod < 2 || nmod > CRT_NMAX || (nmod & 1) || K < 1) return false;
+    if (nmod < 2 || nmod > CRT_NMAX || (nmod & 1) || K < 1 || K > 8192) return false;
     memset(c, 0, sizeof *c);
     c->nmod = nmod;
     unsigned __int128 M = 1;
     for (int t = 0; t < nmod; ++t) M *= (unsigned)kModuli[t];
-    const double log2M = log2(u128_to_double(M));
-    // largest b with 2b + log2(K) + 1 < log2(M)  (strict margin 0.05 bits)
-    c->bits = (int)floor((log2M - 1.0 - log2((double)K) - 0.05) / 2.0);
+    // largest b with K 2^{2b} <= 0.3 M (crt.h: uniqueness, and the margin of the FP32 quotient estimate)
+    {
+        const unsigned __int128 lim = M / 10 * 3;
+        int b = 0;
+        while (2 * (b + 1) + 13 < 128 && ((unsigned __int128)K << (2 * (b + 1))) <= lim) ++b;  // K <= 2^13
+        c->bits = b;
+    }
     if (c->bits < 8) return false;
     for (int t = 0; t < nmod; ++t) {
         const unsigned p = (unsigned)kModuli[t];
@@ -109,6 +113,45 @@ bool crt_constants(int nmod, int K, CrtConst* c) {
     c->Mh = ldexp((double)(uint64_t)(M >> sh), sh);
     c->Ml = u128_to_double(M & mask);
     c->invM = 1.0 / u128_to_double(M);
+    // integer + FP32 reconstruction constants (crt_recon_bits, crt.h)
+    c->ld = u128_bits(M) > 64 ? 1 : 0;
+    const int lsh = 32 * c->ld;
+    for (int t = 0; t < 3; ++t) c->Mw[t] = (uint32_t)((M >> lsh) >> (32 * t));
+    const double Md = u128_to_double(M);
+    unsigned __int128 Dr = 0;  // sum_j h_j w_j = Dq M + Dr, exact (shift-and-add modulo M; M < 2^126)
+    long long Dq = 0;
+    for (int j = 0; j < npair; ++j) {
+        const unsigned a = (unsigned)kModuli[2 * j], b = (unsigned)kModuli[2 * j + 1], m = a * b;
+        const unsigned __int128 Mj = M / m;
+        const unsigned mj = (unsigned)(Mj % m);
+        unsigned y = 0;
+        for (unsigned v = 1; v < m; ++v)
+            if ((unsigned long long)mj * v % m == 1) {
+                y = v;
+                break;
+            }
+        const unsigned __int128 w = Mj * y;
+        for (int t = 0; t < 3; ++t) c->W[j][t] = (uint32_t)((w >> lsh) >> (32 * t));
+        c->cw[j] = (float)(u128_to_double(w) / Md);
+        const unsigned h = m / 2;
+        c->hoff[j] = 8388608.0f + (float)h;
+        unsigned __int128 r = 0;
+        long long qq = 0;
+        for (int bit = 15; bit >= 0; --bit) {
+            r <<= 1;
+            qq <<= 1;
+            if (r >= M) r -= M, ++qq;
+            if ((h >> bit) & 1u) {
+                r += w;
+                if (r >= M) r -= M, ++qq;
+            }
+        }
+        Dr += r;
+        if (Dr >= M) Dr -= M, ++qq;
+        Dq += qq;
+    }
+    c->Dq = (int)Dq;
+    c->fD = (float)(u128_to_double(Dr) / Md);
     return true;
 }
 
@@ -363,10 +406,6 @@ __device__ __forceinline__ void tmem_wait(uint32_t (&r)[32]) {
 #pragma unroll
     for (int i = 0; i < 32; ++i) asm volatile("" : "+r"(r[i]));
 }
-// 2^e as a double from its exponent bits (normal range), ldexp otherwise (ldexp costs ~10x more)
-__device__ __forceinline__ double exp2i(int e) {
-    return (e >= -1022 && e <= 1023) ? __hiloint2double((e + 1023) << 20, 0) : ldexp(1.0, e);
-}
 // canonical residue of a modulo p in [0, p), |a| <= 2^27 (the INT32 accumulator bound K 2^14 for
 // K <= 8192; |(r_b - r_a) ia| < 2^16): exact Barrett reduction.  a' = a + p 2^20 is a multiple-of-p
 // shift of a in [0, 2^29); with m = ceil(2^38/p), floor(a' m / 2^38) = floor(a'/p) because the excess
@@ -550,7 +589,7 @@ __global__ void __launch_bounds__(THREADS, 1) crt_gemm_kernel(const __grid_const
         // the previous tile, whose reconstruction is pending
         bool pv = false;
         int pv_crow0 = 0, pv_ccol0 = 0, pv_tab = 0;
-        double pv_rs = 0.0;
+        int pv_e0 = 0;  // row exponent e_i - 2b of the pending tile (C += X 2^(e_i + f_j - 2b))
         const int* pv_ecol = nullptr;
         const int ew = warp - 4;
         if (lane < 16) scr_free[ew][lane] = (uint8_t)(NP * 16 + lane);  // the spare blocks
@@ -590,21 +629,18 @@ __global__ void __launch_bounds__(THREADS, 1) crt_gemm_kernel(const __grid_const
                 PROF_ADD(pw_ld);
             }
 #endif
-            double sh[8], sl[8];
+            // integer + FP32 reconstruction (crt_recon_bits, crt.h): no FP64 instruction while the
+            // tensor core runs
+            uint64_t o[8];
 #pragma unroll
-            for (int v = 0; v < 8; ++v) sh[v] = sl[v] = 0.0;
+            for (int v = 0; v < 8; ++v) {
+                uint32_t R[NP];
 #pragma unroll
-            for (int jj = 0; jj < NP; ++jj) {
-                const double Hj = p.c.H[jj], Lj = p.c.L[jj];
-                const uint32_t wv[4] = {w[jj].x, w[jj].y, w[jj].z, w[jj].w};
-#pragma unroll
-                for (int v = 0; v < 8; ++v) {
-                    // 2^52 + R exactly (R in the low mantissa bits), minus 2^52
-                    const uint32_t Rv = (v & 1) ? (wv[v >> 1] >> 16) : (wv[v >> 1] & 0xffffu);
-                    const double d = __hiloint2double(0x43300000, (int)Rv) - 4503599627370496.0;
-                    sh[v] = fma(d, Hj, sh[v]);  // exact
-                    sl[v] = fma(d, Lj, sl[v]);
+                for (int jj = 0; jj < NP; ++jj) {
+                    const uint32_t wv = (v >> 1) == 0 ? w[jj].x : (v >> 1) == 1 ? w[jj].y : (v >> 1) == 2 ? w[jj].z : w[jj].w;
+                    R[jj] = (v & 1) ? (wv >> 16) : (wv & 0xffffu);
                 }
+                o[v] = crt_recon_bits<NP>(R, p.c, pv_e0 + __ldg(pv_ecol + col0 + v), p.store ? 0u : 1u);
             }
             // stage -out in the warp's 32 x 8 box (64-byte swizzle: 16-byte chunk k of row l at
             // k ^ ((l >> 1) & 3)); one lane reduces the box into C through the TMA unit
@@ -615,17 +651,10 @@ __global__ void __launch_bounds__(THREADS, 1) crt_gemm_kernel(const __grid_const
                 PROF_ADD(pw_stgwait);
                 __syncwarp();
             }
-            double o[8];
-#pragma unroll
-            for (int v = 0; v < 8; ++v) {
-                const double qm = rint((sh[v] + sl[v]) * p.c.invM);
-                const double X = fma(-qm, p.c.Mh, sh[v]) + fma(-qm, p.c.Ml, sl[v]);
-                o[v] = (p.store ? X : -X) * pv_rs * exp2i(__ldg(pv_ecol + col0 + v) - p.c.bits);
-            }
 #pragma unroll
             for (int v = 0; v < 8; v += 2) {
                 const uint32_t a = sb + (uint32_t)lane * 64u + ((uint32_t)((v >> 1) ^ ((lane >> 1) & 3)) << 4);
-                asm volatile("st.shared.v2.f64 [%0], {%1, %2};" ::"r"(a), "d"(o[v]), "d"(o[v + 1]) : "memory");
+                asm volatile("st.shared.v2.b64 [%0], {%1, %2};" ::"r"(a), "l"(o[v]), "l"(o[v + 1]) : "memory");
             }
             asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
             __syncwarp();
@@ -764,7 +793,7 @@ __global__ void __launch_bounds__(THREADS, 1) crt_gemm_kernel(const __grid_const
             const int grow = bi * 256 + (int)crank * BM + r;  // row inside the tile
             pv = true;
             pv_tab = ct;
-            pv_rs = ldexp(1.0, p.exps[jb.m * p.nb + grow] - p.c.bits);
+            pv_e0 = p.exps[jb.m * p.nb + grow] - 2 * p.c.bits;
             pv_ecol = p.exps + (size_t)jb.n * p.nb + bj * BN + h * 128;
             pv_crow0 = (int)(((const char*)jb.C - (const char*)p.cbase) / ((size_t)p.nb * 8)) + bi * 256 +
                        (int)crank * BM + q * 32;

@@ -3,6 +3,7 @@
 #include <math.h>
 #include <stdio.h>
 #include <stdlib.h>
+#include <string.h>
 #include <algorithm>
 #include <vector>
 
@@ -11,6 +12,19 @@
 #include "crt.h"
 
 using namespace mpgeo;
+
+namespace mpgeo {
+template <int NP>
+static void recon_rows(const CrtConst& c, const uint32_t* R, const int* e0, int n, int neg, double* out) {
+    for (int i = 0; i < n; ++i) {
+        uint32_t r[NP];
+        for (int j = 0; j < NP; ++j) r[j] = R[(size_t)i * NP + j];
+        const uint64_t b = crt_recon_bits<NP>(r, c, e0[i], (uint32_t)neg);
+        memcpy(out + i, &b, 8);
+    }
+}
+
+}  // namespace mpgeo
 
 extern "C" {
 
@@ -249,6 +263,16 @@ mp_status mp_bench_fp64_engine(int nb, int nt, int njobs, int nmod, int reps, fl
     cudaEventDestroy(e1);
     cudaEventDestroy(e2);
     return (e == cudaSuccess && es == cudaSuccess) ? MP_OK : MP_ERR_CUDA;
+}
+
+mp_status mp_test_crt_recon(int nmod, int K, const uint32_t* R, const int* e0, int n, int neg, double* out) {
+    CrtConst c;
+    if (!crt_constants(nmod, K, &c)) return MP_ERR_ARG;
+    if (nmod == 16) mpgeo::recon_rows<8>(c, R, e0, n, neg, out);
+    else if (nmod == 14) mpgeo::recon_rows<7>(c, R, e0, n, neg, out);
+    else if (nmod == 8) mpgeo::recon_rows<4>(c, R, e0, n, neg, out);
+    else return MP_ERR_ARG;
+    return MP_OK;
 }
 
 /* Host constants of the CRT engine (pinned on CPU against big-integer arithmetic). */

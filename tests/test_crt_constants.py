@@ -5,10 +5,12 @@ exact big-integer arithmetic — the Chinese remainder theorem itself, not a ret
     (w_j == 1 mod m_j, == 0 mod m_i, i != j) up to the rounding of L_j (< 2^-53 relative), and H_j is
     a multiple of 2^sh with < 2^33 units (so sum_j R_j H_j is exact in FP64 for R_j < 2^16);
   * the operand bit budget b keeps K 2^{2b} < M/2 (the reconstructed integer is unique);
-  * a pure-Python model of the device epilogue (modulus reduction, pair combination
-    R = r_a + a((r_b - r_a) a^-1 mod b), FP64 reconstruction with exactly the kernel's operations)
-    returns sum_k x'_k y'_k to within its final FP64 rounding + 2^64 (relative 2^-58 of the operand
-    scale K 2^{2b}) for random full-budget integer dot products.
+  * the element reconstruction the GEMM epilogue runs (crt_recon_bits, integer + FP32 arithmetic;
+    called on the host through mp_test_crt_recon) returns X 2^e0 for every integer X with
+    |X| <= K 2^{2b} given only its pair residues, to within one FP64 rounding + 2^(51.6 + e0) (the
+    dropped low limb, ld = 1) — exact quotient included — checked against Python big integers on
+    random, extreme (+-K 2^{2b}, the 0.3 M edge), tiny and zero values;
+  * the bit budget b is the largest with K 2^{2b} <= 0.3 M (the quotient estimate's margin).
 No GPU needed (the constants are host code of libmpgeo)."""
 import ctypes as C
 import math
@@ -49,62 +51,50 @@ def test_crt_constants_exact(nmod, K):
         assert hh % (1 << sh) == 0 and (hh >> sh) < (1 << 33)
         assert abs(Fraction(w - hh) - Fraction(L[j])) <= Fraction(w - hh) * Fraction(1, 1 << 52) + 1
     assert K * 4**bits < M // 2
-    assert not (K * 4 ** (bits + 1) * 2 ** 0.05 < M // 2)
+    assert 10 * K * 4**bits <= 3 * M and not (10 * K * 4 ** (bits + 1) <= 3 * M)
 
 
-def _mod_canon(a, p):
-    """Device mod_canon: q = round(a/p) by a 32-bit multiply-high, then one correction."""
-    mq = ((1 << 32) + p // 2) // p
-    q = (a * mq + (1 << 31)) >> 32
-    r = a - q * p
-    assert -p // 2 - 1 <= r <= p // 2 + 1
-    return r + p if r < 0 else r
+def _recon(nmod, K, X, e0, neg=0):
+    """crt_recon_bits on the host for integers X (Python ints): pair residues in, FP64 out."""
+    from paper_conf_cluster_caoalgkb23_b200._lib import lib
+    _, p, _, _, _ = _consts(nmod, K)
+    m = [p[2 * j] * p[2 * j + 1] for j in range(nmod // 2)]
+    R = (C.c_uint32 * (len(X) * len(m)))(*[x % mj for x in X for mj in m])
+    E = (C.c_int * len(X))(*e0)
+    out = (C.c_double * len(X))()
+    assert lib.mp_test_crt_recon(nmod, K, R, E, len(X), neg, out) == 0
+    return list(out)
 
 
-def _device_epilogue(accs, p, H, L, Mh, Ml):
-    """Residue reduction, pair combination and FP64 reconstruction exactly as crt_gemm_kernel
-    (fma = exact product + one rounding, emulated with Fraction)."""
-    def fma(a, b, c):
-        return float(Fraction(a) * Fraction(b) + Fraction(c))
-    sh = sl = 0.0
-    for j in range(len(p) // 2):
-        a, b = p[2 * j], p[2 * j + 1]
-        ra = _mod_canon(accs[2 * j], a)
-        rb = _mod_canon(accs[2 * j + 1], b)
-        tt = _mod_canon((rb - ra) * pow(a, -1, b), b)
-        R = ra + a * tt
-        assert 0 <= R < a * b
-        sh = fma(float(R), H[j], sh)
-        sl = fma(float(R), L[j], sl)
-    invM = 1.0 / float(math.prod(p))
-    q = float(round((sh + sl) * invM))
-    return fma(-q, Mh, sh) + fma(-q, Ml, sl)
+@pytest.mark.parametrize("nmod,K", [(16, 2048), (16, 512), (14, 2048), (8, 2048)])
+def test_crt_reconstruction_exact_to_final_rounding(nmod, K):
+    bits, p, _, _, _ = _consts(nmod, K)
+    M = math.prod(p)
+    Xmax = K * 4**bits
+    ld = 1 if M.bit_length() > 64 else 0
+    rng = np.random.default_rng(7 + nmod)
+    X = [0, 1, -1, Xmax, -Xmax, Xmax - 1, -(Xmax - 1), 3 * M // 10, -(3 * M // 10)]
+    X += [s * (1 << k) + int(rng.integers(0, 1 << 20)) for k in range(0, Xmax.bit_length(), 3) for s in (1, -1)]
+    X += [int.from_bytes(rng.bytes(16), "little") % (2 * Xmax + 1) - Xmax for _ in range(3000)]
+    # quotient-estimate stress: X near the integer multiples' edges +-0.3 M (S/M = q +- 0.3)
+    X += [3 * M // 10 - int(rng.integers(0, 1 << 40)) for _ in range(200)]
+    X += [-(3 * M // 10) + int(rng.integers(0, 1 << 40)) for _ in range(200)]
+    e0 = [int(v) for v in rng.integers(-2 * bits - 200, -2 * bits + 100, len(X))]
+    for neg in (0, 1):
+        got = _recon(nmod, K, X, e0, neg)
+        for x, e, g in zip(X, e0, got):
+            exact = Fraction(-x if neg else x) * Fraction(2) ** e
+            tol = abs(exact) * Fraction(1, 1 << 52) + (Fraction(2) ** (e + 52) if ld else 0)
+            assert abs(Fraction(g) - exact) <= tol, (nmod, x, e, g, float(exact))
+            if x == 0:
+                assert g == 0.0
 
 
-def test_crt_epilogue_model_exact_to_final_rounding():
+def test_crt_reconstruction_flushes_below_fp64_range():
     nmod, K = 16, 2048
-    bits, p, H, L, (Mh, Ml) = _consts(nmod, K)
-    rng = np.random.default_rng(5)
-    worst = 0.0
-    for trial in range(200):
-        k = 64
-        x = [int(v) >> (62 - bits) for v in rng.integers(-(1 << 62), 1 << 62, k)]
-        y = [int(v) >> (62 - bits) for v in rng.integers(-(1 << 62), 1 << 62, k)]
-        if trial % 3 == 0:
-            y = [abs(v) * (1 if a >= 0 else -1) for v, a in zip(y, x)]  # no cancellation
-        X = sum(a * b for a, b in zip(x, y)) * (K // k)
-        # INT32 accumulators of the residue GEMMs: any value == X (mod p) with |acc| <= K 128^2
-        accs = []
-        for q in p:
-            r = X % q
-            r = r - q if r > 127 else r
-            accs.append(r + q * int(rng.integers(-(K * 128 * 128) // q // 2, (K * 128 * 128) // q // 2)))
-        got = _device_epilogue(accs, p, H, L, Mh, Ml)
-        # error: the L-part FP64 sums (< 2^64 absolute) plus the final rounding of X
-        assert abs(Fraction(got) - X) <= Fraction(abs(X)) * Fraction(1, 1 << 52) + (1 << 64), (trial, got, X)
-        worst = max(worst, float(abs(Fraction(got) - X)) / (K * 4.0**bits))
-    # relative to the operand scale K 2^(2b): at most the final rounding, far below an FP64 GEMM's K u = 2^-42
-    assert worst <= 2.0**-52
+    bits, _, _, _, _ = _consts(nmod, K)
+    got = _recon(nmod, K, [12345, -12345], [-1300, -1300])
+    assert got == [0.0, 0.0]
 
 
 def test_exact_barrett_reduction_of_the_epilogue():
