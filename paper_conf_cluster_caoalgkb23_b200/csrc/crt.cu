@@ -106,6 +106,7 @@ bool crt_constants(int nmod, int K, CrtConst* c) {
         if (!y) return false;
         const unsigned __int128 w = Mj * y;  // < M
         c->ia[j] = (int)ia;
+        c->shoup[j] = (unsigned)(((unsigned long long)ia << 32) / b);  // floor(ia 2^32 / b)
         c->mpair[j] = (int)m;
         c->H[j] = ldexp((double)(uint64_t)(w >> sh), sh);  // exact (< 2^33 units)
         c->L[j] = u128_to_double(w & mask);
@@ -230,6 +231,10 @@ constexpr uint32_t TMEM_COLS = 512;  // two 256-column accumulators
 // operand consecutive jobs share), 2 evict_last for A and B
 #ifndef CRT_L2HINT
 #define CRT_L2HINT 0
+#endif
+// 1: the first scratch group of each pair step's reconstruction is loaded before the residue steps
+#ifndef CRT_EARLY
+#define CRT_EARLY 0
 #endif
 // instruction descriptor: D = S32 (2 << 4), A = B = signed int8 (1 << 7, 1 << 10), K-major,
 // N >> 3 at bit 17, M >> 4 at bit 24 (M = 256 for the pair)
@@ -688,7 +693,18 @@ __global__ void __launch_bounds__(THREADS, 1) crt_gemm_kernel(const __grid_const
             const int ct = it_tile & 1;  // this tile's block table
             for (int jj = 0; jj < NP; ++jj) {
                 const int j = (j0 + jj) & (NP - 1);  // moduli pair (phase-rotated order)
-                if (pv) prefetch_groups((jj * 16) / NP, ((jj + 1) * 16) / NP);
+                // pending tile: L2 prefetch one pair step ahead, and the first group of this step's
+                // reconstruction loaded into registers now (its latency hides behind the residue steps)
+                uint4 wa[NP];
+                if (pv) {
+                    if (CRT_EARLY) {
+                        if (jj == 0) prefetch_groups(0, 16 / NP);
+                        if (jj + 1 < NP) prefetch_groups(((jj + 1) * 16) / NP, ((jj + 2) * 16) / NP);
+                        load_group((jj * 16) / NP, wa);
+                    } else {
+                        prefetch_groups((jj * 16) / NP, ((jj + 1) * 16) / NP);
+                    }
+                }
                 // this pair's 16 destination blocks: those the last reconstruction step freed (the
                 // first tile of the CTA takes the blocks in order)
                 if (lane < 16) scr_tab[ew][ct][j * 16 + lane] = pv ? scr_free[ew][lane] : (uint8_t)(j * 16 + lane);
@@ -712,6 +728,11 @@ __global__ void __launch_bounds__(THREADS, 1) crt_gemm_kernel(const __grid_const
                         uint32_t (&vc)[32] = (c & 1) ? v1 : v0;
                         uint32_t (&vn)[32] = (c & 1) ? v0 : v1;
                         if (c < 3) tmem_ld32_nowait(tmem + tl + buf * (uint32_t)BN + (uint32_t)((c + 1) * 32), vn);
+                        if (c == 3) {  // the whole accumulator is in registers: release it to the MMA now
+                            fence_before();
+                            __syncwarp();
+                            if (lane == 0) mbar_arrive_cluster_relaxed(ae0 + buf * 8u);
+                        }
 #pragma unroll
                         for (int k = 0; k < 8; ++k) {
                             const uint32_t b0 = (uint32_t)mod_canon((int)vc[4 * k], pa, mqa);
@@ -722,9 +743,6 @@ __global__ void __launch_bounds__(THREADS, 1) crt_gemm_kernel(const __grid_const
                         }
                         if (c < 3) tmem_wait(vn);
                     }
-                    fence_before();
-                    __syncwarp();
-                    if (lane == 0) mbar_arrive_cluster_relaxed(ae0 + buf * 8u);
                     ++g;
                     PROF_ADD(pw_resid);
                 }
@@ -736,8 +754,8 @@ __global__ void __launch_bounds__(THREADS, 1) crt_gemm_kernel(const __grid_const
                     PROF_ADD(pw_accfull); }
                     PROF_T0();
                     fence_after();
-                    const int pa = p.c.p[2 * j], pb = p.c.p[2 * j + 1], ia = p.c.ia[j];
-                    const unsigned mqb = p.c.bm[2 * j + 1];
+                    const unsigned pa = (unsigned)p.c.p[2 * j], pb = (unsigned)p.c.p[2 * j + 1], ia = (unsigned)p.c.ia[j];
+                    const unsigned shb = p.c.shoup[j], offb = pb << 21;
                     uint32_t v0[32], v1[32];
                     tmem_ld32_nowait(tmem + tl + buf * (uint32_t)BN, v0);
                     tmem_wait(v0);
@@ -746,6 +764,11 @@ __global__ void __launch_bounds__(THREADS, 1) crt_gemm_kernel(const __grid_const
                         uint32_t (&vc)[32] = (c & 1) ? v1 : v0;
                         uint32_t (&vn)[32] = (c & 1) ? v0 : v1;
                         if (c < 3) tmem_ld32_nowait(tmem + tl + buf * (uint32_t)BN + (uint32_t)((c + 1) * 32), vn);
+                        if (c == 3) {  // accumulator fully in registers: release it
+                            fence_before();
+                            __syncwarp();
+                            if (lane == 0) mbar_arrive_cluster_relaxed(ae0 + buf * 8u);
+                        }
                         uint32_t pk[16];
 #pragma unroll
                         for (int k = 0; k < 16; ++k) {
@@ -753,10 +776,13 @@ __global__ void __launch_bounds__(THREADS, 1) crt_gemm_kernel(const __grid_const
 #pragma unroll
                             for (int u = 0; u < 2; ++u) {
                                 const int e = 2 * k + u;
-                                const int rb = mod_canon((int)vc[e], pb, mqb);
-                                const int rav = (int)((ra[c][e >> 2] >> (8 * (e & 3))) & 0xffu);
-                                const int tt = mod_canon((rb - rav) * ia, pb, mqb);
-                                R2[u] = (uint32_t)(rav + pa * tt);
+                                // t = ((acc_b - r_a) a^-1) mod b by Shoup's multiplication: x = acc_b - r_a +
+                                // b 2^21 in [0, 2^32); q = floor(x shoup / 2^32); x ia - q b in [0, 2b)
+                                const uint32_t rav = (ra[c][e >> 2] >> (8 * (e & 3))) & 0xffu;
+                                const uint32_t x = vc[e] - rav + offb;
+                                const uint32_t r2 = x * ia - __umulhi(x, shb) * pb;
+                                const uint32_t tt = min(r2, r2 - pb);
+                                R2[u] = rav + pa * tt;
                             }
                             pk[k] = R2[0] | (R2[1] << 16);
                         }
@@ -766,9 +792,6 @@ __global__ void __launch_bounds__(THREADS, 1) crt_gemm_kernel(const __grid_const
                                 make_uint4(pk[4 * e], pk[4 * e + 1], pk[4 * e + 2], pk[4 * e + 3]);
                         if (c < 3) tmem_wait(vn);
                     }
-                    fence_before();
-                    __syncwarp();
-                    if (lane == 0) mbar_arrive_cluster_relaxed(ae0 + buf * 8u);
                     ++g;
                     PROF_ADD(pw_resid);
                 }
@@ -776,8 +799,8 @@ __global__ void __launch_bounds__(THREADS, 1) crt_gemm_kernel(const __grid_const
                 if (pv) {
                     PROF_T0();
                     const int g0 = (jj * 16) / NP, g1 = ((jj + 1) * 16) / NP;
-                    uint4 wa[NP], wb[NP];
-                    load_group(g0, wa);
+                    uint4 wb[NP];
+                    if (!CRT_EARLY) load_group(g0, wa);
                     for (int gi = g0; gi < g1; gi += 2) {
                         if (gi + 1 < g1) load_group(gi + 1, wb);
                         recon(gi, wa);

@@ -18,6 +18,7 @@ struct CrtConst {
     unsigned bm[CRT_NMAX];     // ceil(2^38 / p): exact Barrett floor((a + p 2^20) / p) for |a| <= 2^27 (crt.cu)
     double invp[CRT_NMAX];     // 1/p (FP64, for the operand residues)
     int ia[CRT_NMAX / 2];      // p_2j^-1 mod p_2j+1
+    unsigned shoup[CRT_NMAX / 2];  // floor(ia_j 2^32 / p_2j+1): Shoup's modular multiplication by ia_j
     int mpair[CRT_NMAX / 2];   // m_j = p_2j p_2j+1
     double H[CRT_NMAX / 2];    // w_j = (M/m_j) ((M/m_j)^-1 mod m_j) = H_j + L_j, H_j a multiple of 2^sh
     double L[CRT_NMAX / 2];    //   with < 2^33 units (sum_j R_j H_j exact), L_j < 2^sh

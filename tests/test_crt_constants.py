@@ -115,3 +115,31 @@ def test_exact_barrett_reduction_of_the_epilogue():
         q = ((ap * np.uint64(m)) >> np.uint64(32)) >> np.uint64(6)  # __umulhi(a', m) >> 6
         r = (ap - q * np.uint64(p)).astype(np.int64)
         assert np.array_equal(r, np.mod(a, p)), p
+
+
+def test_shoup_pair_combination_of_the_epilogue():
+    """crt.cu residue step of the second modulus b of each pair: t = ((acc_b - r_a) a^-1) mod b by Shoup's
+    multiplication — x = acc_b - r_a + b 2^21 (in [0, 2^32) for |acc_b| <= 2^27, r_a < 256),
+    r = x ia - floor(x floor(ia 2^32 / b) / 2^32) b (mod 2^32) in [0, 2b), t = min(r, r - b) unsigned —
+    equals the exact modular value for every pair of the engine (both range ends + random samples)."""
+    moduli = [256, 255, 253, 251, 247, 241, 239, 233, 229, 227, 223, 217, 211, 199, 197, 193]
+    rng = np.random.default_rng(1)
+    lim = 1 << 27
+    acc = np.concatenate([np.arange(-lim, -lim + 20000), np.arange(-20000, 20000), np.arange(lim - 20000, lim + 1),
+                          rng.integers(-lim, lim + 1, 300000)]).astype(np.int64)
+    ra = rng.integers(0, 256, acc.size).astype(np.int64)
+    M32 = np.uint64(0xFFFFFFFF)
+    for j in range(8):
+        a, b = moduli[2 * j], moduli[2 * j + 1]
+        ia = pow(a, -1, b)
+        ra_j = ra % a
+        sh = (ia << 32) // b
+        x = (acc - ra_j + (b << 21)).astype(np.uint64)
+        assert int(x.min()) >= 0 and int(x.max()) < (1 << 32)
+        q = (x * np.uint64(sh)) >> np.uint64(32)
+        r = (x * np.uint64(ia) - q * np.uint64(b)) & M32
+        assert int(r.max()) < 2 * b
+        t = np.minimum(r, (r - np.uint64(b)) & M32).astype(np.int64)
+        assert np.array_equal(t, np.mod((acc - ra_j) * ia, b)), (a, b)
+        R = ra_j + a * t  # the combined pair residue
+        assert np.array_equal(R % a, np.mod(acc * 0 + ra_j, a)) and np.array_equal(R % b, np.mod(acc, b))
