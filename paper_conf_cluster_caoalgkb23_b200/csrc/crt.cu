@@ -221,11 +221,22 @@ constexpr int STAGES = 5;  // 5 x 32 KB: with the C staging (32 KB) and the scra
 constexpr int RING = 4;  // tile-index ring depth (dynamic scheduler)
 // C update staging: per epilogue warp two 32 x 8 FP64 boxes (2 KB, 64-byte swizzle) reduced into C
 // by the TMA unit (cp.reduce.async.bulk.tensor .add on the FP64 C map)
+// epilogue warps: 8 (two per TMEM lane quarter, 128 columns each) or 16 (four per quarter, 64 columns)
+#ifndef CRT_EPI
+#define CRT_EPI 8
+#endif
+constexpr int EPI_WARPS = CRT_EPI;
+constexpr int PARTS = EPI_WARPS / 4;     // column parts of the 256-column accumulator
+constexpr int PCOLS = BN / PARTS;        // columns per epilogue warp
+constexpr int CHUNKS = PCOLS / 32;       // 32-column TMEM loads per accumulator and warp
+constexpr int GROUPS = PCOLS / 8;        // 8-column reconstruction groups per warp and tile
 constexpr int STG_BOX = 32 * 8 * 8;
-constexpr int STG_WARP = 2 * STG_BOX;
-constexpr int SMEM = STAGES * STAGE_BYTES + 8 * STG_WARP + 1024;
-constexpr int EPI_WARPS = 8;
+constexpr int NSTG = EPI_WARPS == 8 ? 2 : 1;  // staging boxes per warp (shared-memory budget)
+constexpr int STG_WARP = NSTG * STG_BOX;
+constexpr int SMEM = STAGES * STAGE_BYTES + EPI_WARPS * STG_WARP + 1024;
 constexpr int THREADS = (4 + EPI_WARPS) * 32;
+constexpr int SCR_BLOCKS_P = CRT_NMAX / 2 * GROUPS + GROUPS;  // blocks per column part (a tile + one step's spare)
+static_assert(PARTS * SCR_BLOCKS_P * CRT_SCR_BLOCK <= (int)CRT_SLOT_BYTES, "scratch slot too small");
 constexpr uint32_t TMEM_COLS = 512;  // two 256-column accumulators
 // L2 eviction priority of the operand loads (residue planes): 0 normal, 1 evict_last for A (the row
 // operand consecutive jobs share), 2 evict_last for A and B
@@ -235,6 +246,11 @@ constexpr uint32_t TMEM_COLS = 512;  // two 256-column accumulators
 // 1: the first scratch group of each pair step's reconstruction is loaded before the residue steps
 #ifndef CRT_EARLY
 #define CRT_EARLY 0
+#endif
+// 1: reconstructed residue-scratch lines are discarded from L2 (discard.global.L2) instead of being
+// evicted dirty to HBM
+#ifndef CRT_DISCARD
+#define CRT_DISCARD 1
 #endif
 // instruction descriptor: D = S32 (2 << 4), A = B = signed int8 (1 << 7, 1 << 10), K-major,
 // N >> 3 at bit 17, M >> 4 at bit 24 (M = 256 for the pair)
@@ -391,7 +407,7 @@ __device__ __forceinline__ void tile_coords(const CrtParams& p, int t, int& job,
 // residues R (uint16) of one moduli pair and one 8-column group: a warp's 32 rows of one block are
 // 512 contiguous bytes (coalesced stores and loads)
 __device__ __forceinline__ uint32_t scr_off(int b, int h, int r) {
-    return ((uint32_t)(h * CRT_SCR_BLOCKS + b) * 128u + (uint32_t)r) * 16u;
+    return ((uint32_t)(h * SCR_BLOCKS_P + b) * 128u + (uint32_t)r) * 16u;
 }
 
 __device__ __forceinline__ void tmem_ld32_nowait(uint32_t taddr, uint32_t (&r)[32]) {
@@ -439,8 +455,8 @@ __global__ void __launch_bounds__(THREADS, 1) crt_gemm_kernel(const __grid_const
     __shared__ __align__(8) uint64_t ring_full[RING], ring_empty[RING];
     // per epilogue warp: scratch block of (moduli pair j, group gi) for the two tiles in flight, and
     // the 16 blocks the last reconstruction step freed (the next residue step's destinations)
-    __shared__ uint8_t scr_tab[EPI_WARPS][2][CRT_NMAX / 2 * 16];
-    __shared__ uint8_t scr_free[EPI_WARPS][16];
+    __shared__ uint8_t scr_tab[EPI_WARPS][2][CRT_NMAX / 2 * GROUPS];
+    __shared__ uint8_t scr_free[EPI_WARPS][GROUPS];
 
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     const uint32_t crank = cluster_rank();
@@ -585,7 +601,7 @@ __global__ void __launch_bounds__(THREADS, 1) crt_gemm_kernel(const __grid_const
         const int q = (warp - 4) & 3, h = (warp - 4) >> 2;
         const int r = q * 32 + lane;  // CTA row = TMEM lane
         uint8_t* const scr0 = p.scratch + (size_t)slot_sh * CRT_SLOT_BYTES;
-        const uint32_t tl = ((uint32_t)(q * 32) << 16) + (uint32_t)(h * 128);
+        const uint32_t tl = ((uint32_t)(q * 32) << 16) + (uint32_t)(h * PCOLS);
         const uint32_t ae0 = cluster_addr(su32(&acc_empty[0]), 0);
         const uint32_t stg_s = su32(smem + STAGES * STAGE_BYTES + (warp - 4) * STG_WARP);
         constexpr int NP = N / 2;
@@ -597,19 +613,29 @@ __global__ void __launch_bounds__(THREADS, 1) crt_gemm_kernel(const __grid_const
         int pv_e0 = 0;  // row exponent e_i - 2b of the pending tile (C += X 2^(e_i + f_j - 2b))
         const int* pv_ecol = nullptr;
         const int ew = warp - 4;
-        if (lane < 16) scr_free[ew][lane] = (uint8_t)(NP * 16 + lane);  // the spare blocks
+        if (lane < GROUPS) scr_free[ew][lane] = (uint8_t)(NP * GROUPS + lane);  // the spare blocks
         __syncwarp();
 
         // reconstruct groups gi (8 columns each) of the pending tile: X = sum_j R_j w_j - q M, scaled
         auto load_group = [&](int gi, uint4 (&w)[NP]) {
 #pragma unroll
             for (int jj = 0; jj < NP; ++jj)  // last use of each block
-                w[jj] = __ldcs((const uint4*)(scr0 + scr_off(scr_tab[ew][pv_tab][jj * 16 + gi], h, r)));
+                w[jj] = __ldcs((const uint4*)(scr0 + scr_off(scr_tab[ew][pv_tab][jj * GROUPS + gi], h, r)));
         };
         // after reconstructing groups [g0, g0 + 16/NP) of the pending tile their 16 blocks are free
         auto free_groups = [&](int g0) {
             __syncwarp();
-            if (lane < 16) scr_free[ew][lane] = scr_tab[ew][pv_tab][(lane % NP) * 16 + g0 + lane / NP];
+            if (CRT_DISCARD) {
+                // the residues are dead once read: drop this warp's 4 lines (32 rows x 16 B) of every freed
+                // block from L2 without writing them back (otherwise each is evicted dirty to HBM later)
+                for (int i = lane; i < GROUPS * 4; i += 32) {
+                    const int blk = scr_tab[ew][pv_tab][((i >> 2) % NP) * GROUPS + g0 + (i >> 2) / NP];
+                    asm volatile("discard.global.L2 [%0], 128;" ::"l"(scr0 + scr_off(blk, h, q * 32 + (i & 3) * 8)) : "memory");
+                }
+                asm volatile("fence.acq_rel.cta;" ::: "memory");
+                __syncwarp();
+            }
+            if (lane < GROUPS) scr_free[ew][lane] = scr_tab[ew][pv_tab][(lane % NP) * GROUPS + g0 + lane / NP];
             __syncwarp();
         };
         // L2 prefetch of groups [g0, g1) of the pending tile (all 128 rows of this column half: one
@@ -618,7 +644,7 @@ __global__ void __launch_bounds__(THREADS, 1) crt_gemm_kernel(const __grid_const
             if (q == 0 && lane == 0)
                 for (int gi = g0; gi < g1; ++gi)
                     for (int jj = 0; jj < NP; ++jj) {
-                        const uint8_t* src = scr0 + scr_off(scr_tab[ew][pv_tab][jj * 16 + gi], h, 0);
+                        const uint8_t* src = scr0 + scr_off(scr_tab[ew][pv_tab][jj * GROUPS + gi], h, 0);
                         asm volatile("cp.async.bulk.prefetch.L2.global [%0], 2048;" ::"l"(src) : "memory");
                     }
         };
@@ -634,32 +660,37 @@ __global__ void __launch_bounds__(THREADS, 1) crt_gemm_kernel(const __grid_const
                 PROF_ADD(pw_ld);
             }
 #endif
-            // integer + FP32 reconstruction (crt_recon_bits, crt.h): no FP64 instruction while the
-            // tensor core runs
-            uint64_t o[8];
-#pragma unroll
-            for (int v = 0; v < 8; ++v) {
-                uint32_t R[NP];
-#pragma unroll
-                for (int jj = 0; jj < NP; ++jj) {
-                    const uint32_t wv = (v >> 1) == 0 ? w[jj].x : (v >> 1) == 1 ? w[jj].y : (v >> 1) == 2 ? w[jj].z : w[jj].w;
-                    R[jj] = (v & 1) ? (wv >> 16) : (wv & 0xffffu);
-                }
-                o[v] = crt_recon_bits<NP>(R, p.c, pv_e0 + __ldg(pv_ecol + col0 + v), p.store ? 0u : 1u);
-            }
             // stage -out in the warp's 32 x 8 box (64-byte swizzle: 16-byte chunk k of row l at
-            // k ^ ((l >> 1) & 3)); one lane reduces the box into C through the TMA unit
-            const uint32_t sb = stg_s + (nred & 1u) * (uint32_t)STG_BOX;
-            if (nred >= 2) {
+            // k ^ ((l >> 1) & 3)); one lane reduces the box into C through the TMA unit.  The box is
+            // free once the TMA unit has read the reduce-add issued NSTG groups ago.
+            const uint32_t sb = stg_s + (nred % NSTG) * (uint32_t)STG_BOX;
+            if (nred >= NSTG) {
                 PROF_T0();
-                if (lane == 0) asm volatile("cp.async.bulk.wait_group.read 1;" ::: "memory");
+                if (lane == 0) {
+                    if (NSTG == 2) asm volatile("cp.async.bulk.wait_group.read 1;" ::: "memory");
+                    else asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory");
+                }
                 PROF_ADD(pw_stgwait);
                 __syncwarp();
             }
+            // integer + FP32 reconstruction (crt_recon_bits, crt.h): no FP64 instruction while the
+            // tensor core runs; two elements at a time, stored as they are done
 #pragma unroll
             for (int v = 0; v < 8; v += 2) {
+                uint64_t o[2];
+#pragma unroll
+                for (int u = 0; u < 2; ++u) {
+                    uint32_t R[NP];
+                    const int vv = v + u;
+#pragma unroll
+                    for (int jj = 0; jj < NP; ++jj) {
+                        const uint32_t wv = (vv >> 1) == 0 ? w[jj].x : (vv >> 1) == 1 ? w[jj].y : (vv >> 1) == 2 ? w[jj].z : w[jj].w;
+                        R[jj] = (vv & 1) ? (wv >> 16) : (wv & 0xffffu);
+                    }
+                    o[u] = crt_recon_bits<NP>(R, p.c, pv_e0 + __ldg(pv_ecol + col0 + vv), p.store ? 0u : 1u);
+                }
                 const uint32_t a = sb + (uint32_t)lane * 64u + ((uint32_t)((v >> 1) ^ ((lane >> 1) & 3)) << 4);
-                asm volatile("st.shared.v2.b64 [%0], {%1, %2};" ::"r"(a), "l"(o[v]), "l"(o[v + 1]) : "memory");
+                asm volatile("st.shared.v2.b64 [%0], {%1, %2};" ::"r"(a), "l"(o[0]), "l"(o[1]) : "memory");
             }
             asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
             __syncwarp();
@@ -677,6 +708,41 @@ __global__ void __launch_bounds__(THREADS, 1) crt_gemm_kernel(const __grid_const
                 asm volatile("cp.async.bulk.commit_group;" ::: "memory");
             }
             ++nred;
+        };
+
+        // Walk the warp's CHUNKS 32-column TMEM chunks of accumulator buffer `buf`: double-buffered loads
+        // with 8 epilogue warps, single-buffered with 16 (register budget); the accumulator is released to
+        // the MMA as soon as its last chunk is in registers.
+        auto tmem_chunks = [&](uint32_t buf, auto&& f) {
+            const uint32_t base = tmem + tl + buf * (uint32_t)BN;
+            auto release = [&]() {
+                fence_before();
+                __syncwarp();
+                if (lane == 0) mbar_arrive_cluster_relaxed(ae0 + buf * 8u);
+            };
+            if constexpr (EPI_WARPS == 8) {
+                uint32_t v0[32], v1[32];
+                tmem_ld32_nowait(base, v0);
+                tmem_wait(v0);
+#pragma unroll
+                for (int c = 0; c < CHUNKS; ++c) {
+                    uint32_t (&vc)[32] = (c & 1) ? v1 : v0;
+                    uint32_t (&vn)[32] = (c & 1) ? v0 : v1;
+                    if (c < CHUNKS - 1) tmem_ld32_nowait(base + (uint32_t)((c + 1) * 32), vn);
+                    if (c == CHUNKS - 1) release();
+                    f(vc, c);
+                    if (c < CHUNKS - 1) tmem_wait(vn);
+                }
+            } else {
+#pragma unroll
+                for (int c = 0; c < CHUNKS; ++c) {
+                    uint32_t v0[32];
+                    tmem_ld32_nowait(base + (uint32_t)(c * 32), v0);
+                    tmem_wait(v0);
+                    if (c == CHUNKS - 1) release();
+                    f(v0, c);
+                }
+            }
         };
 
         int it_tile = 0;
@@ -698,19 +764,19 @@ __global__ void __launch_bounds__(THREADS, 1) crt_gemm_kernel(const __grid_const
                 uint4 wa[NP];
                 if (pv) {
                     if (CRT_EARLY) {
-                        if (jj == 0) prefetch_groups(0, 16 / NP);
-                        if (jj + 1 < NP) prefetch_groups(((jj + 1) * 16) / NP, ((jj + 2) * 16) / NP);
-                        load_group((jj * 16) / NP, wa);
+                        if (jj == 0) prefetch_groups(0, GROUPS / NP);
+                        if (jj + 1 < NP) prefetch_groups(((jj + 1) * GROUPS) / NP, ((jj + 2) * GROUPS) / NP);
+                        load_group((jj * GROUPS) / NP, wa);
                     } else {
-                        prefetch_groups((jj * 16) / NP, ((jj + 1) * 16) / NP);
+                        prefetch_groups((jj * GROUPS) / NP, ((jj + 1) * GROUPS) / NP);
                     }
                 }
                 // this pair's 16 destination blocks: those the last reconstruction step freed (the
                 // first tile of the CTA takes the blocks in order)
-                if (lane < 16) scr_tab[ew][ct][j * 16 + lane] = pv ? scr_free[ew][lane] : (uint8_t)(j * 16 + lane);
+                if (lane < GROUPS) scr_tab[ew][ct][j * GROUPS + lane] = pv ? scr_free[ew][lane] : (uint8_t)(j * GROUPS + lane);
                 __syncwarp();
                 // ---- first modulus a of pair j: canonical residues r_a kept as bytes (32 registers)
-                uint32_t ra[4][8];
+                uint32_t ra[CHUNKS][8];
                 {
                     const uint32_t buf = g & 1u;
                     { PROF_T0();
@@ -720,19 +786,7 @@ __global__ void __launch_bounds__(THREADS, 1) crt_gemm_kernel(const __grid_const
                     fence_after();
                     const int pa = p.c.p[2 * j];
                     const unsigned mqa = p.c.bm[2 * j];
-                    uint32_t v0[32], v1[32];
-                    tmem_ld32_nowait(tmem + tl + buf * (uint32_t)BN, v0);
-                    tmem_wait(v0);
-#pragma unroll
-                    for (int c = 0; c < 4; ++c) {
-                        uint32_t (&vc)[32] = (c & 1) ? v1 : v0;
-                        uint32_t (&vn)[32] = (c & 1) ? v0 : v1;
-                        if (c < 3) tmem_ld32_nowait(tmem + tl + buf * (uint32_t)BN + (uint32_t)((c + 1) * 32), vn);
-                        if (c == 3) {  // the whole accumulator is in registers: release it to the MMA now
-                            fence_before();
-                            __syncwarp();
-                            if (lane == 0) mbar_arrive_cluster_relaxed(ae0 + buf * 8u);
-                        }
+                    auto resid_a = [&](const uint32_t (&vc)[32], int c) {
 #pragma unroll
                         for (int k = 0; k < 8; ++k) {
                             const uint32_t b0 = (uint32_t)mod_canon((int)vc[4 * k], pa, mqa);
@@ -741,8 +795,8 @@ __global__ void __launch_bounds__(THREADS, 1) crt_gemm_kernel(const __grid_const
                             const uint32_t b3 = (uint32_t)mod_canon((int)vc[4 * k + 3], pa, mqa);
                             ra[c][k] = __byte_perm(__byte_perm(b0, b1, 0x0040), __byte_perm(b2, b3, 0x0040), 0x5410);
                         }
-                        if (c < 3) tmem_wait(vn);
-                    }
+                    };
+                    tmem_chunks(buf, resid_a);
                     ++g;
                     PROF_ADD(pw_resid);
                 }
@@ -756,56 +810,52 @@ __global__ void __launch_bounds__(THREADS, 1) crt_gemm_kernel(const __grid_const
                     fence_after();
                     const unsigned pa = (unsigned)p.c.p[2 * j], pb = (unsigned)p.c.p[2 * j + 1], ia = (unsigned)p.c.ia[j];
                     const unsigned shb = p.c.shoup[j], offb = pb << 21;
-                    uint32_t v0[32], v1[32];
-                    tmem_ld32_nowait(tmem + tl + buf * (uint32_t)BN, v0);
-                    tmem_wait(v0);
+                    auto resid_b = [&](const uint32_t (&vc)[32], int c) {
 #pragma unroll
-                    for (int c = 0; c < 4; ++c) {
-                        uint32_t (&vc)[32] = (c & 1) ? v1 : v0;
-                        uint32_t (&vn)[32] = (c & 1) ? v0 : v1;
-                        if (c < 3) tmem_ld32_nowait(tmem + tl + buf * (uint32_t)BN + (uint32_t)((c + 1) * 32), vn);
-                        if (c == 3) {  // accumulator fully in registers: release it
-                            fence_before();
-                            __syncwarp();
-                            if (lane == 0) mbar_arrive_cluster_relaxed(ae0 + buf * 8u);
-                        }
-                        uint32_t pk[16];
+                        for (int e4 = 0; e4 < 4; ++e4) {  // 8 columns -> one 16-byte store per block
+                            uint32_t pk[4];
 #pragma unroll
-                        for (int k = 0; k < 16; ++k) {
-                            uint32_t R2[2];
+                            for (int k = 0; k < 4; ++k) {
+                                uint32_t R2[2];
 #pragma unroll
-                            for (int u = 0; u < 2; ++u) {
-                                const int e = 2 * k + u;
-                                // t = ((acc_b - r_a) a^-1) mod b by Shoup's multiplication: x = acc_b - r_a +
-                                // b 2^21 in [0, 2^32); q = floor(x shoup / 2^32); x ia - q b in [0, 2b)
-                                const uint32_t rav = (ra[c][e >> 2] >> (8 * (e & 3))) & 0xffu;
-                                const uint32_t x = vc[e] - rav + offb;
-                                const uint32_t r2 = x * ia - __umulhi(x, shb) * pb;
-                                const uint32_t tt = min(r2, r2 - pb);
-                                R2[u] = rav + pa * tt;
+                                for (int u = 0; u < 2; ++u) {
+                                    const int e = 8 * e4 + 2 * k + u;
+                                    // t = ((acc_b - r_a) a^-1) mod b by Shoup's multiplication: x = acc_b - r_a +
+                                    // b 2^21 in [0, 2^32); q = floor(x shoup / 2^32); x ia - q b in [0, 2b)
+                                    const uint32_t rav = (ra[c][e >> 2] >> (8 * (e & 3))) & 0xffu;
+                                    const uint32_t x = vc[e] - rav + offb;
+                                    const uint32_t r2 = x * ia - __umulhi(x, shb) * pb;
+                                    const uint32_t tt = min(r2, r2 - pb);
+                                    R2[u] = rav + pa * tt;
+                                }
+                                pk[k] = R2[0] | (R2[1] << 16);
                             }
-                            pk[k] = R2[0] | (R2[1] << 16);
+                            *(uint4*)(scr0 + scr_off(scr_tab[ew][ct][j * GROUPS + c * 4 + e4], h, r)) =
+                                make_uint4(pk[0], pk[1], pk[2], pk[3]);
                         }
-#pragma unroll
-                        for (int e = 0; e < 4; ++e)
-                            *(uint4*)(scr0 + scr_off(scr_tab[ew][ct][j * 16 + c * 4 + e], h, r)) =
-                                make_uint4(pk[4 * e], pk[4 * e + 1], pk[4 * e + 2], pk[4 * e + 3]);
-                        if (c < 3) tmem_wait(vn);
-                    }
+                    };
+                    tmem_chunks(buf, resid_b);
                     ++g;
                     PROF_ADD(pw_resid);
                 }
                 // ---- two groups of the pending tile's reconstruction (16 groups over the NP pairs)
                 if (pv) {
                     PROF_T0();
-                    const int g0 = (jj * 16) / NP, g1 = ((jj + 1) * 16) / NP;
-                    uint4 wb[NP];
+                    const int g0 = (jj * GROUPS) / NP, g1 = ((jj + 1) * GROUPS) / NP;
                     if (!CRT_EARLY) load_group(g0, wa);
-                    for (int gi = g0; gi < g1; gi += 2) {
-                        if (gi + 1 < g1) load_group(gi + 1, wb);
-                        recon(gi, wa);
-                        if (gi + 1 < g1) recon(gi + 1, wb);
-                        if (gi + 2 < g1) load_group(gi + 2, wa);
+                    if constexpr (EPI_WARPS == 8) {  // two groups in flight
+                        uint4 wb[NP];
+                        for (int gi = g0; gi < g1; gi += 2) {
+                            if (gi + 1 < g1) load_group(gi + 1, wb);
+                            recon(gi, wa);
+                            if (gi + 1 < g1) recon(gi + 1, wb);
+                            if (gi + 2 < g1) load_group(gi + 2, wa);
+                        }
+                    } else {  // one (register budget of 20 warps)
+                        for (int gi = g0; gi < g1; ++gi) {
+                            if (gi > g0) load_group(gi, wa);
+                            recon(gi, wa);
+                        }
                     }
                     free_groups(g0);
                     PROF_ADD(pw_recon);
@@ -817,21 +867,29 @@ __global__ void __launch_bounds__(THREADS, 1) crt_gemm_kernel(const __grid_const
             pv = true;
             pv_tab = ct;
             pv_e0 = p.exps[jb.m * p.nb + grow] - 2 * p.c.bits;
-            pv_ecol = p.exps + (size_t)jb.n * p.nb + bj * BN + h * 128;
+            pv_ecol = p.exps + (size_t)jb.n * p.nb + bj * BN + h * PCOLS;
             pv_crow0 = (int)(((const char*)jb.C - (const char*)p.cbase) / ((size_t)p.nb * 8)) + bi * 256 +
                        (int)crank * BM + q * 32;
-            pv_ccol0 = bj * BN + h * 128;
+            pv_ccol0 = bj * BN + h * PCOLS;
         }
         if (pv) {  // drain: the last tile's reconstruction
             PROF_T0();
-            prefetch_groups(0, 16);
-            uint4 wa[NP], wb[NP];
-            load_group(0, wa);
-            for (int gi = 0; gi < 16; gi += 2) {
-                load_group(gi + 1, wb);
-                recon(gi, wa);
-                if (gi + 2 < 16) load_group(gi + 2, wa);
-                recon(gi + 1, wb);
+            prefetch_groups(0, GROUPS);
+            uint4 wa[NP];
+            if constexpr (EPI_WARPS == 8) {
+                uint4 wb[NP];
+                load_group(0, wa);
+                for (int gi = 0; gi < GROUPS; gi += 2) {
+                    load_group(gi + 1, wb);
+                    recon(gi, wa);
+                    if (gi + 2 < GROUPS) load_group(gi + 2, wa);
+                    recon(gi + 1, wb);
+                }
+            } else {
+                for (int gi = 0; gi < GROUPS; ++gi) {
+                    load_group(gi, wa);
+                    recon(gi, wa);
+                }
             }
             PROF_ADD(pw_recon);
         }

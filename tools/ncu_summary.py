@@ -8,7 +8,8 @@ import sys
 def raw(path):
     out = subprocess.run(["ncu", "-i", path, "--page", "raw", "--csv"], capture_output=True, text=True).stdout
     rows = list(csv.reader(out.splitlines()))
-    return [dict(zip(rows[0], r)) for r in rows[2:]]
+    units = dict(zip(rows[0], rows[1]))
+    return [dict(((k, (v + " " + units.get(k, "")).strip()) for k, v in zip(rows[0], r))) for r in rows[2:]]
 
 
 KEYS = ["Kernel Name", "gpu__time_duration.sum", "sm__cycles_elapsed.avg",
