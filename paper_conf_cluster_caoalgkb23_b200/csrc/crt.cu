@@ -250,7 +250,11 @@ constexpr uint32_t TMEM_COLS = 512;  // two 256-column accumulators
 // 1: reconstructed residue-scratch lines are discarded from L2 (discard.global.L2) instead of being
 // evicted dirty to HBM
 #ifndef CRT_DISCARD
-#define CRT_DISCARD 1
+#define CRT_DISCARD 0
+#endif
+// 1: residue-scratch stores carry an L2 evict_last policy
+#ifndef CRT_SCRHINT
+#define CRT_SCRHINT 0
 #endif
 // instruction descriptor: D = S32 (2 << 4), A = B = signed int8 (1 << 7, 1 << 10), K-major,
 // N >> 3 at bit 17, M >> 4 at bit 24 (M = 256 for the pair)
@@ -601,6 +605,8 @@ __global__ void __launch_bounds__(THREADS, 1) crt_gemm_kernel(const __grid_const
         const int q = (warp - 4) & 3, h = (warp - 4) >> 2;
         const int r = q * 32 + lane;  // CTA row = TMEM lane
         uint8_t* const scr0 = p.scratch + (size_t)slot_sh * CRT_SLOT_BYTES;
+        uint64_t scr_pol = 0;
+        if (CRT_SCRHINT) asm volatile("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(scr_pol));
         const uint32_t tl = ((uint32_t)(q * 32) << 16) + (uint32_t)(h * PCOLS);
         const uint32_t ae0 = cluster_addr(su32(&acc_empty[0]), 0);
         const uint32_t stg_s = su32(smem + STAGES * STAGE_BYTES + (warp - 4) * STG_WARP);
@@ -830,8 +836,13 @@ __global__ void __launch_bounds__(THREADS, 1) crt_gemm_kernel(const __grid_const
                                 }
                                 pk[k] = R2[0] | (R2[1] << 16);
                             }
-                            *(uint4*)(scr0 + scr_off(scr_tab[ew][ct][j * GROUPS + c * 4 + e4], h, r)) =
-                                make_uint4(pk[0], pk[1], pk[2], pk[3]);
+                            uint8_t* const dst = scr0 + scr_off(scr_tab[ew][ct][j * GROUPS + c * 4 + e4], h, r);
+                            if (CRT_SCRHINT)  // keep the residues in L2 until the reconstruction reads them
+                                asm volatile("st.global.L2::cache_hint.v4.b32 [%0], {%1, %2, %3, %4}, %5;" ::"l"(dst), "r"(pk[0]),
+                                             "r"(pk[1]), "r"(pk[2]), "r"(pk[3]), "l"(scr_pol)
+                                             : "memory");
+                            else
+                                *(uint4*)dst = make_uint4(pk[0], pk[1], pk[2], pk[3]);
                         }
                     };
                     tmem_chunks(buf, resid_b);
