@@ -62,7 +62,18 @@ typedef enum {
     MP_ERR_STATE = 7         /* call order violated (e.g. potrf before generation) */
 } mp_status;
 
-typedef enum { MP_FP64 = 0, MP_FP32 = 1, MP_FP16 = 2 } mp_prec;
+/* Precision classes (smaller value = higher precision).  MP_FP16 is the paper's FP16_32 (FP16 operands,
+ * FP32 accumulation); MP_FP16H is the paper's pure FP16 class (FP16 operands AND FP16
+ * accumulation, "A, B, C, and operation are all in FP16"), used only by four-level maps
+ * (mp_precision_map4, MP_MAP_ADAPTIVE4).  Data (storage / communication) precisions
+ * are FP64, FP32 and FP16 only: an FP16H tile is stored in FP32 and receives FP16 operands. */
+typedef enum { MP_FP64 = 0, MP_FP32 = 1, MP_FP16 = 2, MP_FP16H = 3 } mp_prec;
+
+/* u_low of the FP16_32 class in four-level maps.  The paper fixes it "experimentally" (citing
+ * [23]: FP16_32 has a lower error bound than FP16) and prints no value; reading C7': the
+ * ratio of the measured tile-GEMM errors of the FP16_32 and pure-FP16 classes on the application's
+ * FP16-class tiles times FP16's machine epsilon 2^-10 (tools/fp16_eps.py). */
+#define MP_EPS_FP16_32 (1.0 / 8192.0)
 
 /* Communication-precision policy.
  * MP_COMM_TTC : target-task conversion — every tile travels in its storage
@@ -77,7 +88,8 @@ typedef enum {
     MP_MAP_FP64 = 1,      /* everything FP64 (the "same code forced to all-FP64" baseline) */
     MP_MAP_BAND = 2,      /* FP64 band / FP32 outside (config 2; reading C21) */
     MP_MAP_EXTREME = 3,   /* FP64 diagonal, FP16 elsewhere (performance-only) */
-    MP_MAP_USER = 4       /* kernel_prec supplied by the caller */
+    MP_MAP_USER = 4,      /* kernel_prec supplied by the caller */
+    MP_MAP_ADAPTIVE4 = 5  /* four-level rule (FP64, FP32, FP16_32, FP16; mp_precision_map4) at u_req */
 } mp_map_mode;
 
 /* Covariance family of the generated matrix (§III-A). */
@@ -102,6 +114,8 @@ typedef struct {
     int64_t stc_tiles;            /* off-diagonal tiles whose comm precision < storage */
     int64_t gpu_launches;         /* kernels launched by this call */
     uint64_t workspace_bytes;     /* bytes this evaluation's map needs (set also on MP_ERR_NOMEM) */
+    int64_t tiles_fp16h;          /* four-level maps: tiles of the pure-FP16 class (counted apart from tiles[2]) */
+    double flops_update_fp16h;    /*   and their GEMM flops (apart from flops_update[2]) */
 } mp_eval_report;
 
 /* ---------------------------------------------------------------- configuration */
@@ -252,6 +266,15 @@ mp_status mp_matern_gen(mp_handle* h, mp_matrix* A, const double* d_x, const dou
 mp_status mp_precision_map(int nt, const double* tile_sqnorm, double u_req, const double* eps,
                            mp_comm_policy policy, uint8_t* kernel_prec, uint8_t* storage_prec,
                            uint8_t* comm_prec);
+
+/* Four-level variant (P:113 / P:117: "FP64, FP32, FP16_32, and FP16"): eps[4] =
+ * {FP64, FP32, FP16_32, FP16} (NULL = {2^-52, 2^-23, MP_EPS_FP16_32, 2^-10}; eps[3] >= eps[2]);
+ * kernel = MP_FP16H if r <= u_req/eps[3], else MP_FP16 if r <= u_req/eps[2], else FP32 if
+ * r <= u_req/eps[1], else FP64.  Storage and communication maps as above (data precisions
+ * FP64 / FP32 / FP16: an FP16H successor receives FP16).  A user kernel map may contain MP_FP16H. */
+mp_status mp_precision_map4(int nt, const double* tile_sqnorm, double u_req, const double* eps,
+                            mp_comm_policy policy, uint8_t* kernel_prec, uint8_t* storage_prec,
+                            uint8_t* comm_prec);
 
 /* (3) In-place mixed-precision tile Cholesky A = L L^T (Algorithm 1):
  * DPOTRF (FP64) on diagonal tiles; TRSM(m,k) with L_kk received at comm(k,k): FP64 substitution

@@ -45,4 +45,5 @@ Pins (what fixes each part independently of this code; tests/test_oracle_*.py):
 """
 
 FP64, FP32, FP16 = 0, 1, 2  # smaller value = higher precision (SURVEY §8(b) mp_prec)
-PREC_NAMES = {FP64: "FP64", FP32: "FP32", FP16: "FP16"}
+FP16H = 3  # four-level maps only: the paper's pure FP16 class (FP16 operands AND accumulation)
+PREC_NAMES = {FP64: "FP64", FP32: "FP32", FP16: "FP16_32", FP16H: "FP16"}

@@ -31,7 +31,7 @@ from __future__ import annotations
 
 import numpy as np
 
-from . import FP16, FP32, FP64
+from . import FP16, FP16H, FP32, FP64
 from .tiles import global_sqnorm
 
 EPS_DEFAULT = (2.0**-52, 2.0**-23, 2.0**-10)  # reading C7: literal machine epsilons
@@ -44,9 +44,15 @@ def tile_ratio(s_mk: float, nt: int, S: float) -> float:
 
 
 def kernel_map(s: np.ndarray, u_req: float, eps=EPS_DEFAULT) -> np.ndarray:
-    """kernel_precision[m, k] for m >= k (upper triangle left at 255 = unused). P:117."""
+    """kernel_precision[m, k] for m >= k (upper triangle left at 255 = unused). P:117.
+
+    Three levels (len(eps) == 3; FP16 = FP16_32) or four (len(eps) == 4: eps = (FP64, FP32,
+    FP16_32, FP16), P:113 / P:117 "FP64, FP32, FP16_32, and FP16"; the pure-FP16 class FP16H is
+    tried first: FP16H if r <= u_req/eps[3], else FP16_32 if r <= u_req/eps[2], ...)."""
     nt = s.shape[0]
     S = global_sqnorm(s)
+    four = len(eps) == 4
+    thr16h = u_req / eps[FP16H] if four else -1.0
     thr16 = u_req / eps[FP16]
     thr32 = u_req / eps[FP32]
     kmap = np.full((nt, nt), 255, dtype=np.uint8)
@@ -54,7 +60,9 @@ def kernel_map(s: np.ndarray, u_req: float, eps=EPS_DEFAULT) -> np.ndarray:
         kmap[k, k] = FP64
         for m in range(k + 1, nt):
             r = tile_ratio(float(s[m, k]), nt, S)
-            if r <= thr16:
+            if r <= thr16h:
+                kmap[m, k] = FP16H
+            elif r <= thr16:
                 kmap[m, k] = FP16
             elif r <= thr32:
                 kmap[m, k] = FP32
@@ -64,7 +72,8 @@ def kernel_map(s: np.ndarray, u_req: float, eps=EPS_DEFAULT) -> np.ndarray:
 
 
 def storage_precision(kernel_prec: int) -> int:
-    """get_storage_precision of Alg. 2 line 16: FP64 stays FP64, FP32 and FP16 kernels store FP32."""
+    """get_storage_precision of Alg. 2 line 16: FP64 stays FP64, FP32 and FP16 kernels (FP16_32 and
+    pure FP16) store FP32."""
     return FP64 if kernel_prec == FP64 else FP32
 
 
@@ -103,7 +112,8 @@ def comm_map(kmap: np.ndarray, policy: int = COMM_AUTO) -> np.ndarray:
     for k in range(nt - 1):
         for m in range(k + 1, nt):  # reading C10 (i): m starts at k+1
             st = int(smap[m, k])
-            comm = FP16  # line 14: initialised to the lowest precision
+            comm = FP16  # line 14: initialised to the lowest precision (FP16 data; an FP16H
+            # consumer receives FP16 operands too, so higher() with it leaves FP16)
             comm = higher(comm, int(kmap[m, k]))  # reading C10 (ii): SYRK(m,k) successor
             done = False
             if comm <= st:

@@ -23,7 +23,7 @@ import numpy as np
 from ._lib import (Config, EvalReport, MpError, Profile, PROF_CLASSES, lib, MP_OK, MP_ERR_NOT_SPD,  # noqa: F401
                    MP_ERR_NOMEM, MP_FP64, MP_FP32, MP_FP16, MP_COMM_TTC, MP_COMM_AUTO, MP_MAP_ADAPTIVE, MP_MAP_FP64,
                    MP_MAP_BAND, MP_MAP_EXTREME, MP_MAP_USER, MP_COV_MATERN, MP_COV_SQEXP, MP_F64_CRT16, MP_F64_DMMA,
-                   MP_F32_3XFP16, MP_F32_3XTF32, MP_F32_DMMA)
+                   MP_F32_3XFP16, MP_F32_3XTF32, MP_F32_DMMA, MP_FP16H, MP_MAP_ADAPTIVE4, MP_EPS_FP16_32)
 
 __all__ = ["Handle", "Matrix", "Evaluator", "precision_map", "exchange_plan", "exact_sum", "unique_id", "MpError",
            "EvalReport", "default_config", "shared_unique_id"]
@@ -280,8 +280,9 @@ class Matrix:
 
 
 def precision_map(tile_sqnorm: np.ndarray | None, u_req: float = 1e-9, eps=None, policy: int = MP_COMM_AUTO,
-                  kernel_prec: np.ndarray | None = None):
-    """mp_precision_map (host only).  Returns (kernel, storage, comm) NT x NT uint8 maps."""
+                  kernel_prec: np.ndarray | None = None, levels: int = 3):
+    """mp_precision_map (levels = 3) or mp_precision_map4 (levels = 4; host only).  Returns (kernel,
+    storage, comm) NT x NT uint8 maps."""
     if tile_sqnorm is not None:
         s = np.ascontiguousarray(tile_sqnorm, dtype=np.float64)
         nt = s.shape[0]
@@ -293,7 +294,8 @@ def precision_map(tile_sqnorm: np.ndarray | None, u_req: float = 1e-9, eps=None,
     sm = np.full((nt, nt), 255, np.uint8)
     cm = np.full((nt, nt), 255, np.uint8)
     e = None if eps is None else np.ascontiguousarray(eps, dtype=np.float64)
-    st = lib.mp_precision_map(nt, _d(s), float(u_req), _d(e), policy, _u8(km), _u8(sm), _u8(cm))
+    fn = lib.mp_precision_map4 if levels == 4 else lib.mp_precision_map
+    st = fn(nt, _d(s), float(u_req), _d(e), policy, _u8(km), _u8(sm), _u8(cm))
     if st != MP_OK:
         raise MpError(st, "mp_precision_map failed")
     return km, sm, cm

@@ -15,9 +15,10 @@ LIB_PATH = os.path.join(_HERE, "libmpgeo.so")
 MP_OK, MP_ERR_ARG, MP_ERR_NOT_SPD, MP_ERR_CUDA, MP_ERR_COMM, MP_ERR_NOMEM, MP_ERR_UNSUPPORTED, MP_ERR_STATE = range(8)
 STATUS_NAMES = ["MP_OK", "MP_ERR_ARG", "MP_ERR_NOT_SPD", "MP_ERR_CUDA", "MP_ERR_COMM", "MP_ERR_NOMEM",
                 "MP_ERR_UNSUPPORTED", "MP_ERR_STATE"]
-MP_FP64, MP_FP32, MP_FP16 = 0, 1, 2
+MP_FP64, MP_FP32, MP_FP16, MP_FP16H = 0, 1, 2, 3  # MP_FP16 = FP16_32; MP_FP16H = pure FP16 (four-level maps)
 MP_COMM_TTC, MP_COMM_AUTO = 0, 1
-MP_MAP_ADAPTIVE, MP_MAP_FP64, MP_MAP_BAND, MP_MAP_EXTREME, MP_MAP_USER = range(5)
+MP_MAP_ADAPTIVE, MP_MAP_FP64, MP_MAP_BAND, MP_MAP_EXTREME, MP_MAP_USER, MP_MAP_ADAPTIVE4 = range(6)
+MP_EPS_FP16_32 = 1.0 / 8192.0  # include/mpgeo.h
 MP_COV_MATERN, MP_COV_SQEXP = 0, 1
 MP_F64_CRT16, MP_F64_DMMA = 0, 1
 MP_F32_3XFP16, MP_F32_3XTF32, MP_F32_DMMA = 0, 1, 2
@@ -32,6 +33,7 @@ class EvalReport(C.Structure):
         ("flops_potrf", C.c_double), ("flops_update", C.c_double * 3),
         ("tiles", C.c_int64 * 3), ("stc_tiles", C.c_int64), ("gpu_launches", C.c_int64),
         ("workspace_bytes", C.c_uint64),
+        ("tiles_fp16h", C.c_int64), ("flops_update_fp16h", C.c_double),
     ]
 
 
@@ -88,6 +90,7 @@ def _load() -> C.CDLL:
         "mp_matrix_bind": (i32, [vp, u8p, vp, C.c_size_t]),
         "mp_matern_gen": (i32, [vp, vp, vp, vp, dp, u8p, dp]),
         "mp_precision_map": (i32, [i32, dp, dbl, dp, i32, u8p, u8p, u8p]),
+        "mp_precision_map4": (i32, [i32, dp, dbl, dp, i32, u8p, u8p, u8p]),
         "mp_tile_potrf": (i32, [vp, vp, u8p, u8p, C.POINTER(i64)]),
         "mp_loglik": (i32, [vp, vp, vp, dp, dp, dp]),
         "mp_gp_sample": (i32, [vp, vp, vp, vp]),

@@ -114,3 +114,33 @@ def test_multirank_init_requires_the_communicator_id():
     h = C.c_void_p()
     assert lib.mp_init(0, 0, 2, 1, 2, None, None, C.byref(h)) == MP_ERR_ARG
     assert lib.mp_init(0, 0, 16, 4, 4, None, None, C.byref(h)) != 0  # more ranks than MAX_PEERS
+
+
+@pytest.mark.parametrize("beta,u_req,policy", [(0.03, 1e-9, 1), (0.1, 1e-9, 1), (0.03, 1e-6, 0)])
+def test_precision_map4_bit_exact_vs_oracle(beta, u_req, policy):
+    from paper_conf_cluster_caoalgkb23_b200 import MP_EPS_FP16_32, precision_map
+    s = _matern_norms(6400, 256, beta)
+    eps4 = (2.0**-52, 2.0**-23, MP_EPS_FP16_32, 2.0**-10)
+    km, sm, cm = precision_map(s, u_req, policy=policy, levels=4)  # eps = NULL: the library default
+    okm, osm, ocm = oprec.precision_maps(s, u_req, eps=eps4, policy=policy)
+    nt = s.shape[0]
+    low = np.tril(np.ones((nt, nt), bool))
+    assert np.array_equal(km[low], okm[low])
+    assert np.array_equal(sm[low], osm[low])
+    assert np.array_equal(cm[low], ocm[low])
+
+
+def test_precision_map4_handbuilt_golden():
+    from paper_conf_cluster_caoalgkb23_b200 import precision_map
+    from tests.test_oracle_precision import EPS4_GOLDEN, load_handbuilt4
+    s, expect = load_handbuilt4()
+    km, _, _ = precision_map(s, 2.0**-30, eps=EPS4_GOLDEN, levels=4)
+    for (m, k), e in expect.items():
+        assert km[m, k] == e
+    # a three-level call rejects a user map holding the four-level class; the four-level call takes it
+    from paper_conf_cluster_caoalgkb23_b200 import MpError
+    user = km.copy()
+    with pytest.raises(MpError):
+        precision_map(None, kernel_prec=user)
+    _, sm, cm = precision_map(None, kernel_prec=user, levels=4)
+    assert sm[1, 0] == 1 and cm[1, 0] <= 2

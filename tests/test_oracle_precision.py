@@ -133,3 +133,64 @@ def test_band_map():
             if two[m, k] == FP64:
                 assert bm[m, k] == FP64
     assert set(np.unique(bm[np.tril_indices(nt)]).tolist()) <= {FP64, FP32}
+
+
+# ---------------------------------------------------------------- four-level maps
+GOLDEN4 = os.path.join(os.path.dirname(__file__), "golden", "map4_handbuilt.txt")
+EPS4_GOLDEN = (2.0**-52, 2.0**-23, 2.0**-13, 2.0**-10)
+
+
+def load_handbuilt4():
+    nt = 4
+    s = np.zeros((nt, nt))
+    expect = {}
+    for line in open(GOLDEN4):
+        if line.startswith("#") or not line.strip():
+            continue
+        m, k, v, e = line.split()[:4]
+        s[int(m), int(k)] = float.fromhex(v)
+        expect[int(m), int(k)] = int(e)
+    s[0, 0] = 14.0 - 2.0**-13 - 2.0**-33 - 2.0**-35 - 2.0**-39 - 2.0**-49
+    return s, expect
+
+
+def test_handbuilt_map_four_levels():
+    from oracle import FP16H
+    s, expect = load_handbuilt4()
+    assert global_sqnorm(s) == 16.0
+    km = kernel_map(s, 2.0**-30, EPS4_GOLDEN)
+    for k in range(4):
+        assert km[k, k] == FP64
+    for (m, k), e in expect.items():
+        assert km[m, k] == e, (m, k, km[m, k], e)
+    assert sorted(set(expect.values())) == [FP64, FP32, FP16, FP16H]  # every class appears
+
+
+def test_four_level_refines_three_level():
+    """Invariants of the four-level rule on Matérn norms: a tile is FP16 (pure) only if the three-level rule
+    with the same FP16 epsilon already makes it FP16(_32); FP64 / FP32 are unchanged; with
+    eps[FP16_32] = eps[FP16] the FP16_32 band is empty; storage is FP32 for every non-FP64 class; Algorithm 2
+    gives an FP16H tile's successors FP16 data (no comm code above FP16)."""
+    from oracle import FP16H
+    s = small_norms(0.03, 4096, 256)
+    u = 1e-9
+    k3 = kernel_map(s, u, (2.0**-52, 2.0**-23, 2.0**-10))
+    k4 = kernel_map(s, u, (2.0**-52, 2.0**-23, 2.0**-13, 2.0**-10))
+    nt = s.shape[0]
+    low = np.tril(np.ones((nt, nt), bool), -1)
+    assert np.array_equal(k4[low] == FP64, k3[low] == FP64)
+    assert np.array_equal(k4[low] == FP16H, k3[low] == FP16)
+    assert ((k4[low] == FP16) <= (k3[low] == FP32)).all()
+    assert (k4[low] == FP16).any() and (k4[low] == FP16H).any()
+    same = kernel_map(s, u, (2.0**-52, 2.0**-23, 2.0**-10, 2.0**-10))
+    assert not (same[low] == FP16).any()
+    sm = storage_map(k4)
+    assert np.array_equal(sm[low] == FP64, k4[low] == FP64) and set(np.unique(sm[low])) <= {FP64, FP32}
+    cm = comm_map(k4)
+    assert int(cm[np.tril(np.ones((nt, nt), bool))].max()) <= FP16
+    # an all-FP16H map behaves like the extreme FP16 map for communication: every tile STC in FP16
+    ext = extreme_map(nt, FP16H)
+    ce = comm_map(ext)
+    for k in range(nt - 1):
+        for m in range(k + 1, nt):
+            assert ce[m, k] == FP16

@@ -82,6 +82,10 @@ __global__ void __launch_bounds__(384, 1) k(Res* out, int iters, double a, doubl
                 if (OP == 2) y[i] = y[i] * (uint32_t)iters + (uint32_t)i;
                 if (OP == 3) y[i] = __umulhi(y[i], 0x9E3779B9u) + (uint32_t)i;
                 if (OP == 4) x[i] = x[i] + b;
+                if (OP == 5 && (i & 1) == 0) {  // DMMA m8n8k4: 2 FP64 MACs x 64 per thread-instruction pair
+                    asm volatile("mma.sync.aligned.m8n8k4.row.col.f64.f64.f64.f64 {%0, %1}, {%2}, {%3}, {%0, %1};"
+                                 : "+d"(x[i]), "+d"(x[i + 1]) : "d"(a), "d"(b));
+                }
             }
         }
         long long t1 = clock64();
@@ -113,7 +117,8 @@ void run(const char* name, int sms, Res* d) {
     cudaError_t e = cudaDeviceSynchronize();
     Res h;
     cudaMemcpy(&h, d, sizeof h, cudaMemcpyDeviceToHost);
-    const double alu_rate = 8.0 * 32 * iters * 8 / (double)h.alu_cyc;  // lane-ops per clock per SM (8 warps)
+    // lane-ops per clock per SM (8 warps); DMMA: FP64 MACs per clock per SM (4 mma per iteration and warp, 256 MACs each)
+    const double alu_rate = OP == 5 ? 8.0 * iters * 4 * 256 / (double)h.alu_cyc : 8.0 * 32 * iters * 8 / (double)h.alu_cyc;
     const double mac = MMA ? (double)h.mmas * 128 * 256 * 32 / (double)h.mma_cyc : 0.0;
     printf("%-8s mma=%-4s: ALU %6.1f lane-op/clk/SM   MMA %7.0f MAC/clk/SM  (%s)\n", name, MMA == 0 ? "none" : MMA == 1 ? "i8" : "f16",
            alu_rate, mac, cudaGetErrorString(e));
@@ -130,5 +135,6 @@ int main() {
     run<1, 0>("FFMA", sms, d); run<1, 1>("FFMA", sms, d); run<1, 2>("FFMA", sms, d);
     run<2, 0>("IMAD", sms, d); run<2, 1>("IMAD", sms, d); run<2, 2>("IMAD", sms, d);
     run<3, 0>("IMAD.HI", sms, d); run<3, 1>("IMAD.HI", sms, d);
+    run<5, 0>("DMMA", sms, d); run<5, 1>("DMMA", sms, d); run<5, 2>("DMMA", sms, d);
     return 0;
 }
