@@ -107,7 +107,9 @@ __global__ void __launch_bounds__(256) transpose_kernel(const double* __restrict
 // 3xTF32, now within FP16 range; e_i = -s_i is stored for the GEMM epilogue.  hi + lo are the
 // 3xFP16 FP32-class operands; hi alone is the FP16-class operand (FP16 = 11 significant bits, with
 // the power-of-two row scale keeping small entries out of the FP16 subnormal range).  lo may be
-// null (FP16 class only).  One warp per row.
+// null (FP16 class only).  hs (optional, four-level maps' pure FP16 class) = rn(x 2^(s - 13)): the same
+// row scale with the row max in [2, 4), so K = nb products of two such rows sum to <= K 2^4 < 65504 in an
+// FP16 accumulator (tc_gemm KIND 3 multiplies by 2^(e_i + e_j + 26)).  One warp per row.
 __global__ void __launch_bounds__(256) split16_kernel(const Split16Item* items, int nb) {
     const Split16Item it = items[blockIdx.y];
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
@@ -126,14 +128,17 @@ __global__ void __launch_bounds__(256) split16_kernel(const Split16Item* items, 
     const int sc = min(max(15 - e, -100), 115);  // 2^sc and 2^-sc are normal FP32 numbers
     if (lane == 0) it.exps[row] = -sc;
     const float f = ldexpf(1.f, sc);
-    __half* hi = it.hi + (size_t)row * nb;
+    __half* hi = it.hi ? it.hi + (size_t)row * nb : nullptr;
     __half* lo = it.lo ? it.lo + (size_t)row * nb : nullptr;
+    __half* hs = it.hs ? it.hs + (size_t)row * nb : nullptr;
     for (int j = lane * 2; j < nb; j += 64) {
         const double2 v = *(const double2*)(x + j);
         const float a0 = __double2float_rn(v.x) * f, a1 = __double2float_rn(v.y) * f;
         const __half h0 = __float2half_rn(a0), h1 = __float2half_rn(a1);
-        *(__half2*)(hi + j) = __halves2half2(h0, h1);
+        if (hi) *(__half2*)(hi + j) = __halves2half2(h0, h1);
         if (lo) *(__half2*)(lo + j) = __halves2half2(__float2half_rn(a0 - __half2float(h0)), __float2half_rn(a1 - __half2float(h1)));
+        // pure-FP16 class operand: the row at max in [2, 4) (|sums| <= K 2^4 in an FP16 accumulator)
+        if (hs) *(__half2*)(hs + j) = __halves2half2(__float2half_rn(a0 * 0x1p-13f), __float2half_rn(a1 * 0x1p-13f));
     }
 }
 

@@ -93,7 +93,7 @@ static Engines engines_for(const mp_handle* h, int nb) {
 
 struct Regions {
     size_t total = 0;
-    size_t inputs = 0, p64 = 0, h16 = 0, e16 = 0, phi = 0, plo = 0, oz32 = 0, e32 = 0, ltilde = 0, wbuf = 0,
+    size_t inputs = 0, p64 = 0, h16 = 0, h16s = 0, e16 = 0, phi = 0, plo = 0, oz32 = 0, e32 = 0, ltilde = 0, wbuf = 0,
            wbuf2 = 0, wfac = 0, oz = 0, ozexp = 0, wdiag = 0, mtab = 0, crt = 0, crtflags = 0, crtctr = 0;
     int p64_sets = 1;              // 2 when the update reads the FP64 panel buffer (Engines::p64_double)
     size_t vec_r = 0, vec_y = 0, partials = 0, norms = 0, ctrl = 0, ctrl_bytes = 0;
@@ -125,6 +125,7 @@ struct mp_matrix {
     std::vector<uint8_t> storage, kmap, cmap;
     std::vector<double> sqn;      // tile sums of squares of the last generation pass 1 (NT*NT, all-gathered)
     std::vector<int> tscale;      // FP16 storage class: per-tile exponent t (stored value fp16(x 2^t))
+    bool h16h = false;            // the bound map has pure-FP16 (MP_FP16H) tiles: the hs operand planes exist
     int ts(int m, int k) const { return tscale.empty() ? 0 : tscale[(size_t)m * nt + k]; }
     Regions R;
     int owner(int m, int k) const { return (m % h->P) * h->Q + (k % h->Q); }
@@ -215,6 +216,7 @@ static Regions layout(const mp_matrix* A, const uint8_t* storage) {
     if (E.h16) {  // row-scaled FP16 hi and lo planes + row exponents (3xFP16 FP32 class, FP16 class)
         R.h16 = take(2 * slots * 2);
         R.e16 = take(nvec * 4);
+        if (A->h16h) R.h16s = take(slots * 2);  // four-level maps: pure-FP16 operands (split16 hs)
     }
     if (E.f32 == MP_F32_3XTF32) {
         R.phi = take(slots * 4);
@@ -861,7 +863,7 @@ mp_status mp_matern_gen(mp_handle* h, mp_matrix* A, const double* d_x, const dou
 
 // ------------------------------------------------------------------ (3) factorisation
 struct FlopCount {
-    double potrf = 0, trsm = 0, upd[3] = {0, 0, 0};
+    double potrf = 0, trsm = 0, upd[4] = {0, 0, 0, 0};  // upd[MP_FP16H]: four-level maps
 };
 
 static mp_status plan_potrf(mp_handle* h, mp_matrix* A, const uint8_t* km, const uint8_t* cm, Arena& ar,
@@ -874,6 +876,7 @@ static mp_status plan_potrf(mp_handle* h, mp_matrix* A, const uint8_t* km, const
     double* const p64b = A->at<double>(RG.p64);
     __half* const h16hi = E.h16 ? A->at<__half>(RG.h16) : nullptr;  // [nt*nb][nb] hi planes, then lo
     __half* const h16lo = E.h16 ? h16hi + slots : nullptr;
+    __half* const h16s = RG.h16s ? A->at<__half>(RG.h16s) : nullptr;  // pure-FP16 operands (four-level maps)
     int* const e16 = E.h16 ? A->at<int>(RG.e16) : nullptr;
     float* const phi = RG.phi ? A->at<float>(RG.phi) : nullptr;
     float* const plo = RG.plo ? A->at<float>(RG.plo) : nullptr;
@@ -939,10 +942,10 @@ static mp_status plan_potrf(mp_handle* h, mp_matrix* A, const uint8_t* km, const
         for (auto& x : xs) (x.dir == 0 ? xpub : xpull)[x.k].push_back(x);
     }
     // the operand classes MY successors of L_mk run at: SYRK(m,k) on (m,m), GEMM(m,n,k), GEMM(n,m,k)
-    auto needs = [&](int k, int m, bool& n16, bool& n32, bool& n64) {
-        n16 = n32 = false;
+    auto needs = [&](int k, int m, bool& n16, bool& n32, bool& n64, bool& n16h) {
+        n16 = n32 = n16h = false;
         n64 = A->mine(m, m);
-        auto cls = [&](int p) { n16 |= p == MP_FP16, n32 |= p == MP_FP32, n64 |= p == MP_FP64; };
+        auto cls = [&](int p) { n16 |= p == MP_FP16, n32 |= p == MP_FP32, n64 |= p == MP_FP64, n16h |= p == MP_FP16H; };
         for (int n = k + 1; n < m; ++n)
             if (A->mine(m, n)) cls(K(m, n));
         for (int n = m + 1; n < nt; ++n)
@@ -1214,13 +1217,13 @@ static mp_status plan_potrf(mp_handle* h, mp_matrix* A, const uint8_t* km, const
             std::vector<CrtSplitItem> c16;
             for (int m = k + 1; m < nt; ++m) {
                 if (!have[m]) continue;
-                bool n16, n32, n64;
-                needs(k, m, n16, n32, n64);
+                bool n16, n32, n64, n16h;
+                needs(k, m, n16, n32, n64, n16h);
                 const double* src = p64 + (size_t)m * nb2;
                 const bool lo3 = n32 && E.f32 == MP_F32_3XFP16;
-                if (E.h16 && (lo3 || (n16 && E.tc16)))
+                if (E.h16 && (lo3 || (n16 && E.tc16) || (n16h && h16s)))
                     s16.push_back(Split16Item{src, h16hi + (size_t)m * nb2, lo3 ? h16lo + (size_t)m * nb2 : nullptr,
-                                              e16 + (size_t)m * nb});
+                                              e16 + (size_t)m * nb, n16h && h16s ? h16s + (size_t)m * nb2 : nullptr});
                 if (n32 && E.f32 == MP_F32_3XTF32) t32s.push_back(Tf32Item{src, phi + (size_t)m * nb2, plo + (size_t)m * nb2});
                 if (n64 && E.crt) c16.push_back(CrtSplitItem{src, ozs + (size_t)m * nb2, oze + (size_t)m * nb, plane});
             }
@@ -1246,7 +1249,7 @@ static mp_status plan_potrf(mp_handle* h, mp_matrix* A, const uint8_t* km, const
             cur = part == 0 ? &nxt[k] : &rst[k];
             std::vector<GemmJob> syrk, g64, g32, g16;
             std::vector<CrtJob> csyrk, c64;
-            std::vector<TcJob> t32, t16;
+            std::vector<TcJob> t32, t16, t16h;
             for (int m = k + 1; m < nt; ++m) {
                 if (A->mine(m, m) && ((m == k + 1) == (part == 0))) {
                     if (E.crt) csyrk.push_back(CrtJob{m, m, A->tile(m, m)});
@@ -1257,7 +1260,9 @@ static mp_status plan_potrf(mp_handle* h, mp_matrix* A, const uint8_t* km, const
                     if (!A->mine(m, n) || ((n == k + 1) != (part == 0))) continue;
                     const int p = K(m, n);
                     fc.upd[p] += 2.0 * fnb * fnb * fnb;
-                    if (p == MP_FP64) {
+                    if (p == MP_FP16H) {  // pure FP16 (four-level maps): tcgen05 with an F16 accumulator
+                        t16h.push_back(TcJob{m, n, A->tile(m, n), 0, 0});
+                    } else if (p == MP_FP64) {
                         if (E.crt) c64.push_back(CrtJob{m, n, A->tile(m, n)});
                         else g64.push_back(GemmJob{p64 + (size_t)m * nb2, p64 + (size_t)n * nb2, A->tile(m, n)});
                     } else if (p == MP_FP32 ? E.f32 != MP_F32_DMMA : E.tc16) {
@@ -1320,6 +1325,19 @@ static mp_status plan_potrf(mp_handle* h, mp_matrix* A, const uint8_t* km, const
                 }
                 cur->push_back({[=](cudaStream_t s) { return tc_gemm_f16_launch(ta, nj, s); }, C_UPD16, 2 * f3 * nj});
             }
+            if (!t16h.empty()) {
+                TcJob* dj = ar.push(t16h);
+                const int nj = (int)t16h.size();
+                TcArgs ta{};
+                ta.jobs = dj;
+                ta.nb = nb;
+                ta.nt = nt;
+                ta.h16hi = h16s;
+                ta.e16 = e16;
+                ta.cbase = cpool;
+                ta.crows = crows;
+                cur->push_back({[=](cudaStream_t s) { return tc_gemm_f16h_launch(ta, nj, s); }, C_UPD16, 2 * f3 * nj});
+            }
         }  // part
     }
     // ---- assemble the schedule
@@ -1364,8 +1382,11 @@ static mp_status potrf_run(mp_handle* h, mp_matrix* A, const uint8_t* km, const 
     for (int k = 0; k < nt; ++k)
         for (int m = k; m < nt; ++m) {
             const size_t i = (size_t)m * nt + k;
-            if (km[i] > MP_FP16 || cm[i] > MP_FP16 || (m == k && km[i] != MP_FP64))
+            if (km[i] > MP_FP16H || cm[i] > MP_FP16 || (m == k && km[i] != MP_FP64))
                 FAIL(h, MP_ERR_ARG, "bad map entry at (%d,%d)", m, k);
+            if (km[i] == MP_FP16H && !A->R.h16s)
+                FAIL(h, MP_ERR_UNSUPPORTED, "pure-FP16 tile (%d,%d): needs the tcgen05 FP16 engine and a matrix laid out "
+                     "for a four-level map (mp_eval with MP_MAP_ADAPTIVE4 / MP_MAP_USER)", m, k);
             if (m > k && A->st(m, k) != (km[i] == MP_FP64 ? MP_FP64 : MP_FP32) &&
                 !(A->st(m, k) == MP_FP16 && km[i] == MP_FP16 && h->cfg.fp16_storage))
                 FAIL(h, MP_ERR_ARG, "kernel map inconsistent with the bound storage map at (%d,%d)", m, k);
@@ -1672,7 +1693,7 @@ mp_status mp_eval(mp_handle* h, mp_matrix* A, const double* x, const double* y, 
     const size_t wsb = A->ws_bytes;
     std::vector<double> s(NN, 0.0);
     std::vector<uint8_t> km(NN, 255), sm(NN, 255), cm(NN, 255);
-    if (mode == MP_MAP_ADAPTIVE || mode == MP_MAP_BAND) {
+    if (mode == MP_MAP_ADAPTIVE || mode == MP_MAP_ADAPTIVE4 || mode == MP_MAP_BAND) {
         if (mp_status st = mp_matern_gen(h, A, dx, dy, theta, nullptr, s.data())) return st;
     }
     CK(h, cudaEventRecord(ev[1], h->stream));
@@ -1680,6 +1701,9 @@ mp_status mp_eval(mp_handle* h, mp_matrix* A, const double* x, const double* y, 
     switch (mode) {
         case MP_MAP_ADAPTIVE:
             st = mp_precision_map(nt, s.data(), u_req, eps, policy, km.data(), sm.data(), cm.data());
+            break;
+        case MP_MAP_ADAPTIVE4:  // four levels: eps = 4 entries or NULL
+            st = mp_precision_map4(nt, s.data(), u_req, eps, policy, km.data(), sm.data(), cm.data());
             break;
         case MP_MAP_BAND:
             band_kernel_map(nt, s.data(), u_req, eps, km);
@@ -1695,7 +1719,7 @@ mp_status mp_eval(mp_handle* h, mp_matrix* A, const double* x, const double* y, 
         case MP_MAP_USER:
             if (!user_kernel_prec) return MP_ERR_ARG;
             km.assign(user_kernel_prec, user_kernel_prec + NN);
-            st = mp_precision_map(nt, nullptr, u_req, eps, policy, km.data(), sm.data(), cm.data());
+            st = mp_precision_map4(nt, nullptr, u_req, eps, policy, km.data(), sm.data(), cm.data());
             break;
         default:
             return MP_ERR_ARG;
@@ -1707,6 +1731,9 @@ mp_status mp_eval(mp_handle* h, mp_matrix* A, const double* x, const double* y, 
                 const size_t i = (size_t)m * nt + k;
                 if (km[i] == MP_FP16) sm[i] = cm[i] = MP_FP16;
             }
+    A->h16h = false;  // the pure-FP16 operand planes only for a map that has such tiles
+    for (int k = 0; k < nt; ++k)
+        for (int m = k + 1; m < nt; ++m) A->h16h |= km[(size_t)m * nt + k] == MP_FP16H;
     {  // the workspace this map needs (tiles in storage precision + the map-independent regions)
         const size_t need = layout(A, sm.data()).total;
         rep->workspace_bytes = need;
@@ -1723,10 +1750,12 @@ mp_status mp_eval(mp_handle* h, mp_matrix* A, const double* x, const double* y, 
     for (int k = 0; k < nt; ++k)
         for (int m = k + 1; m < nt; ++m) {
             const size_t i = (size_t)m * nt + k;
-            rep->tiles[km[i]]++;
+            if (km[i] == MP_FP16H) rep->tiles_fp16h++;
+            else rep->tiles[km[i]]++;
             if (cm[i] > sm[i]) rep->stc_tiles++;
         }
     for (int c = 0; c < 3; ++c) rep->flops_update[c] = fc.upd[c];
+    rep->flops_update_fp16h = fc.upd[MP_FP16H];
     rep->flops_potrf = fc.potrf + fc.trsm;
     if (pst == MP_ERR_NOT_SPD) {
         rep->loglik = -HUGE_VAL;

@@ -85,6 +85,7 @@ struct Split16Item {
     __half* hi;         // row-scaled FP16 hi / lo (nb x nb); lo may be null (FP16 class only)
     __half* lo;
     int* exps;          // [nb]: 2^exps undoes row i's scale
+    __half* hs = nullptr;  // optional pure-FP16 operand rn(x 2^(s - 13)) (four-level maps)
 };
 cudaError_t split16_launch(const Split16Item* items, int n, int nb, cudaStream_t s);
 // p64 = (double) store

@@ -22,6 +22,10 @@
 // KIND 2 (FP32 class, 3xFP16, reading C13c): the same three products with an 11-bit hi/lo split in
 //   FP16 (kind::f16, twice the TF32 rate): each panel row is scaled by a power of two so its max is
 //   below 2^15 (split16_kernel, convert.cu); the epilogue multiplies by 2^(eA_i + eB_j).
+// KIND 3 (the paper's pure FP16 class, "A, B, C, and operation are all in FP16"; four-level
+//   maps): KIND 0 with an F16 accumulator (idesc dtype F16) over the whole K; the
+//   operands are the hs planes of split16_kernel (row max in [2, 4), so |sum| <= K 2^4 stays inside
+//   FP16's range), the epilogue widens the FP16 result to FP32 and multiplies by 2^(eA_i + eB_j + 26).
 #include <cudaTypedefs.h>
 #include <stdint.h>
 #include <stdlib.h>
@@ -38,10 +42,15 @@ constexpr int TC_BM = 128;  // output rows per CTA (TMEM lanes)
 #ifndef TC16X3_CHUNK_KB
 #define TC16X3_CHUNK_KB 2  // KIND 2: k-blocks of 64 per TMEM accumulator chunk (K = 128; measured 187 vs 181 Tflop/s at K = 64)
 #endif
+// TMEM layout of an F16 accumulator (tools/dbg/tmem_f16acc.cu): 0 = one FP16 per 32-bit column (low
+// half), 1 = two per column
+#ifndef TC_F16ACC_PACKED
+#define TC_F16ACC_PACKED 0
+#endif
 template <int KIND>
 struct TcThreads {
     // 3xTF32: two warpgroups, one per 128-column half; 3xFP16: TC16X3_EPI_WARPS / 4 column groups
-    static constexpr int EPI_WARPS = KIND == 0 ? 4 : KIND == 1 ? 8 : TC16X3_EPI_WARPS;
+    static constexpr int EPI_WARPS = (KIND == 0 || KIND == 3) ? 4 : KIND == 1 ? 8 : TC16X3_EPI_WARPS;
     static constexpr int N = (4 + EPI_WARPS) * 32;
 };
 
@@ -68,20 +77,21 @@ struct TcCfg {
     static constexpr int UK = KIND == 1 ? 8 : 16;  // K per tcgen05.mma (32 bytes)
     static constexpr int A_BYTES = TC_BM * 128;
     static constexpr int B_BYTES = (BN / CL) * 128;
-    static constexpr int STAGE_BYTES = KIND == 0 ? A_BYTES + B_BYTES : 2 * (A_BYTES + B_BYTES);
+    static constexpr bool ONE = KIND == 0 || KIND == 3;  // one operand plane each (FP16 class, pure FP16)
+    static constexpr int STAGE_BYTES = ONE ? A_BYTES + B_BYTES : 2 * (A_BYTES + B_BYTES);
     // KIND 0: 96 KB of stages so two CTAs share an SM (one's epilogue overlaps the other's main
     // loop; 2 x 256 TMEM columns); KIND 1: 192 KB, one CTA per SM (512 TMEM columns)
-    static constexpr int STAGES = (KIND == 0 ? 96 * 1024 : 192 * 1024) / STAGE_BYTES;
-    static constexpr int MIN_BLOCKS = KIND == 0 ? 2 : 1;
+    static constexpr int STAGES = (ONE ? 96 * 1024 : 192 * 1024) / STAGE_BYTES;
+    static constexpr int MIN_BLOCKS = ONE ? 2 : 1;
     static constexpr int SMEM = STAGES * STAGE_BYTES + 1024;
     // KIND 1: accumulate CHUNK_KB k-blocks (64 of K) per TMEM accumulator, two accumulators
     // ping-pong; the epilogue sums the chunks in FP32 registers (round-to-nearest), which keeps
     // the tensor core's non-RN FP32 accumulation error from growing with K (reading C13).
-    static constexpr int CHUNK_KB = KIND == 0 ? 1 << 20 : KIND == 1 ? 2 : TC16X3_CHUNK_KB;
-    static constexpr uint32_t TMEM_COLS = KIND == 0 ? BN : 2 * BN;  // power of two >= 32
+    static constexpr int CHUNK_KB = ONE ? 1 << 20 : KIND == 1 ? 2 : TC16X3_CHUNK_KB;
+    static constexpr uint32_t TMEM_COLS = ONE ? BN : 2 * BN;  // power of two >= 32
     // instruction descriptor: D = F32 (bit 4), A/B format (bits 7-9 / 10-12), K-major both,
     // N >> 3 (bits 17-22), M >> 4 (bits 24-28)
-    static constexpr uint32_t IDESC = (1u << 4) | ((KIND == 1 ? 2u : 0u) << 7) | ((KIND == 1 ? 2u : 0u) << 10) |
+    static constexpr uint32_t IDESC = ((KIND == 3 ? 0u : 1u) << 4) | ((KIND == 1 ? 2u : 0u) << 7) | ((KIND == 1 ? 2u : 0u) << 10) |
                                       ((uint32_t)(BN >> 3) << 17) | ((uint32_t)(BM >> 4) << 24);
 };
 
@@ -198,6 +208,16 @@ __device__ __forceinline__ void tmem_ld32(uint32_t taddr, uint32_t (&r)[32]) {
           "=r"(r[8]), "=r"(r[9]), "=r"(r[10]), "=r"(r[11]), "=r"(r[12]), "=r"(r[13]), "=r"(r[14]), "=r"(r[15]),
           "=r"(r[16]), "=r"(r[17]), "=r"(r[18]), "=r"(r[19]), "=r"(r[20]), "=r"(r[21]), "=r"(r[22]), "=r"(r[23]),
           "=r"(r[24]), "=r"(r[25]), "=r"(r[26]), "=r"(r[27]), "=r"(r[28]), "=r"(r[29]), "=r"(r[30]), "=r"(r[31])
+        : "r"(taddr));
+    asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
+}
+
+// 16 consecutive 32-bit TMEM columns of the warp's 32 lanes (KIND 3 with packed FP16 accumulators)
+__device__ __forceinline__ void tmem_ld16(uint32_t taddr, uint32_t (&r)[32]) {
+    asm volatile(
+        "tcgen05.ld.sync.aligned.32x32b.x16.b32 {%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15}, [%16];"
+        : "=r"(r[0]), "=r"(r[1]), "=r"(r[2]), "=r"(r[3]), "=r"(r[4]), "=r"(r[5]), "=r"(r[6]), "=r"(r[7]),
+          "=r"(r[8]), "=r"(r[9]), "=r"(r[10]), "=r"(r[11]), "=r"(r[12]), "=r"(r[13]), "=r"(r[14]), "=r"(r[15])
         : "r"(taddr));
     asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
 }
@@ -328,7 +348,7 @@ __global__ void __launch_bounds__(TcThreads<KIND>::N, TcCfg<KIND, CL>::MIN_BLOCK
             const uint32_t fb = CL > 1 ? cluster_addr(lb, 0) : lb;
             if (crank == 0) mbar_expect_tx(lb, CL * Cfg::STAGE_BYTES);
             const int kc = kb * Cfg::BK;
-            if (KIND == 0) {
+            if (Cfg::ONE) {
                 tma_load_2d<CL>(st, &p.a, fb, kc, rowA);
                 tma_load_2d<CL>(st + Cfg::A_BYTES, &p.b, fb, kc, rowB);
             } else {
@@ -345,8 +365,8 @@ __global__ void __launch_bounds__(TcThreads<KIND>::N, TcCfg<KIND, CL>::MIN_BLOCK
             const uint32_t ph = (uint32_t)(kb / Cfg::STAGES) & 1u;
             const int chunk = kb / Cfg::CHUNK_KB, kin = kb % Cfg::CHUNK_KB;
             const uint32_t abuf = (uint32_t)(chunk & 1);
-            const uint32_t dacc = KIND == 0 ? tmem : tmem + abuf * Cfg::BN;
-            if (KIND != 0 && kin == 0) {  // wait until the epilogues drained this accumulator
+            const uint32_t dacc = Cfg::ONE ? tmem : tmem + abuf * Cfg::BN;
+            if (!Cfg::ONE && kin == 0) {  // wait until the epilogues drained this accumulator
                 mbar_wait(smem_u32(&acc_empty[abuf]), ((uint32_t)(chunk >> 1) & 1u) ^ 1u);
                 tc_fence_after();
             }
@@ -357,8 +377,8 @@ __global__ void __launch_bounds__(TcThreads<KIND>::N, TcCfg<KIND, CL>::MIN_BLOCK
             for (int k = 0; k < Cfg::BK / Cfg::UK; ++k) {
                 const uint32_t koff = k * 32;  // bytes along K inside the 128-byte swizzle atom
                 const uint32_t acc = (kin | k) != 0;
-                if (KIND == 0) {
-                    tc_mma<0, CL>(dacc, desc_sw128(base + koff), desc_sw128(base + Cfg::A_BYTES + koff), acc);
+                if (Cfg::ONE) {
+                    tc_mma<KIND, CL>(dacc, desc_sw128(base + koff), desc_sw128(base + Cfg::A_BYTES + koff), acc);
                 } else {
                     const uint64_t ahi = desc_sw128(base + koff);
                     const uint64_t alo = desc_sw128(base + Cfg::A_BYTES + koff);
@@ -370,9 +390,9 @@ __global__ void __launch_bounds__(TcThreads<KIND>::N, TcCfg<KIND, CL>::MIN_BLOCK
                 }
             }
             tc_commit<CL>(smem_u32(&empty_bar[s]));
-            if (KIND != 0 && (kin == Cfg::CHUNK_KB - 1 || kb == KB - 1)) tc_commit<CL>(smem_u32(&acc_full[abuf]));
+            if (!Cfg::ONE && (kin == Cfg::CHUNK_KB - 1 || kb == KB - 1)) tc_commit<CL>(smem_u32(&acc_full[abuf]));
         }
-        if (KIND == 0) tc_commit<CL>(smem_u32(&done_bar));
+        if (Cfg::ONE) tc_commit<CL>(smem_u32(&done_bar));
     } else if (warp >= 4) {
         // ---------------- epilogue: C -= acc.  Warp w reads TMEM lanes 32 (w % 4) .. +31 (its rows);
         // with 8 epilogue warps the two warpgroups split the columns in halves.  The stage ring is
@@ -385,23 +405,35 @@ __global__ void __launch_bounds__(TcThreads<KIND>::N, TcCfg<KIND, CL>::MIN_BLOCK
         const int ccol0 = bj * Cfg::BN + half * COLS;
         const uint32_t tl = ((uint32_t)(q * 32) << 16) + (uint32_t)(half * COLS);
         const uint32_t stg = smem_u32(smem) + (uint32_t)(warp - 4) * 8192u;  // two 4 KB boxes per warp
-        if (KIND == 0) {
-            const float ra = __int_as_float((p.exps[rowA + q * 32 + lane] + 127) << 23);
+        if (Cfg::ONE) {
+            // KIND 3: the hs planes carry an extra 2^-13 per operand (split16_kernel)
+            const float ra = __int_as_float((p.exps[rowA + q * 32 + lane] + (KIND == 3 ? 26 : 0) + 127) << 23);
             const int4* eb = (const int4*)(p.exps + jb.n * p.nb + ccol0);
             mbar_wait(smem_u32(&done_bar), 0);
             tc_fence_after();
 #pragma unroll 1
             for (int g = 0; g < COLS / 32; ++g) {
                 uint32_t r[32];
-                tmem_ld32(tmem + tl + (uint32_t)(g * 32), r);
+                float v[32];
+                if (KIND == 3 && TC_F16ACC_PACKED) {  // two FP16 accumulators per 32-bit TMEM column
+                    tmem_ld16(tmem + tl + (uint32_t)(g * 16), r);
+#pragma unroll
+                    for (int i = 0; i < 16; ++i) {
+                        const float2 f = __half22float2(*(const __half2*)&r[i]);
+                        v[2 * i] = f.x;
+                        v[2 * i + 1] = f.y;
+                    }
+                } else {
+                    tmem_ld32(tmem + tl + (uint32_t)(g * 32), r);
+#pragma unroll
+                    for (int i = 0; i < 32; ++i)
+                        v[i] = KIND == 3 ? __half2float(__ushort_as_half((unsigned short)(r[i] & 0xffffu))) : __uint_as_float(r[i]);
+                }
                 const uint32_t buf = stg + (uint32_t)(g & 1) * 4096u;
                 if (g >= 2) {
                     if (lane == 0) bulk_wait_read_1();
                     __syncwarp();
                 }
-                float v[32];
-#pragma unroll
-                for (int i = 0; i < 32; ++i) v[i] = __uint_as_float(r[i]);
                 scale_group(v, ra, eb + g * 8);  // undo the operands' power-of-two row scales
                 if (p.c16) stage_box_neg16(buf, lane, v, __int_as_float((jb.cscale + 127) << 23));
                 else stage_box_neg(buf, lane, v);
@@ -686,7 +718,7 @@ static cudaError_t launch(const TcArgs& a, int njobs, cudaStream_t s) {
     const uint64_t rows = (uint64_t)a.nt * a.nb;
     constexpr uint32_t BROWS = Cfg::BN / CL;
     bool ok;
-    if (KIND == 0) {
+    if (KIND == 0 || KIND == 3) {
         ok = a.h16hi && a.e16 &&
              make_map(&p.a, a.h16hi, CU_TENSOR_MAP_DATA_TYPE_FLOAT16, 2, rows, a.nb, Cfg::BK, TC_BM) &&
              make_map(&p.b, a.h16hi, CU_TENSOR_MAP_DATA_TYPE_FLOAT16, 2, rows, a.nb, Cfg::BK, BROWS);
@@ -754,6 +786,9 @@ static cudaError_t launch(const TcArgs& a, int njobs, cudaStream_t s) {
 
 // CTA pairs (cta_group::2) for every kind: faster than single CTAs for both (profiles/r01/README.md)
 cudaError_t tc_gemm_f16_launch(const TcArgs& a, int njobs, cudaStream_t s) { return launch<0, 2>(a, njobs, s); }
+cudaError_t tc_gemm_f16h_launch(const TcArgs& a, int njobs, cudaStream_t s) {
+    return a.c16 ? cudaErrorInvalidValue : launch<3, 2>(a, njobs, s);
+}
 cudaError_t tc_gemm_f16x3_launch(const TcArgs& a, int njobs, cudaStream_t s) { return launch<2, 2>(a, njobs, s); }
 cudaError_t tc_gemm_tf32x3_launch(const TcArgs& a, int njobs, cudaStream_t s) { return launch<1, 2>(a, njobs, s); }
 

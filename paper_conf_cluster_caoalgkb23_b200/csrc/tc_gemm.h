@@ -41,5 +41,8 @@ struct TcArgs {
 bool tc_gemm_available();
 cudaError_t tc_gemm_tf32x3_launch(const TcArgs& a, int njobs, cudaStream_t s);
 cudaError_t tc_gemm_f16_launch(const TcArgs& a, int njobs, cudaStream_t s);
+// pure-FP16 class (four-level maps): h16hi = the hs planes (split16_kernel, extra 2^-13 per row), F16
+// accumulation in TMEM over the whole K, FP32 C
+cudaError_t tc_gemm_f16h_launch(const TcArgs& a, int njobs, cudaStream_t s);
 cudaError_t tc_gemm_f16x3_launch(const TcArgs& a, int njobs, cudaStream_t s);
 }  // namespace mpgeo

@@ -82,7 +82,7 @@ mp_status mp_test_tc_gemm(int kind, const void* d_panel, const void* d_panel_lo,
 mp_status mp_test_tc_gemm_split(int kind, const double* d_panel, float* d_C, int nb, int nt, int m, int n,
                                 int persistent) {
     if (!tc_gemm_available()) return MP_ERR_UNSUPPORTED;
-    if (kind != 0 && kind != 2) return MP_ERR_ARG;
+    if (kind != 0 && kind != 2 && kind != 3) return MP_ERR_ARG;  // 3: pure FP16 (F16 accumulation, hs planes)
     const size_t elems = (size_t)nt * nb * nb;
     __half *hi = nullptr, *lo = nullptr;
     int* ex = nullptr;
@@ -97,8 +97,9 @@ mp_status mp_test_tc_gemm_split(int kind, const double* d_panel, float* d_C, int
     if (e == cudaSuccess) e = cudaMalloc(&di, nt * sizeof(Split16Item));
     if (e == cudaSuccess) {
         for (int t = 0; t < nt; ++t)  // the FP16 class derives hi only (lo stays untouched)
-            items.push_back({d_panel + (size_t)t * nb * nb, hi + (size_t)t * nb * nb,
-                             kind == 2 ? lo + (size_t)t * nb * nb : nullptr, ex + (size_t)t * nb});
+            items.push_back({d_panel + (size_t)t * nb * nb, kind == 3 ? nullptr : hi + (size_t)t * nb * nb,
+                             kind == 2 ? lo + (size_t)t * nb * nb : nullptr, ex + (size_t)t * nb,
+                             kind == 3 ? hi + (size_t)t * nb * nb : nullptr});
         cudaMemcpy(dj, &j, sizeof j, cudaMemcpyHostToDevice);
         cudaMemcpy(di, items.data(), nt * sizeof(Split16Item), cudaMemcpyHostToDevice);
         e = split16_launch(di, nt, nb, 0);
@@ -114,7 +115,7 @@ mp_status mp_test_tc_gemm_split(int kind, const double* d_panel, float* d_C, int
         a.cbase = d_C;
         a.crows = (uint64_t)nb;
         a.persistent = persistent;
-        e = kind == 2 ? tc_gemm_f16x3_launch(a, 1, 0) : tc_gemm_f16_launch(a, 1, 0);
+        e = kind == 2 ? tc_gemm_f16x3_launch(a, 1, 0) : kind == 3 ? tc_gemm_f16h_launch(a, 1, 0) : tc_gemm_f16_launch(a, 1, 0);
     }
     cudaError_t e2 = cudaDeviceSynchronize();
     cudaFree(hi);

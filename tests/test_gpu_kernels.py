@@ -237,3 +237,33 @@ def test_crt_int8_syrk_lower(lib):
                 assert np.array_equal(got[blk], Cm[blk])
             else:
                 assert np.max(np.abs(got[blk] - ref[blk])) <= 8 * nb * 2.0**-53 * np.abs(A).max() ** 2
+
+
+@pytest.mark.parametrize("scale", [1.0, 4e-8])
+def test_tc_gemm_pure_fp16_accumulates_in_fp16(lib, scale):
+    """Pure FP16 class (four-level maps, "A, B, C, and operation are all in FP16"): row-scaled FP16
+    operands (the hs planes) and an F16 TMEM accumulator over the whole K.  Pins: (i) the error against the
+    exact product of the FP32-rounded operands stays within the FP16-accumulation bound
+    (2^-10 + K 2^-11) |A||B|^T entrywise; (ii) it is the FP16 accumulator that ran: the normwise error is
+    several times the FP16_32 kernel's on the same operands (FP32 accumulation), and close to an emulated
+    FP16 accumulation; (iii) no overflow at the C3 FP16-class magnitude (scale 4e-8) thanks to the row scale."""
+    assert lib.mp_tc_available() == 1
+    nb, nt = 2048, 2
+    rng = np.random.default_rng(11)
+    P = np.abs(rng.standard_normal((nt * nb, nb))) * scale * np.exp2(-rng.integers(0, 6, size=(nt * nb, 1)))
+    out = {}
+    for kind in (0, 3):
+        dP, dC = dev(P), dev(np.zeros((nb, nb), np.float32))
+        assert lib.mp_test_tc_gemm_split(kind, C.c_void_p(dP.data_ptr()), C.c_void_p(dC.data_ptr()), nb, nt, 1, 0, 0) == 0
+        out[kind] = -dC.cpu().numpy().astype(np.float64)
+    A32 = P.astype(np.float32).astype(np.float64)
+    A, B = A32[nb:2 * nb], A32[0:nb]
+    exact = A @ B.T
+    assert np.all(np.isfinite(out[3]))
+    bound = (2.0**-10 + nb * 2.0**-11) * (np.abs(A) @ np.abs(B).T)
+    assert np.all(np.abs(out[3] - exact) <= bound)
+    e3 = np.linalg.norm(out[3] - exact) / np.linalg.norm(exact)
+    e0 = np.linalg.norm(out[0] - exact) / np.linalg.norm(exact)
+    print(f"scale {scale}: pure FP16 {e3:.3e}, FP16_32 {e0:.3e}, ratio {e3 / e0:.1f}")
+    assert e3 > 3 * e0, (e3, e0)   # positive entries: FP16 accumulation error grows with K
+    assert e3 < 2.0**-4, e3

@@ -189,6 +189,40 @@ def test_mixed_precision_path(mp, handle, beta):
 
 
 @pytest.mark.parametrize("beta", [0.03, 0.1])
+def test_four_level_precision_path(mp, handle, beta):
+    """Four-level maps (P:113 / P:117 "FP64, FP32, FP16_32, and FP16"; MP_MAP_ADAPTIVE4 with
+    the library's default eps = (2^-52, 2^-23, MP_EPS_FP16_32, 2^-10)): maps bit-exact vs the oracle's
+    four-level rule, pure-FP16 tiles present and run through the F16-accumulator kernel, l within the
+    north-star 1e-5 of the FP64 oracle, and the factor's backward error within the bound the maps imply
+    (FP16 accumulation unit 2^-11 for the pure-FP16 class, tests/gpu_helpers.py)."""
+    from oracle import FP16H
+    n, nb, u_req = 10000, 512, 1e-9
+    theta = (1.0, beta, 0.5)
+    eps4 = (2.0**-52, 2.0**-23, mp.MP_EPS_FP16_32, 2.0**-10)
+    x, y = synth.locations(n, 0)
+    z = synth.normal_vector(n, 1)
+    ref = oracle_loglik(x, y, z, theta, nb)
+    nt = num_tiles(n, nb)
+    so = tile_sqnorms(ref["tiles"], nt)
+    near_tie_guard(so, nt, u_req, eps4)
+    maps = precision_maps(so, u_req, eps=eps4)
+    ev = mp.Evaluator(n, nb, handle=handle)
+    r = ev.eval(x, y, z, theta, u_req=u_req, mode=mp.MP_MAP_ADAPTIVE4)
+    km, sm, cm = ev.M.maps()
+    low = np.tril(np.ones((nt, nt), bool))
+    for g, o in zip((km, sm, cm), maps):
+        assert np.array_equal(g[low], o[low])
+    n16h = int((km[np.tril(np.ones((nt, nt), bool), -1)] == FP16H).sum())
+    assert r.tiles_fp16h == n16h and (beta > 0.05 or n16h > 0)
+    err = abs(r.loglik - ref["loglik"]) / abs(ref["loglik"])
+    print(f"beta {beta}: tiles FP64/FP32/FP16_32/FP16 = {list(r.tiles)} + {r.tiles_fp16h}, l rel. error {err:.2e}")
+    assert err <= 1e-5  # north-star MP tolerance
+    Lhat = {key: ev.M.tile(*key)[: t.shape[0], : t.shape[1]] for key, t in ref["tiles"].items()}
+    worst, _ = mp_backward_check(ref["tiles"], Lhat, ref["factor"], km, sm, cm, nt, nb)
+    assert worst <= 1.0, worst
+
+
+@pytest.mark.parametrize("beta", [0.03, 0.1])
 def test_extreme_map_stc_and_ttc(mp, handle, beta):
     """P:294 extreme FP64/FP16 map: AUTO -> every communication STC; TTC keeps storage precision.
     Pass criteria (no emulation): the GPU factor's backward error per tile within the bound the maps
