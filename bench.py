@@ -229,7 +229,7 @@ def main():
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--config", default="c5", choices=sorted(CONFIGS))
-    ap.add_argument("--map", default=None, choices=["adaptive", "fp64", "band", "extreme"])
+    ap.add_argument("--map", default=None, choices=["adaptive", "adaptive4", "fp64", "band", "extreme"])
     ap.add_argument("--policy", default="auto", choices=["auto", "ttc"])
     ap.add_argument("--u-req", type=float, default=1e-9)
     ap.add_argument("--theta", default=None, help="sigma2,beta,nu override (e.g. 1,0.03,0.8 for the Bessel path)")
@@ -276,8 +276,8 @@ def main():
         # path is the library's own peer-memory exchange), so gloo is enough
         dist.init_process_group("gloo")
     n, nb, theta = cfg["n"], cfg["nb"], cfg["theta"]
-    mode = {"adaptive": mp.MP_MAP_ADAPTIVE, "fp64": mp.MP_MAP_FP64, "band": mp.MP_MAP_BAND,
-            "extreme": mp.MP_MAP_EXTREME}[cfg["map"]]
+    mode = {"adaptive": mp.MP_MAP_ADAPTIVE, "adaptive4": mp.MP_MAP_ADAPTIVE4, "fp64": mp.MP_MAP_FP64,
+            "band": mp.MP_MAP_BAND, "extreme": mp.MP_MAP_EXTREME}[cfg["map"]]
     policy = mp.MP_COMM_AUTO if args.policy == "auto" else mp.MP_COMM_TTC
     distributed = world > 1 and not args.replicas
     seed = 0 if distributed or world == 1 else rank
@@ -371,7 +371,7 @@ def main():
         te = max_over_ranks(es.elapsed_time(ee))
         nt = ev.nt
         chunks = (n + 4095) // 4096
-        d2h = (nt * (nt + 1) // 2) * 8 if mode in (mp.MP_MAP_ADAPTIVE, mp.MP_MAP_BAND) else 0
+        d2h = (nt * (nt + 1) // 2) * 8 if mode in (mp.MP_MAP_ADAPTIVE, mp.MP_MAP_ADAPTIVE4, mp.MP_MAP_BAND) else 0
         d2h += 4 + (nt + chunks) * 8
         e2e = {"value": evals_per_step * ke * flops_eval / (te / 1e3) / 1e12, "unit": "Tflop/s",
                "h2d_bytes_per_step": 3 * n * 8, "d2h_bytes_per_step": d2h, "ms_per_step": te / ke, "steps": ke}
@@ -407,6 +407,7 @@ def main():
     traffic = (tr["dram_bytes_per_flop"] * flops_per_launch) if tr else None
     last = reps[-1]
     upd = list(last.flops_update)
+    upd[2] += last.flops_update_fp16h  # four-level maps: the pure-FP16 class runs at the f16 rate too (class upd_fp16)
     # update time at the engines' peaks (FP64 class at INT8 peak / 16 with CRT, FP32 class at the f16 rate / 3
     # (3xFP16) or TF32 / 3, FP16 class at the f16 rate) and at the NATIVE peaks of the classes (FP64 DMMA, TF32
     # for the FP32 class as the survey's 3xTF32 plan counts it — 1 product —, FP16)
@@ -451,6 +452,8 @@ def main():
         "factorization_tflops": flops_eval / (potrf_ms / 1e3) / 1e12 if potrf_ms > 0 else None,
         "joules_per_eval": None if joules is None else joules / args.steps,
         "loglik": last.loglik, "tiles_fp64_fp32_fp16": list(last.tiles), "stc_tiles": last.stc_tiles,
+        **({"tiles_pure_fp16": last.tiles_fp16h, "flops_update_pure_fp16": last.flops_update_fp16h}
+           if cfg["map"] == "adaptive4" else {}),
         "flops_update_per_class": upd,
         "phase_ms": {"gen+map": last.t_gen_ms, "potrf": last.t_potrf_ms, "solve": last.t_solve_ms},
         "profile": None if prof is None else {
