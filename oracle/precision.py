@@ -2,7 +2,10 @@
 
 Three precision classes (reading C7): FP64 > FP32 > FP16, encoded 0/1/2 (smaller
 = higher precision).  "FP16" is the paper's FP16_32 (FP16 operands, FP32
-accumulation and storage; P:113, P:146, P:152).
+accumulation and storage).  Four-level maps ("we
+incorporate FP64, FP32, FP16_32, and FP16") add FP16H = 3, the
+paper's pure FP16 class (FP16 operands and accumulation), tried before FP16_32
+with its own epsilon (eps = 4-tuple; reading C7' in DESIGN.md for FP16_32's).
 
 kernel map  (§V; readings C6, C7):
     kernel(k, k) = FP64  ("computations ... on tiles ... along the diagonal ...
