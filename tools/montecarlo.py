@@ -54,7 +54,8 @@ def main():
         rec["seconds"] = time.time() - t0
         print(json.dumps(rec), flush=True)
         reps.append(rec)
-        json.dump({"partial": reps}, open(f"gpurun_out/montecarlo_n{n}_R{R}_b{beta}_nu{nu}.json", "w"), indent=1)
+        json.dump({"partial": reps, "theta_true": theta_true, "n": n, "u_req": u_req, "maxfev": maxfev},
+                  open(f"gpurun_out/montecarlo_n{n}_R{R}_b{beta}_nu{nu}.json", "w"), indent=1)
     a64 = np.array([q["fp64"] for q in reps if "fp64" in q])
     amp = np.array([q["mp"] for q in reps])
     out = {"n": n, "nb": nb, "replicas": R, "fp64_replicas": len(a64), "u_req": u_req, "theta_true": theta_true,
