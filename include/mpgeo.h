@@ -72,8 +72,9 @@ typedef enum { MP_FP64 = 0, MP_FP32 = 1, MP_FP16 = 2, MP_FP16H = 3 } mp_prec;
 /* u_low of the FP16_32 class in four-level maps.  The paper fixes it "experimentally" (citing
  * [23]: FP16_32 has a lower error bound than FP16) and prints no value; reading C7': the
  * ratio of the measured tile-GEMM errors of the FP16_32 and pure-FP16 classes on the application's
- * FP16-class tiles times FP16's machine epsilon 2^-10 (tools/fp16_eps.py). */
-#define MP_EPS_FP16_32 (1.0 / 8192.0)
+ * FP16-class tiles times FP16's machine epsilon 2^-10 (tools/fp16_eps.py; measured on the C2 factor:
+ * median ratio 0.058 -> 5.7e-5, rounded UP to a power of two: 2^-14; profiles/r02/fp16h/fp16_eps.json). */
+#define MP_EPS_FP16_32 (1.0 / 16384.0)
 
 /* Communication-precision policy.
  * MP_COMM_TTC : target-task conversion — every tile travels in its storage

@@ -18,7 +18,7 @@ STATUS_NAMES = ["MP_OK", "MP_ERR_ARG", "MP_ERR_NOT_SPD", "MP_ERR_CUDA", "MP_ERR_
 MP_FP64, MP_FP32, MP_FP16, MP_FP16H = 0, 1, 2, 3  # MP_FP16 = FP16_32; MP_FP16H = pure FP16 (four-level maps)
 MP_COMM_TTC, MP_COMM_AUTO = 0, 1
 MP_MAP_ADAPTIVE, MP_MAP_FP64, MP_MAP_BAND, MP_MAP_EXTREME, MP_MAP_USER, MP_MAP_ADAPTIVE4 = range(6)
-MP_EPS_FP16_32 = 1.0 / 8192.0  # include/mpgeo.h
+MP_EPS_FP16_32 = 1.0 / 16384.0  # include/mpgeo.h (reading C7')
 MP_COV_MATERN, MP_COV_SQEXP = 0, 1
 MP_F64_CRT16, MP_F64_DMMA = 0, 1
 MP_F32_3XFP16, MP_F32_3XTF32, MP_F32_DMMA = 0, 1, 2

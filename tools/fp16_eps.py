@@ -10,7 +10,8 @@ FP64 product: e_c = ||C_c - L_mk L_nk^T||_F / (||L_mk||_F ||L_nk||_F).  Then
 
     eps(FP16_32) = 2^-10 * median(e_FP16_32 / e_FP16)      (FP16's u_low = its machine epsilon 2^-10)
 
-rounded down to a power of two (the value the library ships as MP_EPS_FP16_32).  Output:
+rounded UP to a power of two (the conservative side: a larger eps gives the FP16_32 class fewer
+tiles; the value the library ships as MP_EPS_FP16_32).  Output:
 gpurun_out/fp16_eps.json.  python tools/fp16_eps.py [n] [samples]"""
 import ctypes as C
 import json
@@ -61,7 +62,7 @@ def main():
     eps = 2.0**-10 * ratio
     out = {"n": n, "nb": nb, "theta": theta, "u_req": u_req, "three_level_tiles": list(r.tiles), "samples": rows,
            "median_ratio_e16_32_over_e16": ratio, "eps_fp16_32": eps,
-           "eps_fp16_32_pow2": 2.0 ** math.floor(math.log2(eps)),
+           "eps_fp16_32_pow2": 2.0 ** math.ceil(math.log2(eps)),
            "definition": "eps(FP16_32) = 2^-10 * median over FP16-class GEMMs of ||C_16_32 - C|| / ||C_16 - C|| "
                          "(normwise, vs the FP64 product of the FP32-rounded operands)"}
     os.makedirs("gpurun_out", exist_ok=True)
