@@ -385,6 +385,14 @@ def main():
         prof = h.profile().as_dict()
         h.set_profiling(False)
 
+    # per-rank view (N > 1): own wall time of the timed steps and device-busy time per update class of the
+    # profiled evaluation, gathered on rank 0 (the driver's max-over-ranks value stays the headline)
+    mine = {"rank": rank, "device": local, "ms_per_step": evs[0].elapsed_time(evs[-1]) / args.steps,
+            "busy_ms": None if prof is None else {k: round(v["ms"], 1) for k, v in prof.items()}}
+    per_rank = [mine]
+    if dist:
+        per_rank = [None] * world
+        dist.all_gather_object(per_rank, mine)
     if rank != 0:
         if dist:
             dist.destroy_process_group()
@@ -489,6 +497,7 @@ def main():
              "cublas_dgemm_tflops_live": cub, "frac_vs_cublas_dgemm": (fp64_eq / cub) if cub else None}),
         "gpu_launches": launches,
         "clocks": ck,
+        **({"grid": f"{P}x{Q}", "per_rank": per_rank} if world > 1 else {}),
         "e2e": e2e,
     }
     if world == 1 and not args.no_cpu_baseline:
