@@ -243,7 +243,8 @@ constexpr uint32_t TMEM_COLS = 512;  // two 256-column accumulators
 #ifndef CRT_L2HINT
 #define CRT_L2HINT 0
 #endif
-// 1: the first scratch group of each pair step's reconstruction is loaded before the residue steps
+// 1: the first scratch group of each pair step's reconstruction is loaded before the residue steps;
+// 2: between the two residue steps
 #ifndef CRT_EARLY
 #define CRT_EARLY 0
 #endif
@@ -769,7 +770,7 @@ __global__ void __launch_bounds__(THREADS, 1) crt_gemm_kernel(const __grid_const
                 // reconstruction loaded into registers now (its latency hides behind the residue steps)
                 uint4 wa[NP];
                 if (pv) {
-                    if (CRT_EARLY) {
+                    if (CRT_EARLY == 1) {
                         if (jj == 0) prefetch_groups(0, GROUPS / NP);
                         if (jj + 1 < NP) prefetch_groups(((jj + 1) * GROUPS) / NP, ((jj + 2) * GROUPS) / NP);
                         load_group((jj * GROUPS) / NP, wa);
@@ -806,6 +807,7 @@ __global__ void __launch_bounds__(THREADS, 1) crt_gemm_kernel(const __grid_const
                     ++g;
                     PROF_ADD(pw_resid);
                 }
+                if (CRT_EARLY == 2 && pv) load_group((jj * GROUPS) / NP, wa);  // in flight during modulus b
                 // ---- second modulus b: R = r_a + a ((r_b - r_a) a^-1 mod b) in [0, ab), stored as uint16
                 {
                     const uint32_t buf = g & 1u;
@@ -853,7 +855,7 @@ __global__ void __launch_bounds__(THREADS, 1) crt_gemm_kernel(const __grid_const
                 if (pv) {
                     PROF_T0();
                     const int g0 = (jj * GROUPS) / NP, g1 = ((jj + 1) * GROUPS) / NP;
-                    if (!CRT_EARLY) load_group(g0, wa);
+                    if (CRT_EARLY == 0) load_group(g0, wa);
                     if constexpr (EPI_WARPS == 8) {  // two groups in flight
                         uint4 wb[NP];
                         for (int gi = g0; gi < g1; gi += 2) {
