@@ -28,6 +28,16 @@ case $1 in
     run c3_fp64_dmma --config c3 --map fp64 --engine fp64_engine=1
     run c3_adaptive_dmma --config c3 --engine fp64_engine=1
     run c3_nolook --config c3 --engine lookahead=0 ;;
+  r3)  # refresh after the integer CRT reconstruction (session 3) + the four-level map + reserve pairs at C5
+    run c3_adaptive_v3 --config c3
+    run c3_fp64_crt_v3 --config c3 --map fp64
+    run c3_fp64_dmma_v3 --config c3 --map fp64 --engine fp64_engine=1
+    run c3_adaptive4_v3 --config c3 --map adaptive4
+    run c2_adaptive_v3 --config c2 --map adaptive
+    run c2_fp64_v3 --config c2 --map fp64
+    run c2_adaptive4_v3 --config c2 --map adaptive4
+    run c5_rp3_v3 --config c5 --engine reserve_pairs=3
+    run c5_rp9_v3 --config c5 --engine reserve_pairs=9 ;;
   sens)
     run c3_ureq1e-8 --config c3 --u-req 1e-8
     run c3_nu1 --config c3 --theta 1,0.03,1.0
