@@ -45,6 +45,7 @@ CONFIGS = {
     "c5": dict(n=250000, nb=2048, theta=(1.0, 0.03, 0.5), map="adaptive"),
     "c2a": dict(n=40000, nb=2048, theta=(1.0, 0.03, 0.5), map="adaptive"),  # C2 size, adaptive map (tools)
     "c0": dict(n=4096, nb=512, theta=(1.0, 0.03, 0.5), map="adaptive"),      # small case (sanitizers, tools)
+    "c0q": dict(n=4096, nb=512, theta=(1.0, 0.03, 0.5), map="adaptive4"),    # the same, four-level map (tools)
 }
 METRIC = "Tflop/s & joules per MLE log-likelihood eval (n=360k) at 1/2/4/8 B200"
 FP64_NOMINAL, BF16_NOMINAL, INT8_NOMINAL = 40.0, 2250.0, 4500.0  # dense TFLOP/s (TOP/s), B200 nominal

@@ -20,12 +20,12 @@ def main():
     z = synth.normal_vector(n, seed=1)
     dx, dy, dz = (torch.from_numpy(v).cuda() for v in (x, y, z))
     ev = mp.Evaluator(n, nb)
-    mode = {"adaptive": mp.MP_MAP_ADAPTIVE, "fp64": mp.MP_MAP_FP64, "band": mp.MP_MAP_BAND,
-            "extreme": mp.MP_MAP_EXTREME}[cfg["map"]]
+    mode = {"adaptive": mp.MP_MAP_ADAPTIVE, "adaptive4": mp.MP_MAP_ADAPTIVE4, "fp64": mp.MP_MAP_FP64,
+            "band": mp.MP_MAP_BAND, "extreme": mp.MP_MAP_EXTREME}[cfg["map"]]
     for _ in range(warm + 1):
         r = ev.eval(dx, dy, dz, cfg["theta"], u_req=1e-9, mode=mode)
     torch.cuda.synchronize()
-    print(f"l = {r.loglik:.10f}, launches {r.gpu_launches}")
+    print(f"l = {r.loglik:.10f}, launches {r.gpu_launches}, tiles {list(r.tiles)} + pure FP16 {r.tiles_fp16h}")
 
 
 if __name__ == "__main__":

@@ -9,3 +9,9 @@ for tool in memcheck racecheck synccheck initcheck; do
     > gpurun_out/sanitizer_$tool.log 2>&1
   echo "$tool rc=$?" | tee -a gpurun_out/sanitizer_$tool.log
 done
+# the four-level map (pure-FP16 kernel with the F16 accumulator, hs planes)
+for tool in memcheck synccheck; do
+  timeout 1200 compute-sanitizer --tool $tool --print-limit 20 --error-exitcode 9 python tools/one_eval.py c0q 1 \
+    > gpurun_out/sanitizer_${tool}_c0q.log 2>&1
+  echo "$tool c0q rc=$?" | tee -a gpurun_out/sanitizer_${tool}_c0q.log
+done

@@ -37,7 +37,8 @@ case $1 in
     run c2_fp64_v3 --config c2 --map fp64
     run c2_adaptive4_v3 --config c2 --map adaptive4
     run c5_rp3_v3 --config c5 --engine reserve_pairs=3
-    run c5_rp9_v3 --config c5 --engine reserve_pairs=9 ;;
+    run c5_rp9_v3 --config c5 --engine reserve_pairs=9
+    bash tools/sanitize.sh ;;
   sens)
     run c3_ureq1e-8 --config c3 --u-req 1e-8
     run c3_nu1 --config c3 --theta 1,0.03,1.0
