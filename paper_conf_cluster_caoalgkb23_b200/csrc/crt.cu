@@ -6,27 +6,29 @@
 // tile with max_j |x_ij| < 2^{e_i} becomes the integer row x'_ij = rint(x_ij 2^{b - e_i}), |x'| <=
 // 2^b (exact in FP64: x has 53 significant bits), stored as N int8 residue planes x'_ij mod p_t
 // (symmetric representative in [-128, 127]) for N pairwise coprime moduli p_t <= 256.
-// Product: X_ij = sum_k x'_ik y'_jk is an integer with |X| <= K 2^{2b} < M/2, M = prod p_t, so it is
-// fixed by its residues.  Per modulus one INT8 GEMM (kind::i8, exact INT32 accumulation in TMEM:
-// |acc| <= K 128^2 = 2^25) gives acc_t == X (mod p_t); the epilogue reduces it to r_t in
-// [-128, 127] and, once all N are known, reconstructs
-//     X = sum_t r_t w_t  -  q M,   w_t = (M/p_t) ((M/p_t)^-1 mod p_t),  q = rint(sum_t r_t w_t / M)
-// in FP64 with w_t = H_t + L_t split so that sum_t r_t H_t is exact (H_t: < 42 significant bits,
-// multiples of 2^85) and the L part errs by < 2^49 absolute, far below the final rounding of X
-// (|X| ~ 2^{2b}).  Then C_ij -= X 2^{e_i - b} 2^{f_j - b} (exact scalings, one FP64 rounding).
-// Accuracy: the operand rounding is 2^-(b+1) of the row max (b = 56 for N = 16, K = 2048), i.e.
-// the product error is <= K 2^-(b+1) (max_k|a_ik| max_k|b_jk|) — FP64-GEMM level (K 2^-53 sum|a||b|).
-// N = 16 GEMMs per tile product (an 8-slice Ozaki split needs 36).
+// Product: X_ij = sum_k x'_ik y'_jk is an integer with |X| <= K 2^{2b} <= 0.3 M, M = prod p_t, so it
+// is fixed by its residues.  Per modulus one INT8 GEMM (kind::i8, exact INT32 accumulation in TMEM:
+// |acc| <= K 128^2 = 2^25) gives acc_t == X (mod p_t).  The epilogue reduces the first modulus a of
+// each pair to r_a (exact Barrett), combines it with the second modulus b by Shoup's modular
+// multiplication into the pair residue R_j = r_a + a ((acc_b - r_a) a^-1 mod b) in [0, ab), and, once
+// all pairs are known, reconstructs
+//     X = sum_j R_j w_j  -  q M,   w_j = (M/m_j) ((M/m_j)^-1 mod m_j)
+// with integer + FP32 arithmetic only (crt_recon_bits, crt.h: FP32 quotient estimate, 96-bit limb
+// sums, the FP64 bit pattern of X 2^{e_i + f_j - 2b} assembled by count-leading-zeros) — the FP64
+// pipe runs ~25x slower while the tensor core is busy.  C_ij -= that value by TMA
+// reduce-add.  Accuracy: the operand rounding is 2^-(b+1) of the row max (b = 56 for N = 16,
+// K = 2048), i.e. the product error is <= K 2^-(b+1) (max_k|a_ik| max_k|b_jk|) — FP64-GEMM level
+// (K 2^-53 sum|a||b|); the reconstruction adds < 2^51.6 absolute on X (2^-15 of that bound) and one
+// rounding to 53 bits.  N = 16 GEMMs per tile product (an 8-slice Ozaki split needs 36).
 //
 // Kernel: persistent CTA pairs (cluster of 2 on a TPC, tcgen05.mma.cta_group::2, M = 256, N = 256,
-// K = 32 per MMA), 128-byte-swizzled K-major TMA boxes of 128 x 128 int8 per CTA and operand, six
+// K = 32 per MMA), 128-byte-swizzled K-major TMA boxes of 128 x 128 int8 per CTA and operand, five
 // 32 KB stages.  Accumulators: two 256-column TMEM buffers, one per modulus in flight, so the
 // epilogue reduces modulus t while the tensor core computes modulus t+1.
 //   warp 0: TMA producer; warp 1: MMA issuer (leader CTA); warp 2: TMEM allocator;
-//   warps 4-11: epilogue — warp w owns TMEM lanes 32 (w % 4).. (its rows) and one 128-column half;
-//   per modulus it stores the int8 residues of its 32 x 128 block into a per-CTA L2-resident
-//   scratch slot (128 x 256 x N bytes, acquired at launch), and after the last modulus reads them
-//   back (the same threads: program order suffices) and reconstructs + updates C.
+//   warps 4-11 (CRT_EPI = 8; 16 also builds): epilogue — warp w owns TMEM lanes 32 (w % 4).. (its rows)
+//   and one column part; per moduli pair it stores the uint16 pair residues into a per-CTA scratch of
+//   recycled 2 KB blocks and reconstructs the previous tile group by group in between (see the epilogue).
 #include <cudaTypedefs.h>
 #include <math.h>
 #include <stdint.h>
