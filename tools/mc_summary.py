@@ -11,9 +11,9 @@ import numpy as np
 
 
 def main():
-    print("| beta | nu | replicas (FP64 too) | mean theta_MP (sigma^2, beta, nu) | std | bias vs theta_true | "
-          "max abs(theta_MP - theta_FP64) | s / replica |")
-    print("|---|---|---|---|---|---|---|---|")
+    print("| beta | nu | maxfev | replicas (FP64 too) | converged (MP / FP64) | mean theta_MP (sigma^2, beta, nu) | std | "
+          "bias vs theta_true | max abs(theta_MP - theta_FP64) | s / replica |")
+    print("|---|---|---|---|---|---|---|---|---|---|")
     for path in sys.argv[1:]:
         d = json.load(open(path))
         reps = d.get("reps") or d.get("partial") or []
@@ -25,7 +25,10 @@ def main():
         sec = np.mean([q.get("seconds", float("nan")) for q in reps])
         fmt = lambda v: "(" + ", ".join(f"{x:.4f}" for x in v) + ")"  # noqa: E731
         beta, nu = (th[1], th[2]) if len(th) == 3 else ("?", "?")
-        print(f"| {beta} | {nu} | {len(reps)} ({len(d64)}) | {fmt(amp.mean(0))} | {fmt(amp.std(0))} | "
+        mf = d.get("maxfev", "?")
+        cm = sum(1 for q in reps if q.get("nfev_mp", 0) < (mf if isinstance(mf, int) else 10**9))
+        c64 = sum(1 for q in reps if "nfev_fp64" in q and q["nfev_fp64"] < (mf if isinstance(mf, int) else 10**9))
+        print(f"| {beta} | {nu} | {mf} | {len(reps)} ({len(d64)}) | {cm} / {c64} | {fmt(amp.mean(0))} | {fmt(amp.std(0))} | "
               f"{fmt(amp.mean(0) - th)} | {max(d64) if d64 else float('nan'):.2e} | {sec:.0f} |")
 
 

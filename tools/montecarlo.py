@@ -46,16 +46,17 @@ def main():
         ev.M.gp_sample(de, dz)
         t0 = time.time()
         fmp = fit(ev, dx, dy, dz, mode=mp.MP_MAP_ADAPTIVE, u_req=u_req, maxfev=maxfev)
-        rec = {"replica": r, "mp": list(fmp.theta), "nfev_mp": fmp.nfev}
+        rec = {"replica": r, "mp": list(fmp.theta), "nfev_mp": fmp.nfev, "converged_mp": fmp.nfev < maxfev,
+               "loglik_mp": fmp.loglik}
         if r < n64:
             f64 = fit(ev, dx, dy, dz, mode=mp.MP_MAP_FP64, maxfev=maxfev)
             rec.update({"fp64": list(f64.theta), "max_abs_dtheta": float(np.max(np.abs(fmp.theta - f64.theta))),
-                        "nfev_fp64": f64.nfev})
+                        "nfev_fp64": f64.nfev, "converged_fp64": f64.nfev < maxfev, "loglik_fp64": f64.loglik})
         rec["seconds"] = time.time() - t0
         print(json.dumps(rec), flush=True)
         reps.append(rec)
         json.dump({"partial": reps, "theta_true": theta_true, "n": n, "u_req": u_req, "maxfev": maxfev},
-                  open(f"gpurun_out/montecarlo_n{n}_R{R}_b{beta}_nu{nu}.json", "w"), indent=1)
+                  open(f"gpurun_out/montecarlo_n{n}_R{R}_b{beta}_nu{nu}_f{maxfev}.json", "w"), indent=1)
     a64 = np.array([q["fp64"] for q in reps if "fp64" in q])
     amp = np.array([q["mp"] for q in reps])
     out = {"n": n, "nb": nb, "replicas": R, "fp64_replicas": len(a64), "u_req": u_req, "theta_true": theta_true,
@@ -63,7 +64,7 @@ def main():
            "fp64_mean": a64.mean(0).tolist() if len(a64) else None, "fp64_std": a64.std(0).tolist() if len(a64) else None,
            "max_abs_dtheta": float(max(q["max_abs_dtheta"] for q in reps if "max_abs_dtheta" in q)) if len(a64) else None}
     print(json.dumps(out))
-    json.dump(out, open(f"gpurun_out/montecarlo_n{n}_R{R}_b{beta}_nu{nu}.json", "w"), indent=1)
+    json.dump(out, open(f"gpurun_out/montecarlo_n{n}_R{R}_b{beta}_nu{nu}_f{maxfev}.json", "w"), indent=1)
 
 
 if __name__ == "__main__":
