@@ -8,7 +8,7 @@ cd "$(dirname "$0")/.."
 mkdir -p gpurun_out
 for b in ${1:-0.03 0.3}; do
   for nu in ${2:-0.5 1.0}; do
-    timeout 3000 python tools/montecarlo.py 40000 ${3:-20} 1e-9 $b $nu ${4:-3} ${5:-200} > gpurun_out/mc_b${b}_nu${nu}_f${5:-200}.log 2>&1
+    timeout ${MC_TIMEOUT:-3000} python tools/montecarlo.py 40000 ${3:-20} 1e-9 $b $nu ${4:-3} ${5:-200} > gpurun_out/mc_b${b}_nu${nu}_f${5:-200}.log 2>&1
     echo "beta=$b nu=$nu rc=$? $(tail -c 400 gpurun_out/mc_b${b}_nu${nu}_f${5:-200}.log | tr '\n' ' ' | cut -c1-300)"
   done
 done
