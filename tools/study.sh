@@ -38,6 +38,7 @@ case $1 in
     run c2_adaptive4_v3 --config c2 --map adaptive4
     run c5_rp3_v3 --config c5 --engine reserve_pairs=3
     run c5_rp9_v3 --config c5 --engine reserve_pairs=9
+    python tools/mc_check.py profiles/r02/mc/montecarlo_n40000_R8_b0.03_nu1.0_f1000.json 0 > gpurun_out/mc_check.log 2>&1; tail -1 gpurun_out/mc_check.log
     bash tools/sanitize.sh ;;
   sens)
     run c3_ureq1e-8 --config c3 --u-req 1e-8
