@@ -284,8 +284,11 @@ mp_status mp_precision_map4(int nt, const double* tile_sqnorm, double u_req, con
  * converted once per panel on the consuming GPU to the successor's operand format;
  * DSYRK and FP64-class GEMMs on the handle's FP64 engine (default: CRT on INT8 tcgen05, see
  * mp_config), FP32-class GEMMs as 3xFP16 (default) or 3xTF32 on tcgen05, FP16-class GEMMs as
- * row-scaled FP16 x FP16 -> FP32 on tcgen05, accumulating into the FP32 tile.
- * kernel_prec / comm_prec: host maps (NT*NT, as produced by mp_precision_map
+ * row-scaled FP16 x FP16 -> FP32 on tcgen05, accumulating into the FP32 tile;
+ * pure-FP16 tiles (MP_FP16H, four-level maps) as row-scaled FP16 x FP16 with an F16 TMEM accumulator,
+ * widened and added into the FP32 tile — these need a matrix laid out for a four-level map (mp_eval
+ * with MP_MAP_ADAPTIVE4 / MP_MAP_USER), else MP_ERR_UNSUPPORTED.
+ * kernel_prec / comm_prec: host maps (NT*NT, as produced by mp_precision_map / mp_precision_map4
  * and consistent with the storage map A is bound with).  Blocking.
  * *info = 0 on success, else the 1-based global column of the first
  * non-positive pivot (LAPACK convention) and MP_ERR_NOT_SPD is returned. */
