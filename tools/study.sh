@@ -40,6 +40,8 @@ case $1 in
     run c5_rp9_v3 --config c5 --engine reserve_pairs=9
     python tools/mc_check.py profiles/r02/mc/montecarlo_n40000_R8_b0.03_nu1.0_f1000.json 0 > gpurun_out/mc_check.log 2>&1; tail -1 gpurun_out/mc_check.log
     bash tools/sanitize.sh ;;
+  rp)  # reserve_pairs sweep at C5 on one box (CTA pairs the persistent CRT grid leaves to the panel stream)
+    for r in 6 3 2 4 0; do run c5_rp${r}_sweep --config c5 --engine reserve_pairs=$r; done ;;
   sens)
     run c3_ureq1e-8 --config c3 --u-req 1e-8
     run c3_nu1 --config c3 --theta 1,0.03,1.0
