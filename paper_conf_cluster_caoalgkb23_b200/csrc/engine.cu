@@ -327,7 +327,7 @@ extern "C" {
 
 const char* mp_version(void) {
     return "mpgeo 0.2 sm_100a (FP64 class: CRT INT8 tcgen05 | DMMA; FP32 class: 3xFP16 | 3xTF32 tcgen05 | DMMA; "
-           "FP16 class: row-scaled f16 tcgen05 | DMMA)";
+           "FP16 class: row-scaled f16 tcgen05 | DMMA; four-level pure FP16: f16-accumulator tcgen05)";
 }
 
 void mp_config_default(mp_config* c) {
